@@ -1,0 +1,92 @@
+"""The five BASELINE.json configs as concrete, seeded, synthetic workloads.
+
+    c1  10k uniform points on [0,1024)^2 x 16 convex/concave polygons (overlaps, holes)   COUNT
+    c2  100M taxi-like points x 1 star query polygon (1,000 vertices, bbox 0.3 x domain) SELECT
+    c3  1B taxi-like points x 260 neighbourhood-like tiling polygons (~540 v)            COUNT
+    c4  1B taxi-like points x ~2,200 census-like tiling polygons with island holes        PAIRS
+    c5  8B points (1B per GPU) x 40k zip-code-like tiling polygons (~1.5k v)             COUNT
+
+Sizes/shapes follow PAPER.md Table 1 (Taxi 1.22B points, Neighborhoods 195 polygons /
+538 v avg, Census 2,165 / 72 v, Zip 32,657 / 1,547 v) and the query polygons of P:358 (739 v avg).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import numpy as np
+
+from . import DOMAIN, SgParams, taxi_params, uniform_params
+from . import polygons as pg
+
+
+@dataclass
+class Workload:
+    name: str
+    op: str                    # "count" | "select" | "pairs"
+    points: SgParams
+    point_seed: int
+    n_points: int              # per GPU for the sharded configs
+    polys: dict = field(repr=False)
+    max_dim: int = 4096        # canvas resolution parameter (C5 reading of DESIGN.md)
+    desc: str = ""
+
+
+def c1(n_points: int = 10_000) -> Workload:
+    return Workload("c1_uniform10k_x16poly_1k", "count", uniform_params(0, 0, 1024, 1024), 101, n_points,
+                    pg.c1_polygons(102), max_dim=1024,
+                    desc="10k uniform points x 16 convex/concave polygons on a 1k x 1k int grid, COUNT")
+
+
+def c1_edge_points(polys) -> np.ndarray:
+    """Test-mode extra points for config 1: every polygon vertex, plus every lattice point on an
+    axis-parallel edge and every exact edge midpoint (points exactly on the boundary)."""
+    xy = polys["ring_xy"].astype(np.int64)
+    ro = polys["ring_off"]
+    pts = [xy]
+    for r in range(len(ro) - 1):
+        ring = xy[ro[r]:ro[r + 1]]
+        nxt = np.roll(ring, -1, axis=0)
+        for a, b in zip(ring.tolist(), nxt.tolist()):
+            if a[0] == b[0]:
+                lo, hi = sorted((a[1], b[1]))
+                ys = np.arange(lo, hi + 1)
+                pts.append(np.stack([np.full_like(ys, a[0]), ys], 1))
+            elif a[1] == b[1]:
+                lo, hi = sorted((a[0], b[0]))
+                xs = np.arange(lo, hi + 1)
+                pts.append(np.stack([xs, np.full_like(xs, a[1])], 1))
+            if (a[0] + b[0]) % 2 == 0 and (a[1] + b[1]) % 2 == 0:
+                pts.append(np.array([[(a[0] + b[0]) // 2, (a[1] + b[1]) // 2]]))
+    return np.concatenate(pts).astype(np.int32)
+
+
+def c2(n_points: int = 100_000_000) -> Workload:
+    tp = taxi_params(201)
+    rng = np.random.default_rng(202)
+    r = 0.15 * DOMAIN
+    cx = min(max(tp.cx[0], r), DOMAIN - r)
+    cy = min(max(tp.cy[0], r), DOMAIN - r)
+    poly = pg.assemble([[pg.star(rng, 1000, cx, cy, r, r, rmin=0.35, smooth=0.01)]])
+    return Workload("c2_taxi100M_select_star1000", "select", tp, 201, n_points, poly, max_dim=4096,
+                    desc="spatial selection: 100M clustered taxi-like points inside 1 query polygon (1,000 v)")
+
+
+def c3(n_points: int = 1_000_000_000) -> Workload:
+    return Workload("c3_taxi1B_x260_neighborhoods_count", "count", taxi_params(301), 301, n_points,
+                    pg.jittered_tiling(20, 13, 135, seed=302), max_dim=4096,
+                    desc="point-polygon join COUNT: 1B taxi-like points x 260 neighborhood-like polygons")
+
+
+def c4(n_points: int = 1_000_000_000) -> Workload:
+    return Workload("c4_taxi1B_x2200_census_pairs", "pairs", taxi_params(401), 401, n_points,
+                    pg.jittered_tiling(50, 42, 18, n_islands=100, seed=402), max_dim=8192,
+                    desc="point-polygon join pairs: 1B points x 2,200 census-tract-like polygons with holes")
+
+
+def c5(n_points_per_gpu: int = 1_000_000_000) -> Workload:
+    return Workload("c5_taxi1Bpergpu_x40k_zip_count", "count", taxi_params(501), 501, n_points_per_gpu,
+                    pg.jittered_tiling(200, 200, 375, seed=502), max_dim=8192,
+                    desc="scale-out join COUNT: 1B points per GPU x 40k zip-code-like polygons")
+
+
+ALL = {"c1": c1, "c2": c2, "c3": c3, "c4": c4, "c5": c5}

@@ -1,0 +1,126 @@
+"""CPU oracle for the SPADE point-in-polygon join — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import this package.  The product path
+(``paper_conf_icde_doraiswamyf22_b200``) never imports it and shares no code with it.
+
+The arithmetic lives in ``spade_oracle.c`` (brute force over every (point, polygon) pair,
+half-open even-odd rule, ``__int128`` cross products); see its header for the definition and
+the PAPER.md passages it follows.  This module
+is argument marshalling (numpy -> ctypes) only.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile spade_oracle.c into liboracle.so (plain gcc, -O2, pthreads)."""
+    src = os.path.join(_HERE, "spade_oracle.c")
+    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(src):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-pthread", "-o", _LIB_PATH, src])
+    return _LIB_PATH
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_LIB_PATH)
+        P = ctypes.c_void_p
+        i64, i32 = ctypes.c_int64, ctypes.c_int32
+        lib.oracle_point_in_polygon.argtypes = [i64, i64, P, P, i64, i64]
+        lib.oracle_point_in_polygon.restype = ctypes.c_int
+        lib.oracle_join_count.argtypes = [P, i64, P, P, P, i32, P, ctypes.c_int]
+        lib.oracle_join_count.restype = ctypes.c_int
+        lib.oracle_join_pairs.argtypes = [P, i64, i64, P, P, P, i32, P, P, i64, ctypes.c_int]
+        lib.oracle_join_pairs.restype = i64
+        lib.oracle_select.argtypes = [P, i64, i64, P, P, P, i32, P, i64, ctypes.c_int]
+        lib.oracle_select.restype = i64
+        _lib = lib
+    return _lib
+
+
+def default_threads() -> int:
+    return len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+
+
+def _polys(polys):
+    ring_xy = np.ascontiguousarray(polys["ring_xy"], dtype=np.int32).reshape(-1, 2)
+    ring_off = np.ascontiguousarray(polys["ring_off"], dtype=np.int64)
+    poly_ring_off = np.ascontiguousarray(polys["poly_ring_off"], dtype=np.int64)
+    return ring_xy, ring_off, poly_ring_off, len(poly_ring_off) - 1
+
+
+def _ptr(a):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def point_in_polygon(px: int, py: int, polys, p: int) -> bool:
+    """inside(point, polygon p) under the half-open even-odd rule."""
+    lib = _load()
+    ring_xy, ring_off, poly_ring_off, _ = _polys(polys)
+    return bool(lib.oracle_point_in_polygon(int(px), int(py), _ptr(ring_xy), _ptr(ring_off),
+                                            int(poly_ring_off[p]), int(poly_ring_off[p + 1])))
+
+
+def join_count(xy, polys, nthreads: int | None = None) -> np.ndarray:
+    """int64[P] per-polygon counts."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    ring_xy, ring_off, poly_ring_off, P = _polys(polys)
+    counts = np.zeros(max(P, 1), dtype=np.int64)
+    rc = lib.oracle_join_count(_ptr(xy), len(xy), _ptr(ring_xy), _ptr(ring_off), _ptr(poly_ring_off), P,
+                               _ptr(counts), nthreads or default_threads())
+    if rc != 0:
+        raise MemoryError("oracle_join_count failed")
+    return counts[:P]
+
+
+def join_pairs(xy, polys, point_id_base: int = 0, nthreads: int | None = None):
+    """(point_ids int64[M], poly_ids int32[M]) sorted by (point, polygon)."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    ring_xy, ring_off, poly_ring_off, P = _polys(polys)
+    nt = nthreads or default_threads()
+    total = lib.oracle_join_pairs(_ptr(xy), len(xy), point_id_base, _ptr(ring_xy), _ptr(ring_off),
+                                  _ptr(poly_ring_off), P, None, None, 0, nt)
+    if total < 0:
+        raise MemoryError("oracle_join_pairs failed")
+    pt = np.empty(max(total, 1), dtype=np.int64)
+    pl = np.empty(max(total, 1), dtype=np.int32)
+    lib.oracle_join_pairs(_ptr(xy), len(xy), point_id_base, _ptr(ring_xy), _ptr(ring_off),
+                          _ptr(poly_ring_off), P, _ptr(pt), _ptr(pl), total, nt)
+    return pt[:total], pl[:total]
+
+
+def select(xy, polys, point_id_base: int = 0, nthreads: int | None = None) -> np.ndarray:
+    """int64 ids of points inside at least one polygon, ascending."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    ring_xy, ring_off, poly_ring_off, P = _polys(polys)
+    nt = nthreads or default_threads()
+    out = np.empty(max(len(xy), 1), dtype=np.int64)
+    total = lib.oracle_select(_ptr(xy), len(xy), point_id_base, _ptr(ring_xy), _ptr(ring_off),
+                              _ptr(poly_ring_off), P, _ptr(out), len(out), nt)
+    if total < 0:
+        raise MemoryError("oracle_select failed")
+    return out[:total]
+
+
+def labels_at(xy, polys, nthreads: int | None = None):
+    """For each point, the sorted list of polygons containing it (via join_pairs)."""
+    pt, pl = join_pairs(xy, polys, 0, nthreads)
+    n = len(np.asarray(xy).reshape(-1, 2))
+    out = [[] for _ in range(n)]
+    for a, b in zip(pt.tolist(), pl.tolist()):
+        out[a].append(b)
+    return out
