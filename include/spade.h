@@ -1,0 +1,136 @@
+/*
+ * spade.h — C ABI of the B200-native SPADE point-in-polygon join (paper_conf_icde_doraiswamyf22_b200).
+ *
+ * The method (Doraiswamy & Freire, "GPU-Powered Spatial Database Engine for Commodity Hardware",
+ * ICDE'22; citations are /root/reference/PAPER.md line numbers "P:n"):
+ *   polygons are rasterised into a DISCRETE CANVAS whose pixels hold either the owning polygon or a
+ *   pointer into a BOUNDARY INDEX (Sec. 4.1; Sec. 4.3); points are looked up in
+ *   that canvas and only points on boundary pixels get an exact test (Sec. 5.1-5.2).
+ *   Here the boundary index maps a run of boundary pixels to the exact list of edges touching it
+ *   plus the polygon set just right of the run, so results are EXACT.
+ *
+ * Results are defined by the half-open even-odd rule (reading C1): point (px,py) is in
+ * polygon p iff the number of edges (a,b) over all rings of p with (a.y>py) != (b.y>py) whose
+ * crossing with the line y=py lies strictly right of px is odd.  All arithmetic is exact integer.
+ *
+ * Conventions for every entry point:
+ *   - array arguments are DEVICE pointers (cudaMalloc / torch CUDA tensors) unless the name ends
+ *     in _host; all work is enqueued on `stream` (a cudaStream_t, e.g. torch's current stream);
+ *   - coordinates are int32 fixed point; points are int32 (x, y) pairs interleaved, N x 8 bytes,
+ *     any 8-byte alignment (32-byte alignment is fastest);
+ *   - point ids are int64: point_id_base + index of the point in the call's array;
+ *   - polygon ids are the index 0..P-1 of the polygon in the canvas's input;
+ *   - the return value is a status code (SPADE_OK or a negative SPADE_ERR_*); nothing throws
+ *     across the ABI; spade_last_error() gives a thread-local detail message;
+ *   - no host<->device synchronisation unless stated.
+ * The library owns the canvas and its device memory; the caller owns every other buffer.
+ */
+#ifndef SPADE_H
+#define SPADE_H
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define SPADE_API __attribute__((visibility("default")))
+#else
+#define SPADE_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct spade_canvas spade_canvas;   /* opaque; owns its device memory */
+typedef struct CUstream_st* spade_stream_t;  /* == cudaStream_t (NULL = legacy default stream) */
+
+enum {
+    SPADE_OK = 0,
+    SPADE_ERR_INVALID_ARG = -1,  /* null pointer, negative size, malformed offsets        */
+    SPADE_ERR_COORD_RANGE = -2,  /* a polygon vertex outside [-2^30, 2^30)                 */
+    SPADE_ERR_CAPACITY = -3,     /* output capacity too small; *n_out = required count     */
+    SPADE_ERR_CUDA = -4,         /* a CUDA runtime error (detail in spade_last_error)      */
+    SPADE_ERR_OOM = -5,          /* device or host allocation failed                       */
+    SPADE_ERR_INTERNAL = -6      /* an internal consistency check failed (a bug)           */
+};
+
+/* Canvas resolution (reading C5; the paper fixes no resolution for constraint
+ * canvases).  Pixel = 2^log2_pixel grid units.  log2_pixel = -1 selects the smallest s with
+ * max(W, H) <= max_dim, where W = ((maxx-minx) >> s) + 1 over the polygon extent.  Results do
+ * not depend on the resolution; only speed and memory do. */
+typedef struct {
+    int32_t log2_pixel;   /* -1 = auto                                    */
+    int32_t max_dim;      /* used when log2_pixel == -1; 0 means 4096     */
+} spade_canvas_params;
+
+/* Build the discrete canvas + boundary index for a polygon set (P:113-123 canvas creation,
+ * Sec. 4.2; P:146 and P:268 boundary index, Sec. 4.3 / 5.5).
+ *   ring_xy       [V*2]  int32 vertex coordinates (x,y) of all rings, each ring implicitly closed
+ *                        (last vertex connects to first); every coordinate in [-2^30, 2^30)
+ *   ring_off      [R+1]  int64: ring r = vertices [ring_off[r], ring_off[r+1]); ring_off[0] = 0
+ *   poly_ring_off [P+1]  int64: polygon p = rings [poly_ring_off[p], poly_ring_off[p+1]);
+ *                        poly_ring_off[0] = 0, poly_ring_off[P] = R.  Polygons may have holes,
+ *                        several outer rings, self-intersections and degenerate rings
+ *                        (even-odd over all rings, reading C2); polygons may overlap (C3).
+ *   num_polys     P >= 0
+ *   prm           NULL = defaults {-1, 4096}
+ *   out           receives the canvas handle (NULL on error)
+ * The input buffers may be freed once this returns.  Synchronises `stream` (a few times: sizes
+ * are data dependent).  Errors: INVALID_ARG, COORD_RANGE, OOM, CUDA. */
+SPADE_API int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off,
+                       int32_t num_polys, const spade_canvas_params* prm, spade_stream_t stream,
+                       spade_canvas** out);
+
+/* Release a canvas (NULL is a no-op).  Synchronises the device. */
+SPADE_API void spade_canvas_free(spade_canvas* c);
+
+/* Canvas statistics for reports: fine canvas W x H at 2^log2_pixel units per pixel; coarse
+ * (shared-memory) tile grid Wc x Hc of 2^log2_tile fine pixels per side; number of boundary
+ * runs (+ multi-owner records) and of listed run edges; fraction of coarse tiles that are mixed.
+ * Any output pointer may be NULL. */
+SPADE_API int spade_canvas_info(const spade_canvas* c, int32_t* W, int32_t* H, int32_t* log2_pixel,
+                      int32_t* Wc, int32_t* Hc, int32_t* log2_tile,
+                      int64_t* num_runs, int64_t* num_run_edges, double* mixed_tile_frac);
+
+/* Aggregation: per-polygon COUNT of the points of xy[0..n) inside each polygon (P:214,
+ * Sec. 5.2, "aggregation plan 2" for points: partial aggregates without materialising the join).
+ *   xy      [n*2] int32 device points
+ *   counts  [P]   int64 device counts, ACCUMULATED INTO (the caller zeroes them)
+ * Asynchronous (no host sync).  n == 0 is a no-op.  Errors: INVALID_ARG, CUDA. */
+SPADE_API int spade_join_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts,
+                     spade_stream_t stream);
+
+/* Selection (Sec. 5.2): ids of the points inside AT LEAST ONE polygon of the canvas
+ * (a 1-polygon canvas is the paper's polygonal selection), each id once, order unspecified.
+ *   out_ids   [capacity] int64 device
+ *   n_out     HOST int64: number of selected points
+ * Map with n_max = n is the paper's 1-pass Map: capacity >= n always suffices.
+ * If capacity < needed: returns SPADE_ERR_CAPACITY with *n_out = needed, out_ids unspecified;
+ * call again with a larger buffer (the paper's 2-pass Map).  Synchronises `stream`. */
+SPADE_API int spade_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t point_id_base,
+                 int64_t* out_ids, int64_t capacity, int64_t* n_out, spade_stream_t stream);
+
+/* Join (pair form P:208): all (point_id, polygon_id) with the point inside the
+ * polygon, as two device arrays (SoA), order unspecified.  n_max = n when polygons do not
+ * overlap.  Capacity protocol and synchronisation as spade_select. */
+SPADE_API int spade_join_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t point_id_base,
+                     int64_t* out_point_ids, int32_t* out_poly_ids, int64_t capacity,
+                     int64_t* n_out, spade_stream_t stream);
+
+/* End-to-end COUNT from HOST memory: streams xy_host[0..n) to the device in chunks (copies
+ * overlapped with the probe on two internal streams; pinned memory gives full PCIe bandwidth),
+ * and ACCUMULATES the int64 counts into counts_host[P].  Synchronises `stream` before return.
+ * This is the user-facing call for point sets that live on the host (the
+ * paper's times are dominated by exactly this host->GPU transfer). */
+SPADE_API int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t n,
+                          int64_t* counts_host, spade_stream_t stream);
+
+/* Number of kernels this library has launched in this process (for the bench's gpu_launches). */
+SPADE_API int64_t spade_launch_count(void);
+
+SPADE_API const char* spade_status_string(int code);
+SPADE_API const char* spade_last_error(void);   /* thread-local detail message of the last failure */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPADE_H */

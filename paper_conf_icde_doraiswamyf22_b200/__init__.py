@@ -1,0 +1,237 @@
+"""paper_conf_icde_doraiswamyf22_b200 — B200-native SPADE point-in-polygon join (thin binding).
+
+Argument marshalling only: every step of the path runs in libspade.so (CUDA kernels for sm_100a
+behind the C ABI of include/spade.h).  PyTorch supplies device memory and streams.  There is no
+CPU fallback: if the extension cannot be loaded, or no CUDA device is present, calls raise.
+
+    canvas = Canvas(polys)                       # spade_build_canvas   (Sec. 4.2-4.3)
+    counts = join_count(canvas, xy)              # spade_join_count     (aggregation)
+    ids    = select(canvas, xy)                  # spade_select         (selection)
+    pt, pl = join_pairs(canvas, xy)              # spade_join_pairs     (join)
+    counts = join_count_host(canvas, xy_numpy)   # spade_join_count_host (host-resident points)
+
+`polys` is a dict with ``ring_xy`` (V,2) int32, ``ring_off`` (R+1) int64, ``poly_ring_off``
+(P+1) int64 (numpy arrays or torch tensors), the layout spade_build_canvas takes.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libspade.so")
+_lib = None
+
+SPADE_OK, SPADE_ERR_INVALID_ARG, SPADE_ERR_COORD_RANGE = 0, -1, -2
+SPADE_ERR_CAPACITY, SPADE_ERR_CUDA, SPADE_ERR_OOM, SPADE_ERR_INTERNAL = -3, -4, -5, -6
+
+
+class SpadeError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"spade error {code}: {msg}")
+        self.code = code
+
+
+class CapacityError(SpadeError):
+    def __init__(self, code, msg, needed):
+        super().__init__(code, msg)
+        self.needed = needed
+
+
+class CanvasParams(ctypes.Structure):
+    _fields_ = [("log2_pixel", ctypes.c_int32), ("max_dim", ctypes.c_int32)]
+
+
+def load(path: str | None = None):
+    """Load libspade.so (build it first with __graft_entry__.build()); raises if missing."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    p = path or LIB_PATH
+    if not os.path.exists(p):
+        raise ImportError(f"libspade.so not built ({p}); run `python -c 'import __graft_entry__ as g; g.build()'`")
+    lib = ctypes.CDLL(p)
+    P, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+    lib.spade_build_canvas.argtypes = [P, P, P, i32, ctypes.POINTER(CanvasParams), P, ctypes.POINTER(P)]
+    lib.spade_build_canvas.restype = ctypes.c_int
+    lib.spade_canvas_free.argtypes = [P]
+    lib.spade_canvas_free.restype = None
+    lib.spade_canvas_info.argtypes = [P] + [ctypes.POINTER(i32)] * 6 + [ctypes.POINTER(i64)] * 2 + [ctypes.POINTER(ctypes.c_double)]
+    lib.spade_canvas_info.restype = ctypes.c_int
+    lib.spade_join_count.argtypes = [P, P, i64, P, P]
+    lib.spade_join_count.restype = ctypes.c_int
+    lib.spade_select.argtypes = [P, P, i64, i64, P, i64, ctypes.POINTER(i64), P]
+    lib.spade_select.restype = ctypes.c_int
+    lib.spade_join_pairs.argtypes = [P, P, i64, i64, P, P, i64, ctypes.POINTER(i64), P]
+    lib.spade_join_pairs.restype = ctypes.c_int
+    lib.spade_join_count_host.argtypes = [P, P, i64, P, P]
+    lib.spade_join_count_host.restype = ctypes.c_int
+    lib.spade_launch_count.argtypes = []
+    lib.spade_launch_count.restype = i64
+    lib.spade_status_string.argtypes = [ctypes.c_int]
+    lib.spade_status_string.restype = ctypes.c_char_p
+    lib.spade_last_error.argtypes = []
+    lib.spade_last_error.restype = ctypes.c_char_p
+    _lib = lib
+    return lib
+
+
+EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_canvas_free", "spade_canvas_info", "spade_join_count",
+                    "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_launch_count",
+                    "spade_status_string", "spade_last_error"]
+
+
+def _check(rc: int, what: str):
+    if rc != SPADE_OK:
+        lib = load()
+        raise SpadeError(rc, f"{what}: {lib.spade_last_error().decode()}")
+
+
+def _torch():
+    import torch
+    if not torch.cuda.is_available():
+        raise RuntimeError("paper_conf_icde_doraiswamyf22_b200 needs a CUDA device (no CPU fallback)")
+    return torch
+
+
+def _stream(stream):
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _dev(a, dtype, shape_last=None):
+    """numpy array / torch tensor -> contiguous CUDA tensor of dtype."""
+    torch = _torch()
+    t = torch.as_tensor(a) if not isinstance(a, torch.Tensor) else a
+    t = t.to(device="cuda", dtype=dtype).contiguous()
+    if shape_last is not None:
+        t = t.reshape(-1, shape_last)
+    return t
+
+
+def launch_count() -> int:
+    return int(load().spade_launch_count())
+
+
+class Canvas:
+    """Discrete canvas + boundary index of a polygon set (owns device memory)."""
+
+    def __init__(self, polys, log2_pixel: int = -1, max_dim: int = 4096, stream=None):
+        torch = _torch()
+        lib = load()
+        ring_xy = _dev(polys["ring_xy"], torch.int32, 2)
+        ring_off = _dev(polys["ring_off"], torch.int64)
+        poly_ring_off = _dev(polys["poly_ring_off"], torch.int64)
+        self.num_polys = int(poly_ring_off.numel()) - 1
+        prm = CanvasParams(log2_pixel, max_dim)
+        h = ctypes.c_void_p()
+        rc = lib.spade_build_canvas(ctypes.c_void_p(ring_xy.data_ptr()), ctypes.c_void_p(ring_off.data_ptr()),
+                                    ctypes.c_void_p(poly_ring_off.data_ptr()), self.num_polys, ctypes.byref(prm),
+                                    _stream(stream), ctypes.byref(h))
+        _check(rc, "spade_build_canvas")
+        self._h = h
+        self._lib = lib
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self) -> dict:
+        i32 = [ctypes.c_int32() for _ in range(6)]
+        i64 = [ctypes.c_int64() for _ in range(2)]
+        d = ctypes.c_double()
+        _check(self._lib.spade_canvas_info(self._h, *[ctypes.byref(x) for x in i32],
+                                           *[ctypes.byref(x) for x in i64], ctypes.byref(d)), "spade_canvas_info")
+        W, H, s, Wc, Hc, b = (x.value for x in i32)
+        return {"W": W, "H": H, "log2_pixel": s, "Wc": Wc, "Hc": Hc, "log2_tile": b,
+                "num_records": i64[0].value, "num_run_edges": i64[1].value, "mixed_tile_frac": d.value}
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.spade_canvas_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def _points(xy):
+    torch = _torch()
+    if not (isinstance(xy, torch.Tensor) and xy.is_cuda and xy.dtype == torch.int32 and xy.is_contiguous()):
+        xy = _dev(xy, torch.int32, 2)
+    return xy, xy.numel() // 2
+
+
+def join_count(canvas: Canvas, xy, counts=None, stream=None):
+    """Per-polygon COUNT (int64[P] CUDA tensor); accumulates into `counts` if given."""
+    torch = _torch()
+    xy, n = _points(xy)
+    if counts is None:
+        counts = torch.zeros(canvas.num_polys, dtype=torch.int64, device="cuda")
+    rc = load().spade_join_count(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n,
+                                 ctypes.c_void_p(counts.data_ptr()), _stream(stream))
+    _check(rc, "spade_join_count")
+    return counts
+
+
+def select(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = None, stream=None):
+    """int64 CUDA tensor of the ids of points inside >= 1 polygon (order unspecified).
+    capacity=None uses n_max = n (1-pass Map); a too-small capacity retries once with the
+    reported size (2-pass Map)."""
+    torch = _torch()
+    xy, n = _points(xy)
+    cap = n if capacity is None else capacity
+    for _ in range(2):
+        out = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+        n_out = ctypes.c_int64()
+        rc = load().spade_select(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n, point_id_base,
+                                 ctypes.c_void_p(out.data_ptr()), cap, ctypes.byref(n_out), _stream(stream))
+        if rc == SPADE_ERR_CAPACITY:
+            cap = n_out.value
+            continue
+        _check(rc, "spade_select")
+        return out[: n_out.value]
+    raise SpadeError(SPADE_ERR_CAPACITY, "select: capacity retry failed")
+
+
+def join_pairs(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = None, stream=None):
+    """(point_ids int64, poly_ids int32) CUDA tensors, order unspecified."""
+    torch = _torch()
+    xy, n = _points(xy)
+    cap = n if capacity is None else capacity
+    for _ in range(2):
+        pt = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+        pl = torch.empty(max(cap, 1), dtype=torch.int32, device="cuda")
+        n_out = ctypes.c_int64()
+        rc = load().spade_join_pairs(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n, point_id_base,
+                                     ctypes.c_void_p(pt.data_ptr()), ctypes.c_void_p(pl.data_ptr()), cap,
+                                     ctypes.byref(n_out), _stream(stream))
+        if rc == SPADE_ERR_CAPACITY:
+            cap = n_out.value
+            continue
+        _check(rc, "spade_join_pairs")
+        return pt[: n_out.value], pl[: n_out.value]
+    raise SpadeError(SPADE_ERR_CAPACITY, "join_pairs: capacity retry failed")
+
+
+def join_count_host(canvas: Canvas, xy_host, counts_host=None, stream=None) -> np.ndarray:
+    """COUNT over HOST-resident points (numpy array or pinned CPU tensor); returns int64 numpy."""
+    lib = load()
+    if hasattr(xy_host, "data_ptr"):      # torch CPU tensor (pinned for full bandwidth)
+        assert not xy_host.is_cuda and xy_host.is_contiguous()
+        ptr, n = xy_host.data_ptr(), xy_host.numel() // 2
+    else:
+        xy_host = np.ascontiguousarray(xy_host, dtype=np.int32)
+        ptr, n = xy_host.ctypes.data, xy_host.size // 2
+    if counts_host is None:
+        counts_host = np.zeros(canvas.num_polys, dtype=np.int64)
+    rc = lib.spade_join_count_host(canvas.handle, ctypes.c_void_p(ptr), n,
+                                   counts_host.ctypes.data_as(ctypes.c_void_p), _stream(stream))
+    _check(rc, "spade_join_count_host")
+    return counts_host

@@ -1,0 +1,231 @@
+// spade_api.cu — the C ABI (include/spade.h): argument validation, status codes, thread-local
+// error detail, launch accounting, the capacity protocol of the Map operator (PAPER.md P:167-175:
+// 1-pass Map when n_max fits, else count first and retry) and the host-resident streaming join.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <atomic>
+#include <algorithm>
+#include <vector>
+#include "spade_internal.cuh"
+
+namespace spade {
+
+int build_canvas(const int32_t*, const int64_t*, const int64_t*, int32_t, const spade_canvas_params*, cudaStream_t,
+                 spade_canvas**);
+
+namespace {
+thread_local char g_err[512] = "";
+std::atomic<int64_t> g_launches{0};
+}  // namespace
+
+int set_error(int code, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+  return code;
+}
+
+int check_cuda(cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return SPADE_OK;
+  if (e == cudaErrorMemoryAllocation) return set_error(SPADE_ERR_OOM, "%s: %s", what, cudaGetErrorString(e));
+  return set_error(SPADE_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+void count_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+int device_sm_count() {
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
+  return sms;
+}
+
+static int check_points(const spade_canvas* c, const int32_t* xy, int64_t n, const char* fn) {
+  if (!c) return set_error(SPADE_ERR_INVALID_ARG, "%s: canvas is NULL", fn);
+  if (n < 0) return set_error(SPADE_ERR_INVALID_ARG, "%s: negative n", fn);
+  if (n > 0 && !xy) return set_error(SPADE_ERR_INVALID_ARG, "%s: xy is NULL", fn);
+  if (n > 0 && ((uintptr_t)xy & 7)) return set_error(SPADE_ERR_INVALID_ARG, "%s: xy must be 8-byte aligned", fn);
+  return SPADE_OK;
+}
+
+}  // namespace spade
+
+namespace spade {
+// Map with capacity: one device counter; the kernel writes results below `capacity` and counts
+// all of them; the host reads the total (P:173 1-pass, P:175 2-pass on overflow).
+template <class F>
+int run_with_capacity(int64_t capacity, int64_t* n_out, cudaStream_t st, const char* fn, F launch) {
+  if (!n_out) return set_error(SPADE_ERR_INVALID_ARG, "%s: n_out is NULL", fn);
+  if (capacity < 0) return set_error(SPADE_ERR_INVALID_ARG, "%s: negative capacity", fn);
+  unsigned long long* d_total = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&d_total, sizeof(unsigned long long), st);
+  if (e != cudaSuccess) return check_cuda(e, fn);
+  e = cudaMemsetAsync(d_total, 0, sizeof(unsigned long long), st);
+  int rc = e == cudaSuccess ? launch(d_total) : check_cuda(e, fn);
+  unsigned long long h = 0;
+  if (rc == SPADE_OK) {
+    e = cudaMemcpyAsync(&h, d_total, sizeof(h), cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) rc = check_cuda(e, fn);
+  }
+  cudaFreeAsync(d_total, st);
+  if (rc != SPADE_OK) return rc;
+  *n_out = (int64_t)h;
+  if ((int64_t)h > capacity)
+    return set_error(SPADE_ERR_CAPACITY, "%s: %lld results exceed capacity %lld", fn, (long long)h, (long long)capacity);
+  return SPADE_OK;
+}
+
+}  // namespace spade
+
+using namespace spade;
+
+extern "C" {
+
+int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off,
+                       int32_t num_polys, const spade_canvas_params* prm, spade_stream_t stream, spade_canvas** out) {
+  if (!out) return set_error(SPADE_ERR_INVALID_ARG, "spade_build_canvas: out is NULL");
+  *out = nullptr;
+  return build_canvas(ring_xy, ring_off, poly_ring_off, num_polys, prm, (cudaStream_t)stream, out);
+}
+
+void spade_canvas_free(spade_canvas* c) {
+  if (!c) return;
+  cudaDeviceSynchronize();
+  cudaFree(c->fine); cudaFree(c->coarse); cudaFree(c->runs); cudaFree(c->run_seg); cudaFree(c->run_poly);
+  cudaFree(c->sets); cudaFree(c->set_rng);
+  delete c;
+}
+
+int spade_canvas_info(const spade_canvas* c, int32_t* W, int32_t* H, int32_t* log2_pixel, int32_t* Wc, int32_t* Hc,
+                      int32_t* log2_tile, int64_t* num_runs, int64_t* num_run_edges, double* mixed_tile_frac) {
+  if (!c) return set_error(SPADE_ERR_INVALID_ARG, "spade_canvas_info: canvas is NULL");
+  if (W) *W = c->empty ? 0 : c->d.W;
+  if (H) *H = c->empty ? 0 : c->d.H;
+  if (log2_pixel) *log2_pixel = c->empty ? 0 : c->d.s;
+  if (Wc) *Wc = c->empty ? 0 : c->d.Wc;
+  if (Hc) *Hc = c->empty ? 0 : c->d.Hc;
+  if (log2_tile) *log2_tile = c->empty ? 0 : c->d.b;
+  if (num_runs) *num_runs = c->num_records;
+  if (num_run_edges) *num_run_edges = c->num_run_edges;
+  if (mixed_tile_frac) *mixed_tile_frac = c->mixed_tile_frac;
+  return SPADE_OK;
+}
+
+int spade_join_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts, spade_stream_t stream) {
+  int rc = check_points(c, xy, n, "spade_join_count");
+  if (rc) return rc;
+  if (c->d.num_polys > 0 && !counts) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_count: counts is NULL");
+  return launch_count(c, xy, n, counts, (cudaStream_t)stream);
+}
+
+int spade_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t point_id_base, int64_t* out_ids,
+                 int64_t capacity, int64_t* n_out, spade_stream_t stream) {
+  int rc = check_points(c, xy, n, "spade_select");
+  if (rc) return rc;
+  if (capacity > 0 && !out_ids) return set_error(SPADE_ERR_INVALID_ARG, "spade_select: out_ids is NULL");
+  return run_with_capacity(capacity, n_out, (cudaStream_t)stream, "spade_select", [&](unsigned long long* t) {
+    return launch_select(c, xy, n, point_id_base, out_ids, capacity, t, (cudaStream_t)stream);
+  });
+}
+
+int spade_join_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t point_id_base, int64_t* out_point_ids,
+                     int32_t* out_poly_ids, int64_t capacity, int64_t* n_out, spade_stream_t stream) {
+  int rc = check_points(c, xy, n, "spade_join_pairs");
+  if (rc) return rc;
+  if (capacity > 0 && (!out_point_ids || !out_poly_ids))
+    return set_error(SPADE_ERR_INVALID_ARG, "spade_join_pairs: output arrays are NULL");
+  return run_with_capacity(capacity, n_out, (cudaStream_t)stream, "spade_join_pairs", [&](unsigned long long* t) {
+    return launch_pairs(c, xy, n, point_id_base, out_point_ids, out_poly_ids, capacity, t, (cudaStream_t)stream);
+  });
+}
+
+// Host-resident points: chunks of kChunk points are copied into two device staging buffers on a
+// copy stream while the probe consumes the previous chunk on a compute stream (P:480 proposes
+// exactly this pipelining of I/O with GPU work).
+int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, int64_t* counts_host,
+                          spade_stream_t stream) {
+  int rc = check_points(c, xy_host, n, "spade_join_count_host");
+  if (rc) return rc;
+  const int P = c->d.num_polys;
+  if (P > 0 && !counts_host) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_count_host: counts_host is NULL");
+  if (n == 0 || P == 0) return SPADE_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t kChunk = 1ll << 25;             // 32 Mi points = 256 MiB per staging buffer
+  const int64_t chunk = std::min(kChunk, n);
+  int32_t* stage[2] = {nullptr, nullptr};
+  int64_t* d_counts = nullptr;
+  cudaStream_t cs = nullptr, ks = nullptr;
+  cudaEvent_t copied[2] = {nullptr, nullptr}, consumed[2] = {nullptr, nullptr};
+  cudaError_t e = cudaSuccess;
+  auto cleanup = [&]() {
+    if (ks) cudaStreamSynchronize(ks);
+    if (cs) cudaStreamSynchronize(cs);
+    for (int i = 0; i < 2; ++i) {
+      if (stage[i]) cudaFree(stage[i]);
+      if (copied[i]) cudaEventDestroy(copied[i]);
+      if (consumed[i]) cudaEventDestroy(consumed[i]);
+    }
+    if (d_counts) cudaFree(d_counts);
+    if (cs) cudaStreamDestroy(cs);
+    if (ks) cudaStreamDestroy(ks);
+  };
+#define HTRY(call, what) do { e = (call); if (e != cudaSuccess) { int r_ = check_cuda(e, what); cleanup(); return r_; } } while (0)
+  HTRY(cudaMalloc(&stage[0], chunk * 8), "staging");
+  HTRY(cudaMalloc(&stage[1], chunk * 8), "staging");
+  HTRY(cudaMalloc(&d_counts, sizeof(int64_t) * P), "counts");
+  HTRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking), "stream");
+  HTRY(cudaStreamCreateWithFlags(&ks, cudaStreamNonBlocking), "stream");
+  for (int i = 0; i < 2; ++i) {
+    HTRY(cudaEventCreateWithFlags(&copied[i], cudaEventDisableTiming), "event");
+    HTRY(cudaEventCreateWithFlags(&consumed[i], cudaEventDisableTiming), "event");
+  }
+  // order after prior work on the caller's stream
+  HTRY(cudaEventRecord(consumed[0], st), "event");
+  HTRY(cudaStreamWaitEvent(cs, consumed[0], 0), "wait");
+  HTRY(cudaStreamWaitEvent(ks, consumed[0], 0), "wait");
+  HTRY(cudaMemsetAsync(d_counts, 0, sizeof(int64_t) * P, ks), "memset");
+  int64_t k = 0;
+  for (int64_t off = 0; off < n; off += chunk, ++k) {
+    const int b = (int)(k & 1);
+    const int64_t m = std::min(chunk, n - off);
+    if (k >= 2) HTRY(cudaStreamWaitEvent(cs, consumed[b], 0), "wait");
+    HTRY(cudaMemcpyAsync(stage[b], xy_host + 2 * off, m * 8, cudaMemcpyHostToDevice, cs), "H2D");
+    HTRY(cudaEventRecord(copied[b], cs), "event");
+    HTRY(cudaStreamWaitEvent(ks, copied[b], 0), "wait");
+    rc = launch_count(c, stage[b], m, d_counts, ks);
+    if (rc != SPADE_OK) { cleanup(); return rc; }
+    HTRY(cudaEventRecord(consumed[b], ks), "event");
+  }
+  std::vector<int64_t> h(P);
+  HTRY(cudaMemcpyAsync(h.data(), d_counts, sizeof(int64_t) * P, cudaMemcpyDeviceToHost, ks), "D2H");
+  HTRY(cudaStreamSynchronize(ks), "sync");
+  for (int p = 0; p < P; ++p) counts_host[p] += h[p];
+  // make the caller's stream observe completion
+  HTRY(cudaEventRecord(consumed[0], ks), "event");
+  HTRY(cudaStreamWaitEvent(st, consumed[0], 0), "wait");
+  cleanup();
+  return SPADE_OK;
+#undef HTRY
+}
+
+int64_t spade_launch_count(void) { return g_launches.load(); }
+
+const char* spade_status_string(int code) {
+  switch (code) {
+    case SPADE_OK: return "ok";
+    case SPADE_ERR_INVALID_ARG: return "invalid argument";
+    case SPADE_ERR_COORD_RANGE: return "polygon coordinate outside [-2^30, 2^30)";
+    case SPADE_ERR_CAPACITY: return "output capacity too small";
+    case SPADE_ERR_CUDA: return "CUDA error";
+    case SPADE_ERR_OOM: return "out of memory";
+    case SPADE_ERR_INTERNAL: return "internal error";
+    default: return "unknown status";
+  }
+}
+
+const char* spade_last_error(void) { return g_err; }
+
+}  // extern "C"

@@ -1,0 +1,135 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Bar: bit-exact — counts equal, pair sets equal after sorting, selected id
+sets equal.  All inputs seeded and synthetic.
+"""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from gen import configs
+from gen import polygons as pg
+from tests.helpers import lattice, random_polyset, sorted_pairs
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def spade():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_icde_doraiswamyf22_b200 as sp
+    sp.load()
+    return sp
+
+
+def gpu_all(sp, polys, xy, s=-1, max_dim=4096, base=0):
+    import torch
+    cv = sp.Canvas(polys, log2_pixel=s, max_dim=max_dim)
+    xy_d = torch.as_tensor(np.ascontiguousarray(xy, np.int32)).cuda()
+    counts = sp.join_count(cv, xy_d).cpu().numpy()
+    pt, pl = sp.join_pairs(cv, xy_d, point_id_base=base)
+    ids = sp.select(cv, xy_d, point_id_base=base)
+    torch.cuda.synchronize()
+    return cv, counts, sorted_pairs(pt.cpu().numpy(), pl.cpu().numpy()), np.sort(ids.cpu().numpy())
+
+
+def check_all(sp, polys, xy, s=-1, max_dim=4096, base=0):
+    cv, counts, (pt, pl), ids = gpu_all(sp, polys, xy, s, max_dim, base)
+    ocounts = oracle.join_count(xy, polys)
+    opt, opl = oracle.join_pairs(xy, polys, point_id_base=base)
+    oids = oracle.select(xy, polys, point_id_base=base)
+    np.testing.assert_array_equal(counts, ocounts)
+    np.testing.assert_array_equal(pt, opt)
+    np.testing.assert_array_equal(pl, opl)
+    np.testing.assert_array_equal(ids, oids)
+    return cv
+
+
+@pytest.mark.parametrize("s", [-1, 0, 1, 3, 5, 8, 10])
+def test_c1_all_ops_all_resolutions(spade, s):
+    w = configs.c1()
+    xy = np.concatenate([gen.points_host(w.points, w.point_seed, 0, w.n_points), configs.c1_edge_points(w.polys)])
+    check_all(spade, w.polys, xy, s=s, max_dim=w.max_dim, base=1000)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_tiny_lattice_bruteforce(spade, seed):
+    rng = np.random.default_rng(1000 + seed)
+    polys = random_polyset(rng, 0, 40, int(rng.integers(1, 7)))
+    xy = lattice(-2, -2, 42, 42)
+    for s in (0, 1, 2, 3, 4, 6):
+        check_all(spade, polys, xy, s=s)
+
+
+def test_grid_tiling_closed_form(spade):
+    polys = pg.grid_tiling(4, 4, 0, 0, 256, 256)
+    xy = gen.points_host(gen.uniform_params(0, 0, 1024, 1024), 7, 0, 200_000)
+    import torch
+    for s in (-1, 0, 4, 7):
+        cv = spade.Canvas(polys, log2_pixel=s)
+        counts = spade.join_count(cv, torch.as_tensor(xy).cuda()).cpu().numpy()
+        expect = np.bincount((xy[:, 1] >> 8) * 4 + (xy[:, 0] >> 8), minlength=16)
+        np.testing.assert_array_equal(counts, expect)
+
+
+def test_capacity_protocol(spade):
+    import torch
+    w = configs.c1()
+    xy = torch.as_tensor(gen.points_host(w.points, w.point_seed, 0, w.n_points)).cuda()
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    pt, pl = spade.join_pairs(cv, xy, capacity=5)          # too small -> retry with reported size
+    opt, opl = oracle.join_pairs(xy.cpu().numpy(), w.polys)
+    a, b = sorted_pairs(pt.cpu().numpy(), pl.cpu().numpy())
+    np.testing.assert_array_equal(a, opt)
+    np.testing.assert_array_equal(b, opl)
+    ids = spade.select(cv, xy, capacity=0)
+    np.testing.assert_array_equal(np.sort(ids.cpu().numpy()), oracle.select(xy.cpu().numpy(), w.polys))
+
+
+def test_empty_and_degenerate_inputs(spade):
+    import torch
+    w = configs.c1()
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    empty = torch.zeros((0, 2), dtype=torch.int32, device="cuda")
+    assert spade.join_count(cv, empty).sum().item() == 0
+    assert spade.select(cv, empty).numel() == 0
+    # unaligned views (head / tail scalar paths) of every length 0..40
+    xy = torch.as_tensor(gen.points_host(w.points, w.point_seed, 0, 64)).cuda()
+    for off in range(4):
+        for n in range(0, 41, 3):
+            sub = xy[off:off + n]
+            c = spade.join_count(cv, sub).cpu().numpy()
+            np.testing.assert_array_equal(c, oracle.join_count(sub.cpu().numpy(), w.polys))
+    # extreme coordinates: points far outside, at int32 limits
+    far = np.array([[-2**31, -2**31], [2**31 - 1, 2**31 - 1], [-2**31, 500], [500, 2**31 - 1], [0, 0]], np.int32)
+    check_all(spade, w.polys, far)
+    # polygon set with no vertices at all / zero polygons
+    nothing = pg.assemble([])
+    cv0 = spade.Canvas(nothing)
+    assert spade.join_count(cv0, xy).numel() == 0
+    one_empty = {"ring_xy": np.zeros((0, 2), np.int32), "ring_off": np.zeros(1, np.int64),
+                 "poly_ring_off": np.zeros(2, np.int64)}
+    cv1 = spade.Canvas(one_empty)
+    assert spade.join_count(cv1, xy).cpu().numpy().tolist() == [0]
+
+
+def test_coord_range_error(spade):
+    bad = {"ring_xy": np.array([[0, 0], [2**30, 0], [0, 5]], np.int32), "ring_off": np.array([0, 3], np.int64),
+           "poly_ring_off": np.array([0, 1], np.int64)}
+    with pytest.raises(spade.SpadeError) as e:
+        spade.Canvas(bad)
+    assert e.value.code == spade.SPADE_ERR_COORD_RANGE
+
+
+def test_tiling_with_islands_exactly_one_owner(spade):
+    import torch
+    polys = pg.jittered_tiling(6, 5, 9, domain=1 << 20, n_islands=4, seed=5)
+    xy = gen.points_host(gen.taxi_params(9, domain=1 << 20), 9, 0, 300_000)
+    check_all(spade, polys, xy[:50_000])
+    cv = spade.Canvas(polys)
+    pt, pl = spade.join_pairs(cv, torch.as_tensor(xy).cuda())
+    pt = pt.cpu().numpy()
+    assert len(pt) == len(xy) and len(np.unique(pt)) == len(xy)   # every point in exactly one polygon
