@@ -3,13 +3,19 @@
 // P:140-146, Sec. 5.5 boundary-index creation P:268).  Replaces the paper's OpenGL pipeline
 // (triangulation P:117, two-pass triangle/line render P:121, conservative rasterisation P:123)
 // with data-parallel kernels:
-//   K-B1  edge -> (row, pixel-range) fragments of every closed pixel an edge touches; mark them
-//   K-B2  maximal runs of boundary pixels per row; run -> edge CSR sorted by polygon
-//   K-B3  scanline crossing events at each row's bottom line; per (row, polygon) pairs of events
-//         bound interior spans; fill the non-boundary pixels (multi-owner pixels -> records)
-//   K-B4  terminal owner set of each run = owner set of the first non-boundary pixel to its right
+//   K-B0  edges of all rings (+ polygon id), coordinate range check, extent
+//   K-B1  edge -> (row, pixel-range) fragments of every CLOSED pixel an edge touches (exact
+//         rationals), and scanline crossing events at every row's bottom line y = Y0_j
+//   K-B2  mark boundary pixels; number them; pixel-local edge lists sorted by polygon
+//   K-B3  corner owner sets: per (row, polygon) consecutive event pairs bound the pixels whose
+//         lower-left corner lies inside (all pixels, boundary or not); overlaps -> owner sets
+//   K-B4  per boundary pixel: K = corner set XOR {polygons whose local edges cross the upward
+//         ray from the corner an odd number of times}; records; final canvas encoding
 //   K-B5  coarse tile summary (uniform owner / empty / mixed) for the shared-memory level
-// DESIGN.md "Canvas" has the exactness argument for the run-local PIP this enables.
+// The exactness argument: for p in boundary pixel (i, j) with lower-left
+// corner c = (X, Y0),  inside(p, P) = [P in K] XOR  (sum over P's local edges of
+//          cu(X, py) ^ cr(X, py) ^ cr(px, py))
+// where cr / cu are the half-open rightward / upward ray tests (perturbation reading of C1).
 #include <cub/cub.cuh>
 #include <vector>
 #include <algorithm>
@@ -70,6 +76,8 @@ __global__ void k_edges(const int2* __restrict__ xy, const int64_t* __restrict__
   }
 }
 
+__device__ __forceinline__ bool degenerate(int4 e) { return e.x == e.z && e.y == e.w; }
+
 // rows j whose CLOSED strip [Y0_j, Y0_j + S] meets the edge's y-range
 __device__ __forceinline__ void frag_rows(int4 e, const Geo& g, int64_t& jlo, int64_t& jhi) {
   int64_t ylo = imin64(e.y, e.w), yhi = imax64(e.y, e.w);
@@ -104,134 +112,123 @@ __device__ __forceinline__ void frag_cols(int4 e, const Geo& g, int64_t j, int& 
 }
 
 __global__ void k_count(const int4* __restrict__ seg, int64_t E, Geo g, int64_t* __restrict__ nfrag,
-                        int64_t* __restrict__ nlist, int64_t* __restrict__ nev) {
+                        int64_t* __restrict__ nev) {
   for (int64_t k = blockIdx.x * (int64_t)kBT + threadIdx.x; k < E; k += (int64_t)gridDim.x * kBT) {
     int4 e = seg[k];
     int64_t a, b;
     frag_rows(e, g, a, b);
-    int64_t nf = b >= a ? b - a + 1 : 0;
-    nfrag[k] = nf;
-    nlist[k] = (e.y != e.w) ? nf : 0;        // horizontal edges never straddle: not listed
-    int64_t c0, c1;
-    event_rows(e, g, c0, c1);
-    nev[k] = (e.y != e.w && c1 >= c0) ? c1 - c0 + 1 : 0;
+    nfrag[k] = (!degenerate(e) && b >= a) ? b - a + 1 : 0;   // zero-length edges never cross anything
+    event_rows(e, g, a, b);
+    nev[k] = (e.y != e.w && b >= a) ? b - a + 1 : 0;
   }
 }
 
 struct Frag { int32_t j, ilo, ihi, e; };
 
+// event key: row | polygon | k,  k = 2c + (x* strictly inside column c ? 1 : 0), c = column of x*,
+// so that  x* > X_i  <=>  k > 2i  for every column i.
 __global__ void k_emit(const int4* __restrict__ seg, const int32_t* __restrict__ poly, int64_t E, Geo g,
                        const int64_t* __restrict__ frag_off, const int64_t* __restrict__ ev_off,
-                       Frag* __restrict__ frags, uint64_t* __restrict__ ev_keys, int pbits, int cbits) {
+                       Frag* __restrict__ frags, int64_t* __restrict__ frag_w, uint64_t* __restrict__ ev_keys,
+                       int pbits, int kbits) {
   for (int64_t k = blockIdx.x * (int64_t)kBT + threadIdx.x; k < E; k += (int64_t)gridDim.x * kBT) {
     int4 e = seg[k];
     int64_t a, b;
-    frag_rows(e, g, a, b);
-    int64_t o = frag_off[k];
-    for (int64_t j = a; j <= b; ++j, ++o) {
-      int ilo, ihi;
-      frag_cols(e, g, j, ilo, ihi);
-      frags[o] = Frag{(int32_t)j, ilo, ihi, (int32_t)k};
+    if (!degenerate(e)) {
+      frag_rows(e, g, a, b);
+      int64_t o = frag_off[k];
+      for (int64_t j = a; j <= b; ++j, ++o) {
+        int ilo, ihi;
+        frag_cols(e, g, j, ilo, ihi);
+        frags[o] = Frag{(int32_t)j, ilo, ihi, (int32_t)k};
+        frag_w[o] = ihi >= ilo ? ihi - ilo + 1 : 0;
+      }
     }
     if (e.y == e.w) continue;
     event_rows(e, g, a, b);
-    o = ev_off[k];
+    int64_t o = ev_off[k];
     int64_t dx = (int64_t)e.z - e.x, dy = (int64_t)e.w - e.y;
     uint64_t pk = (uint64_t)poly[k];
     for (int64_t j = a; j <= b; ++j, ++o) {
       int64_t Y0 = g.miny + j * g.S;
-      int64_t xf = e.x + floor_div(dx * (Y0 - e.y), dy);   // floor of the crossing x*
+      int64_t t = dx * (Y0 - e.y);
+      int64_t xf = e.x + floor_div(t, dy);                  // floor of the crossing x*
       int64_t c = floor_div(xf - g.minx, g.S);              // pixel column holding x*
-      ev_keys[o] = ((uint64_t)j << (pbits + cbits)) | (pk << cbits) | (uint64_t)c;
+      bool exact = (t % dy == 0) && ((xf - g.minx) % g.S == 0);
+      uint64_t kk = 2 * (uint64_t)c + (exact ? 0 : 1);
+      ev_keys[o] = ((uint64_t)j << (pbits + kbits)) | (pk << kbits) | kk;
     }
   }
 }
 
-__global__ void k_mark(const Frag* __restrict__ frags, int64_t F, int W, uint8_t* __restrict__ bmap) {
+__global__ void k_mark(const Frag* __restrict__ frags, int64_t F, int W, int32_t* __restrict__ bflag) {
   for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < F; t += (int64_t)gridDim.x * kBT) {
     Frag f = frags[t];
-    uint8_t* row = bmap + (int64_t)f.j * W;
+    int32_t* row = bflag + (int64_t)f.j * W;
     for (int i = f.ilo; i <= f.ihi; ++i) row[i] = 1;
   }
 }
 
-__global__ void k_run_flags(const uint8_t* __restrict__ bmap, int64_t WH, int W, int32_t* __restrict__ flag) {
-  for (int64_t p = blockIdx.x * (int64_t)kBT + threadIdx.x; p < WH; p += (int64_t)gridDim.x * kBT) {
-    int i = (int)(p % W);
-    flag[p] = (bmap[p] && (i == 0 || !bmap[p - 1])) ? 1 : 0;
-  }
+// bscan = inclusive scan of boundary flags: boundary pixel p has id bscan[p] - 1
+__global__ void k_bids(const int32_t* __restrict__ bflag, const int32_t* __restrict__ bscan, int64_t WH,
+                       int64_t* __restrict__ pix_of) {
+  for (int64_t p = blockIdx.x * (int64_t)kBT + threadIdx.x; p < WH; p += (int64_t)gridDim.x * kBT)
+    if (bflag[p]) pix_of[bscan[p] - 1] = p;
 }
 
-// after the inclusive scan: run id of boundary pixel p = scan[p] - 1
-__global__ void k_run_ids(const uint8_t* __restrict__ bmap, const int32_t* __restrict__ scan, int64_t WH, int W,
-                          int32_t* __restrict__ fine, int64_t* __restrict__ run_end) {
-  for (int64_t p = blockIdx.x * (int64_t)kBT + threadIdx.x; p < WH; p += (int64_t)gridDim.x * kBT) {
-    if (!bmap[p]) { fine[p] = kEmpty; continue; }
-    int32_t r = scan[p] - 1;
-    fine[p] = -2 - r;
-    int i = (int)(p % W);
-    if (i == W - 1 || !bmap[p + 1]) run_end[r] = p;
-  }
-}
-
-__global__ void k_list(const Frag* __restrict__ frags, int64_t F, int W, const int4* __restrict__ seg,
-                       const int32_t* __restrict__ poly, const int32_t* __restrict__ scan,
-                       const int64_t* __restrict__ frag_off, const int64_t* __restrict__ list_off,
-                       uint64_t* __restrict__ keys, int32_t* __restrict__ vals, int32_t* __restrict__ run_cnt) {
+// one (boundary pixel, edge) entry per pixel of every fragment
+__global__ void k_local(const Frag* __restrict__ frags, int64_t F, int W, const int64_t* __restrict__ lw_off,
+                        const int32_t* __restrict__ poly, const int32_t* __restrict__ bscan,
+                        uint64_t* __restrict__ keys, int32_t* __restrict__ vals, int32_t* __restrict__ cnt) {
   for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < F; t += (int64_t)gridDim.x * kBT) {
     Frag f = frags[t];
-    int4 e = seg[f.e];
-    if (e.y == e.w) continue;
-    int32_t run = scan[(int64_t)f.j * W + f.ilo] - 1;   // all of [ilo, ihi] lies in this run
-    int64_t pos = list_off[f.e] + (t - frag_off[f.e]);
-    keys[pos] = ((uint64_t)(uint32_t)run << 32) | (uint32_t)poly[f.e];
-    vals[pos] = f.e;
-    atomicAdd(&run_cnt[run], 1);
-  }
-}
-
-__global__ void k_gather_edges(const int32_t* __restrict__ sorted_e, int64_t L, const int4* __restrict__ seg,
-                               const int32_t* __restrict__ poly, int4* __restrict__ run_seg,
-                               int32_t* __restrict__ run_poly) {
-  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < L; t += (int64_t)gridDim.x * kBT) {
-    int32_t e = sorted_e[t];
-    run_seg[t] = seg[e];
-    run_poly[t] = poly[e];
-  }
-}
-
-// K-B3 fill: sorted events of one (row, polygon) come in consecutive pairs (every closed ring
-// crosses a horizontal line an even number of times); non-boundary pixels strictly between the
-// pair's columns have the polygon's parity odd at their lower-left corner.
-__global__ void k_fill(const uint64_t* __restrict__ ev, int64_t NE, int W, int pbits, int cbits,
-                       const uint8_t* __restrict__ bmap, int32_t* __restrict__ fine,
-                       unsigned long long* __restrict__ multi, unsigned long long* __restrict__ nmulti,
-                       int64_t multi_cap, int* __restrict__ bad) {
-  const uint64_t cmask = (1ull << cbits) - 1, pmask = (1ull << pbits) - 1;
-  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; 2 * t + 1 < NE + 1; t += (int64_t)gridDim.x * kBT) {
-    if (2 * t + 1 >= NE) { atomicOr(bad, 2); break; }
-    uint64_t k0 = ev[2 * t], k1 = ev[2 * t + 1];
-    if ((k0 >> cbits) != (k1 >> cbits)) { atomicOr(bad, 2); continue; }
-    int64_t j = (int64_t)(k0 >> (cbits + pbits));
-    int32_t p = (int32_t)((k0 >> cbits) & pmask);
-    int ca = (int)(k0 & cmask), cb = (int)(k1 & cmask);
-    int64_t rowbase = j * W;
-    for (int i = ca + 1; i < cb; ++i) {
-      int64_t px = rowbase + i;
-      if (bmap[px]) continue;
-      int old = atomicCAS(&fine[px], kEmpty, p);
-      if (old == kEmpty) continue;
-      int prev = atomicExch(&fine[px], kMultiMark);
-      unsigned long long q = atomicAdd(nmulti, prev >= 0 ? 2ull : 1ull);
-      if ((int64_t)q < multi_cap) multi[q] = ((unsigned long long)px << 32) | (uint32_t)p;
-      if (prev >= 0 && (int64_t)q + 1 < multi_cap) multi[q + 1] = ((unsigned long long)px << 32) | (uint32_t)prev;
+    int64_t o = lw_off[t];
+    uint32_t pk = (uint32_t)poly[f.e];
+    for (int i = f.ilo; i <= f.ihi; ++i, ++o) {
+      int32_t bid = bscan[(int64_t)f.j * W + i] - 1;
+      keys[o] = ((uint64_t)(uint32_t)bid << 32) | pk;
+      vals[o] = f.e;
+      atomicAdd(&cnt[bid], 1);
     }
   }
 }
 
-__global__ void k_reset_fill(const uint8_t* __restrict__ bmap, int64_t WH, int32_t* __restrict__ fine) {
-  for (int64_t p = blockIdx.x * (int64_t)kBT + threadIdx.x; p < WH; p += (int64_t)gridDim.x * kBT)
-    if (!bmap[p]) fine[p] = kEmpty;
+__global__ void k_gather_edges(const int32_t* __restrict__ sorted_e, int64_t L, const int4* __restrict__ seg,
+                               const int32_t* __restrict__ poly, int4* __restrict__ rseg, int32_t* __restrict__ rpoly) {
+  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < L; t += (int64_t)gridDim.x * kBT) {
+    int32_t e = sorted_e[t];
+    rseg[t] = seg[e];
+    rpoly[t] = poly[e];
+  }
+}
+
+// K-B3: sorted events of one (row, polygon) come in consecutive pairs (a closed ring crosses a
+// horizontal line an even number of times).  Polygon P contains the lower-left corner of pixel
+// i iff 2i lies in [k_a, k_b) for a pair, i.e. i in [ceil(k_a/2), ceil(k_b/2) - 1].
+__global__ void k_fill(const uint64_t* __restrict__ ev, int64_t NE, int W, int pbits, int kbits,
+                       int32_t* __restrict__ corner, unsigned long long* __restrict__ multi,
+                       unsigned long long* __restrict__ nmulti, int64_t multi_cap, int* __restrict__ bad) {
+  const uint64_t kmask = (1ull << kbits) - 1, pmask = (1ull << pbits) - 1;
+  const int64_t NP = NE / 2;
+  if (blockIdx.x == 0 && threadIdx.x == 0 && (NE & 1)) atomicOr(bad, 2);
+  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < NP; t += (int64_t)gridDim.x * kBT) {
+    uint64_t k0 = ev[2 * t], k1 = ev[2 * t + 1];
+    if ((k0 >> kbits) != (k1 >> kbits)) { atomicOr(bad, 2); continue; }
+    int64_t j = (int64_t)(k0 >> (kbits + pbits));
+    int32_t p = (int32_t)((k0 >> kbits) & pmask);
+    int64_t ka = (int64_t)(k0 & kmask), kb = (int64_t)(k1 & kmask);
+    int i0 = (int)((ka + 1) >> 1), i1 = (int)((kb + 1) >> 1);   // [ceil(ka/2), ceil(kb/2))
+    int32_t* row = corner + j * W;
+    for (int i = i0; i < i1; ++i) {
+      int old = atomicCAS(&row[i], kEmpty, p);
+      if (old == kEmpty) continue;
+      int prev = atomicExch(&row[i], kMultiMark);
+      unsigned long long q = atomicAdd(nmulti, prev >= 0 ? 2ull : 1ull);
+      const uint64_t px = (uint64_t)(j * W + i);
+      if ((int64_t)q < multi_cap) multi[q] = (px << 32) | (uint32_t)p;
+      if (prev >= 0 && (int64_t)q + 1 < multi_cap) multi[q + 1] = (px << 32) | (uint32_t)prev;
+    }
+  }
 }
 
 // sorted (pixel << 32 | poly) -> head flags of pixel groups
@@ -240,10 +237,9 @@ __global__ void k_multi_heads(const unsigned long long* __restrict__ m, int64_t 
     head[t] = (t == 0 || (m[t] >> 32) != (m[t - 1] >> 32)) ? 1 : 0;
 }
 
-// head_scan = inclusive scan of heads: group index g = head_scan[t] - 1
-__global__ void k_multi_records(const unsigned long long* __restrict__ m, int64_t M, const int32_t* __restrict__ hs,
-                                int64_t NR, int32_t* __restrict__ sets, int2* __restrict__ set_rng,
-                                RunRec* __restrict__ runs, int32_t* __restrict__ fine) {
+// head_scan = inclusive scan of heads: owner-set index g = head_scan[t] - 1; corner[p] = -2 - g
+__global__ void k_multi_sets(const unsigned long long* __restrict__ m, int64_t M, const int32_t* __restrict__ hs,
+                             int32_t* __restrict__ sets, int2* __restrict__ set_rng, int32_t* __restrict__ corner) {
   for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < M; t += (int64_t)gridDim.x * kBT) {
     int32_t g = hs[t] - 1;
     sets[t] = (int32_t)(m[t] & 0xffffffffu);
@@ -252,23 +248,87 @@ __global__ void k_multi_records(const unsigned long long* __restrict__ m, int64_
     int64_t e = t + 1;
     while (e < M && (m[e] >> 32) == (m[t] >> 32)) ++e;
     set_rng[g] = make_int2((int)t, (int)(e - t));
-    runs[NR + g] = RunRec{0, 0, -2 - g};
-    fine[(int64_t)(m[t] >> 32)] = -2 - (int32_t)(NR + g);
+    corner[(int64_t)(m[t] >> 32)] = -2 - g;
   }
 }
 
-__global__ void k_runs(int64_t NR, int W, const int64_t* __restrict__ run_end, const int32_t* __restrict__ run_cnt,
-                       const int64_t* __restrict__ run_beg, const int32_t* __restrict__ fine, RunRec* __restrict__ runs) {
-  for (int64_t r = blockIdx.x * (int64_t)kBT + threadIdx.x; r < NR; r += (int64_t)gridDim.x * kBT) {
-    int64_t e = run_end[r];
-    int32_t term = kEmpty;
-    if ((int)(e % W) != W - 1) {
-      int32_t v = fine[e + 1];                     // first non-boundary pixel right of the run
-      if (v >= 0) term = v;
-      else if (v <= -2) term = -2 - (int32_t)((-2 - (int64_t)v) - NR);   // multi record -> set index
+// half-open upward-ray test at q = (qx, qy) (perturbation reading: ray from (qx+e', qy+e)).
+__device__ __forceinline__ int cu_test(int4 e, int64_t qx, int64_t qy) {
+  if ((e.x > qx) == (e.z > qx)) return 0;
+  int64_t dx = (int64_t)e.z - e.x, dy = (int64_t)e.w - e.y;
+  int64_t w = dy * (qx - e.x) - dx * (qy - e.y);
+  return dx > 0 ? (w > 0 || (w == 0 && dy > 0)) : (w < 0 || (w == 0 && dy < 0));
+}
+
+// K-B4: K = corner set XOR {P : odd number of P's local edges cross the upward ray from the
+// corner}.  PASS 0 counts |K| into ksize; PASS 1 writes records and the members of sets with
+// |K| >= 2 at kout[koff[b] ...] (ascending polygon order).
+template <int PASS>
+__global__ void k_kset(int64_t NB, const int64_t* __restrict__ pix_of, Geo g, const int32_t* __restrict__ corner,
+                       const int32_t* __restrict__ csets, const int2* __restrict__ crng,
+                       const int64_t* __restrict__ le_beg, const int32_t* __restrict__ le_cnt,
+                       const int4* __restrict__ rseg, const int32_t* __restrict__ rpoly,
+                       int32_t* __restrict__ ksize, const int64_t* __restrict__ koff, int32_t* __restrict__ kout,
+                       RunRec* __restrict__ recs) {
+  for (int64_t b = blockIdx.x * (int64_t)kBT + threadIdx.x; b < NB; b += (int64_t)gridDim.x * kBT) {
+    const int64_t p = pix_of[b];
+    const int64_t i = p % g.W, j = p / g.W;
+    const int64_t X = g.minx + i * g.S, Y0 = g.miny + j * g.S;
+    const int32_t cv = corner[p];
+    int cn, cb = 0;
+    if (cv >= 0) cn = 1; else if (cv == kEmpty) cn = 0; else { int2 r = crng[-2 - cv]; cb = r.x; cn = r.y; }
+    const bool big = PASS == 1 && ksize[b] >= 2;
+    int64_t out = big ? koff[b] : 0;
+    int n = 0;
+    int32_t first = kEmpty;
+    const int64_t e0 = le_beg[b], e1 = e0 + le_cnt[b];
+    int64_t e = e0;
+    int ci = 0;
+    while (e < e1 || ci < cn) {
+      const int32_t P = e < e1 ? rpoly[e] : INT32_MAX;
+      const int32_t Cp = ci < cn ? (cv >= 0 ? cv : csets[cb + ci]) : INT32_MAX;
+      int par = 0;
+      int32_t Q;
+      if (Cp < P) { Q = Cp; par = 1; ++ci; }
+      else {
+        Q = P;
+        for (; e < e1 && rpoly[e] == P; ++e) par ^= cu_test(rseg[e], X, Y0);
+        if (Cp == P) { par ^= 1; ++ci; }
+      }
+      if (par) {
+        if (big) kout[out++] = Q;
+        if (n == 0) first = Q;
+        ++n;
+      }
     }
-    runs[r] = RunRec{run_beg[r], run_cnt[r], term};
+    if (PASS == 0) ksize[b] = n;
+    else recs[b] = RunRec{e0, (int32_t)(e1 - e0), first};   // |K| >= 2 fixed up by k_kset_rng
   }
+}
+
+__global__ void k_kset_rng(int64_t NB, const int32_t* __restrict__ ksize, const int64_t* __restrict__ koff,
+                           const int32_t* __restrict__ kidx, int64_t base_idx, int64_t base_pos,
+                           int2* __restrict__ set_rng, RunRec* __restrict__ recs) {
+  for (int64_t b = blockIdx.x * (int64_t)kBT + threadIdx.x; b < NB; b += (int64_t)gridDim.x * kBT) {
+    if (ksize[b] < 2) continue;
+    int64_t g = base_idx + kidx[b];
+    set_rng[g] = make_int2((int)(base_pos + koff[b]), ksize[b]);
+    recs[b].term = -2 - (int32_t)g;
+  }
+}
+
+__global__ void k_finalize(int64_t WH, const int32_t* __restrict__ bflag, const int32_t* __restrict__ bscan,
+                           const int32_t* __restrict__ corner, int64_t NB, int32_t* __restrict__ fine) {
+  for (int64_t p = blockIdx.x * (int64_t)kBT + threadIdx.x; p < WH; p += (int64_t)gridDim.x * kBT) {
+    if (bflag[p]) { fine[p] = -2 - (bscan[p] - 1); continue; }
+    int32_t v = corner[p];
+    fine[p] = v >= kEmpty ? v : (int32_t)(-2 - (NB + (-2 - (int64_t)v)));   // owner set g -> record NB + g
+  }
+}
+
+__global__ void k_multi_recs(int64_t NG, int64_t NB, RunRec* __restrict__ recs) {
+  for (int64_t g = blockIdx.x * (int64_t)kBT + threadIdx.x; g < NG; g += (int64_t)gridDim.x * kBT)
+    recs[NB + g] = RunRec{0, 0, (int32_t)(-2 - g)};
 }
 
 __global__ void k_coarse(const int32_t* __restrict__ fine, int W, int H, int b, int Wc, int Hc,
@@ -290,6 +350,9 @@ __global__ void k_coarse(const int32_t* __restrict__ fine, int W, int H, int b, 
     coarse[t] = c;
   }
 }
+
+struct BigSize { __host__ __device__ int64_t operator()(int32_t v) const { return v >= 2 ? v : 0; } };
+struct BigFlag { __host__ __device__ int32_t operator()(int32_t v) const { return v >= 2 ? 1 : 0; } };
 
 int bits_for(int64_t v) {  // bits to hold values 0..v
   int b = 1;
@@ -317,25 +380,8 @@ int grid_for(int64_t n) {
   return (int)imax64(1, std::min(g, cap));
 }
 
-#define SPADE_TRY(call, what)                                        \
-  do {                                                               \
-    cudaError_t _e = (call);                                         \
-    if (_e != cudaSuccess) {                                         \
-      return _e == cudaErrorMemoryAllocation                         \
-                 ? set_error(SPADE_ERR_OOM, "%s: out of device memory", what) \
-                 : check_cuda(_e, what);                             \
-    }                                                                \
-  } while (0)
-
-#define LAUNCH(kern, n, st, ...)                                     \
-  do {                                                               \
-    kern<<<grid_for(n), kBT, 0, st>>>(__VA_ARGS__);                  \
-    count_launch();                                                  \
-    SPADE_TRY(cudaGetLastError(), #kern);                            \
-  } while (0)
-
 template <class F>
-cudaError_t cub_call(DevBufs& bufs, cudaStream_t st, F f) {
+cudaError_t cub_call(DevBufs& bufs, F f) {
   size_t tmp = 0;
   cudaError_t e = f(nullptr, tmp);
   if (e != cudaSuccess) return e;
@@ -344,7 +390,6 @@ cudaError_t cub_call(DevBufs& bufs, cudaStream_t st, F f) {
   if (e != cudaSuccess) return e;
   e = f(t, tmp);
   count_launch();
-  (void)st;
   return e;
 }
 
@@ -367,16 +412,19 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
 
   // --- offsets to the host for validation (R+1 and P+1 int64s) ---
   std::vector<int64_t> h_pro(P + 1, 0);
-  if (P > 0) SPADE_TRY(cudaMemcpyAsync(h_pro.data(), poly_ring_off, sizeof(int64_t) * (P + 1), cudaMemcpyDeviceToHost, st), "copy poly_ring_off");
-  SPADE_TRY(cudaStreamSynchronize(st), "sync");
+  cudaError_t ce;
+  if (P > 0 && (ce = cudaMemcpyAsync(h_pro.data(), poly_ring_off, sizeof(int64_t) * (P + 1), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+    return check_cuda(ce, "copy poly_ring_off");
+  if ((ce = cudaStreamSynchronize(st)) != cudaSuccess) return check_cuda(ce, "sync");
   int64_t R = h_pro[P];
   if (h_pro[0] != 0 || R < 0) return set_error(SPADE_ERR_INVALID_ARG, "poly_ring_off must start at 0");
   for (int32_t p = 0; p < P; ++p)
     if (h_pro[p + 1] < h_pro[p]) return set_error(SPADE_ERR_INVALID_ARG, "poly_ring_off not non-decreasing at %d", p);
   std::vector<int64_t> h_ro(R + 1, 0);
   if (R > 0) {
-    SPADE_TRY(cudaMemcpyAsync(h_ro.data(), ring_off, sizeof(int64_t) * (R + 1), cudaMemcpyDeviceToHost, st), "copy ring_off");
-    SPADE_TRY(cudaStreamSynchronize(st), "sync");
+    if ((ce = cudaMemcpyAsync(h_ro.data(), ring_off, sizeof(int64_t) * (R + 1), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+      return check_cuda(ce, "copy ring_off");
+    if ((ce = cudaStreamSynchronize(st)) != cudaSuccess) return check_cuda(ce, "sync");
   }
   int64_t V = h_ro[R];
   if (h_ro[0] != 0 || V < 0) return set_error(SPADE_ERR_INVALID_ARG, "ring_off must start at 0");
@@ -394,19 +442,17 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
     *out = c;
     return SPADE_OK;
   }
+#define TRYF(call, what) do { cudaError_t _e = (call); if (_e != cudaSuccess) return fail(_e == cudaErrorMemoryAllocation ? set_error(SPADE_ERR_OOM, "build: %s: out of device memory", what) : check_cuda(_e, what)); } while (0)
+#define ALLOC(ptr, n, what) TRYF(tmp.alloc(&ptr, (size_t)(n)), what)
+#define LAUNCH(kern, n, ...) do { kern<<<grid_for(n), kBT, 0, st>>>(__VA_ARGS__); count_launch(); TRYF(cudaGetLastError(), #kern); } while (0)
 
   DevBufs tmp;
   int4* seg; int32_t* epoly; int* ext; int* bad;
-  if (tmp.alloc(&seg, V) || tmp.alloc(&epoly, V) || tmp.alloc(&ext, 4) || tmp.alloc(&bad, 1))
-    return fail(set_error(SPADE_ERR_OOM, "build: edge buffers"));
+  ALLOC(seg, V, "edges"); ALLOC(epoly, V, "edges"); ALLOC(ext, 4, "ext"); ALLOC(bad, 1, "flag");
   int h_ext0[4] = {INT_MAX, INT_MAX, INT_MIN, INT_MIN};
-  int rc;
-#define TRYF(call, what) do { cudaError_t _e = (call); if (_e != cudaSuccess) return fail(_e == cudaErrorMemoryAllocation ? set_error(SPADE_ERR_OOM, "%s", what) : check_cuda(_e, what)); } while (0)
   TRYF(cudaMemcpyAsync(ext, h_ext0, sizeof(h_ext0), cudaMemcpyHostToDevice, st), "ext init");
   TRYF(cudaMemsetAsync(bad, 0, sizeof(int), st), "memset");
-  k_edges<<<grid_for(V), kBT, 0, st>>>((const int2*)ring_xy, ring_off, R, poly_ring_off, P, V, seg, epoly, ext, bad);
-  count_launch();
-  TRYF(cudaGetLastError(), "k_edges");
+  LAUNCH(k_edges, V, (const int2*)ring_xy, ring_off, R, poly_ring_off, P, V, seg, epoly, ext, bad);
   int h_ext[4], h_bad = 0;
   TRYF(cudaMemcpyAsync(h_ext, ext, sizeof(h_ext), cudaMemcpyDeviceToHost, st), "ext");
   TRYF(cudaMemcpyAsync(&h_bad, bad, sizeof(int), cudaMemcpyDeviceToHost, st), "bad");
@@ -426,95 +472,87 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   if (W64 * H64 > (1ll << 31) - 4) return fail(set_error(SPADE_ERR_INVALID_ARG, "canvas too large (%lld x %lld)", (long long)W64, (long long)H64));
   g.W = (int)W64; g.H = (int)H64;
   const int64_t WH = (int64_t)g.W * g.H;
-  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries
-  const int64_t kMaxTiles = 65536;
+  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (160 KB)
+  const int64_t kMaxTiles = 81920;
   int b = 0;
   while (((int64_t)(g.W + (1 << b) - 1) >> b) * ((int64_t)(g.H + (1 << b) - 1) >> b) > kMaxTiles) ++b;
   int Wc = (g.W + (1 << b) - 1) >> b, Hc = (g.H + (1 << b) - 1) >> b;
 
-  // --- K-B1 counts, scans ---
-  int64_t *nfrag, *nlist, *nev, *frag_off, *list_off, *ev_off;
-  if (tmp.alloc(&nfrag, V) || tmp.alloc(&nlist, V) || tmp.alloc(&nev, V) || tmp.alloc(&frag_off, V + 1) ||
-      tmp.alloc(&list_off, V + 1) || tmp.alloc(&ev_off, V + 1))
-    return fail(set_error(SPADE_ERR_OOM, "build: count buffers"));
-  k_count<<<grid_for(V), kBT, 0, st>>>(seg, V, g, nfrag, nlist, nev);
-  count_launch();
-  TRYF(cudaGetLastError(), "k_count");
-  for (auto pr : {std::make_pair(nfrag, frag_off), std::make_pair(nlist, list_off), std::make_pair(nev, ev_off)}) {
+  // --- K-B1 counts, scans, emit ---
+  int64_t *nfrag, *nev, *frag_off, *ev_off;
+  ALLOC(nfrag, V, "counts"); ALLOC(nev, V, "counts"); ALLOC(frag_off, V + 1, "counts"); ALLOC(ev_off, V + 1, "counts");
+  LAUNCH(k_count, V, seg, V, g, nfrag, nev);
+  for (auto pr : {std::make_pair(nfrag, frag_off), std::make_pair(nev, ev_off)}) {
     int64_t* in = pr.first; int64_t* o = pr.second;
-    TRYF(cub_call(tmp, st, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, in, o + 1, V, st); }), "scan counts");
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, in, o + 1, V, st); }), "scan counts");
     TRYF(cudaMemsetAsync(o, 0, sizeof(int64_t), st), "memset");
   }
-  int64_t F = 0, L = 0, NE = 0;
+  int64_t F = 0, NE = 0;
   TRYF(cudaMemcpyAsync(&F, frag_off + V, 8, cudaMemcpyDeviceToHost, st), "F");
-  TRYF(cudaMemcpyAsync(&L, list_off + V, 8, cudaMemcpyDeviceToHost, st), "L");
   TRYF(cudaMemcpyAsync(&NE, ev_off + V, 8, cudaMemcpyDeviceToHost, st), "NE");
   TRYF(cudaStreamSynchronize(st), "sync counts");
-  tmp.release(nfrag); tmp.release(nlist); tmp.release(nev);
+  tmp.release(nfrag); tmp.release(nev);
 
-  const int pbits = bits_for(imax64(P - 1, 1)), cbits = bits_for(g.W - 1), jbits = bits_for(g.H - 1);
-  if (pbits + cbits + jbits > 64) return fail(set_error(SPADE_ERR_INVALID_ARG, "canvas/polygon count too large for event keys"));
+  const int pbits = bits_for(std::max<int64_t>(P - 1, 1)), kbits = bits_for(2 * (int64_t)g.W), jbits = bits_for(g.H - 1);
+  if (pbits + kbits + jbits > 64) return fail(set_error(SPADE_ERR_INVALID_ARG, "canvas/polygon count too large for event keys"));
 
-  Frag* frags; uint64_t* ev;
-  if (tmp.alloc(&frags, F) || tmp.alloc(&ev, NE)) return fail(set_error(SPADE_ERR_OOM, "build: fragments"));
-  k_emit<<<grid_for(V), kBT, 0, st>>>(seg, epoly, V, g, frag_off, ev_off, frags, ev, pbits, cbits);
-  count_launch();
-  TRYF(cudaGetLastError(), "k_emit");
+  Frag* frags; int64_t* frag_w; uint64_t* ev;
+  ALLOC(frags, F, "fragments"); ALLOC(frag_w, F + 1, "fragments"); ALLOC(ev, NE, "events");
+  LAUNCH(k_emit, V, seg, epoly, V, g, frag_off, ev_off, frags, frag_w, ev, pbits, kbits);
 
-  // --- mark boundary pixels, runs ---
-  uint8_t* bmap; int32_t* scan;
-  if (tmp.alloc(&bmap, WH) || tmp.alloc(&scan, WH)) return fail(set_error(SPADE_ERR_OOM, "build: bitmap"));
-  if (cudaMalloc(&c->fine, sizeof(int32_t) * WH) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas"));
-  TRYF(cudaMemsetAsync(bmap, 0, WH, st), "memset bmap");
-  if (F > 0) { LAUNCH(k_mark, F, st, frags, F, g.W, bmap); }
-  LAUNCH(k_run_flags, WH, st, bmap, WH, g.W, scan);
-  TRYF(cub_call(tmp, st, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, scan, scan, WH, st); }), "scan runs");
-  int32_t NR32 = 0;
-  TRYF(cudaMemcpyAsync(&NR32, scan + WH - 1, 4, cudaMemcpyDeviceToHost, st), "NR");
-  TRYF(cudaStreamSynchronize(st), "sync runs");
-  const int64_t NR = NR32;
-  int64_t* run_end; int32_t* run_cnt; int64_t* run_beg;
-  if (tmp.alloc(&run_end, NR) || tmp.alloc(&run_cnt, NR) || tmp.alloc(&run_beg, NR + 1))
-    return fail(set_error(SPADE_ERR_OOM, "build: runs"));
-  LAUNCH(k_run_ids, WH, st, bmap, scan, WH, g.W, c->fine, run_end);
-
-  // --- run -> edge CSR, sorted by (run, polygon) ---
+  // --- K-B2 boundary pixels, ids, pixel-local edge lists ---
+  int32_t *bflag, *bscan;
+  ALLOC(bflag, WH, "boundary flags"); ALLOC(bscan, WH, "boundary ids");
+  TRYF(cudaMemsetAsync(bflag, 0, sizeof(int32_t) * WH, st), "memset");
+  if (F > 0) LAUNCH(k_mark, F, frags, F, g.W, bflag);
+  TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, bflag, bscan, WH, st); }), "scan boundary");
+  int64_t* lw_off;
+  ALLOC(lw_off, F + 1, "local offsets");
+  TRYF(cudaMemsetAsync(lw_off, 0, 8, st), "memset");
+  if (F > 0)
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, frag_w, lw_off + 1, F, st); }), "scan local");
+  int32_t NB32 = 0; int64_t L = 0;
+  TRYF(cudaMemcpyAsync(&NB32, bscan + WH - 1, 4, cudaMemcpyDeviceToHost, st), "NB");
+  TRYF(cudaMemcpyAsync(&L, lw_off + F, 8, cudaMemcpyDeviceToHost, st), "L");
+  TRYF(cudaStreamSynchronize(st), "sync boundary");
+  const int64_t NB = NB32;
+  tmp.release(frag_w);
+  int64_t *pix_of, *le_beg; int32_t* le_cnt;
+  ALLOC(pix_of, NB, "pixel ids"); ALLOC(le_beg, NB + 1, "local edges"); ALLOC(le_cnt, NB, "local edges");
+  if (NB > 0) LAUNCH(k_bids, WH, bflag, bscan, WH, pix_of);
   uint64_t *lk, *lk2; int32_t *lv, *lv2;
-  if (tmp.alloc(&lk, L) || tmp.alloc(&lk2, L) || tmp.alloc(&lv, L) || tmp.alloc(&lv2, L))
-    return fail(set_error(SPADE_ERR_OOM, "build: run edges"));
-  TRYF(cudaMemsetAsync(run_cnt, 0, sizeof(int32_t) * imax64(NR, 1), st), "memset");
-  if (F > 0) { LAUNCH(k_list, F, st, frags, F, g.W, seg, epoly, scan, frag_off, list_off, lk, lv, run_cnt); }
-  const int rbits = bits_for(imax64(NR - 1, 1));
-  if (L > 0) {
-    TRYF(cub_call(tmp, st, [&](void* t, size_t& sz) {
-      return cub::DeviceRadixSort::SortPairs(t, sz, lk, lk2, lv, lv2, L, 0, 32 + rbits, st); }), "sort run edges");
-  }
-  if (NR > 0) {
-    TRYF(cub_call(tmp, st, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, run_cnt, run_beg, NR, st); }), "scan run edges");
-  }
-  if (cudaMalloc(&c->run_seg, sizeof(int4) * imax64(L, 1)) != cudaSuccess ||
-      cudaMalloc(&c->run_poly, sizeof(int32_t) * imax64(L, 1)) != cudaSuccess)
-    return fail(set_error(SPADE_ERR_OOM, "build: run edge arrays"));
-  if (L > 0) { LAUNCH(k_gather_edges, L, st, lv2, L, seg, epoly, c->run_seg, c->run_poly); }
-  tmp.release(lk); tmp.release(lk2); tmp.release(lv); tmp.release(lv2);
+  ALLOC(lk, L, "local edges"); ALLOC(lk2, L, "local edges"); ALLOC(lv, L, "local edges"); ALLOC(lv2, L, "local edges");
+  TRYF(cudaMemsetAsync(le_cnt, 0, sizeof(int32_t) * std::max<int64_t>(NB, 1), st), "memset");
+  if (F > 0) LAUNCH(k_local, F, frags, F, g.W, lw_off, epoly, bscan, lk, lv, le_cnt);
+  const int bbits = bits_for(std::max<int64_t>(NB - 1, 1));
+  if (L > 0)
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortPairs(t, sz, lk, lk2, lv, lv2, L, 0, 32 + bbits, st); }), "sort local edges");
+  if (NB > 0)
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, le_cnt, le_beg, NB, st); }), "scan local edges");
+  if (cudaMalloc(&c->run_seg, sizeof(int4) * std::max<int64_t>(L, 1)) != cudaSuccess ||
+      cudaMalloc(&c->run_poly, sizeof(int32_t) * std::max<int64_t>(L, 1)) != cudaSuccess)
+    return fail(set_error(SPADE_ERR_OOM, "build: local edge arrays"));
+  if (L > 0) LAUNCH(k_gather_edges, L, lv2, L, seg, epoly, c->run_seg, c->run_poly);
+  tmp.release(lk); tmp.release(lk2); tmp.release(lv); tmp.release(lv2); tmp.release(frags); tmp.release(lw_off);
 
-  // --- K-B3 scanline fill ---
+  // --- K-B3 corner owner sets ---
   uint64_t* ev2;
-  if (tmp.alloc(&ev2, NE)) return fail(set_error(SPADE_ERR_OOM, "build: events"));
-  if (NE > 0) {
-    TRYF(cub_call(tmp, st, [&](void* t, size_t& sz) {
-      return cub::DeviceRadixSort::SortKeys(t, sz, ev, ev2, NE, 0, jbits + pbits + cbits, st); }), "sort events");
-  }
+  ALLOC(ev2, NE, "events");
+  if (NE > 0)
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortKeys(t, sz, ev, ev2, NE, 0, jbits + pbits + kbits, st); }), "sort events");
   tmp.release(ev);
+  int32_t* corner;
+  ALLOC(corner, WH, "corner sets");
   unsigned long long *multi = nullptr, *nmulti;
   int64_t multi_cap = 1 << 20;
-  if (tmp.alloc(&nmulti, 1)) return fail(set_error(SPADE_ERR_OOM, "build: multi"));
+  ALLOC(nmulti, 1, "multi");
   unsigned long long h_nmulti = 0;
   for (int attempt = 0; attempt < 2; ++attempt) {
-    if (tmp.alloc(&multi, multi_cap)) return fail(set_error(SPADE_ERR_OOM, "build: multi list"));
+    ALLOC(multi, multi_cap, "multi list");
+    TRYF(cudaMemsetAsync(corner, 0xff, sizeof(int32_t) * WH, st), "memset");   // kEmpty
     TRYF(cudaMemsetAsync(nmulti, 0, 8, st), "memset");
     TRYF(cudaMemsetAsync(bad, 0, 4, st), "memset");
-    if (NE > 0) { LAUNCH(k_fill, (NE + 1) / 2, st, ev2, NE, g.W, pbits, cbits, bmap, c->fine, multi, nmulti, multi_cap, bad); }
+    if (NE > 0) LAUNCH(k_fill, (NE + 1) / 2, ev2, NE, g.W, pbits, kbits, corner, multi, nmulti, multi_cap, bad);
     TRYF(cudaMemcpyAsync(&h_nmulti, nmulti, 8, cudaMemcpyDeviceToHost, st), "nmulti");
     TRYF(cudaMemcpyAsync(&h_bad, bad, 4, cudaMemcpyDeviceToHost, st), "bad");
     TRYF(cudaStreamSynchronize(st), "sync fill");
@@ -522,45 +560,81 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
     if ((int64_t)h_nmulti <= multi_cap) break;
     tmp.release(multi);
     multi_cap = (int64_t)h_nmulti;
-    LAUNCH(k_reset_fill, WH, st, bmap, WH, c->fine);
   }
+  tmp.release(ev2);
   const int64_t M = (int64_t)h_nmulti;
   int64_t NG = 0;
+  int32_t* csets = nullptr; int2* crng = nullptr;
   if (M > 0) {
     unsigned long long* m2; int32_t* heads;
-    if (tmp.alloc(&m2, M) || tmp.alloc(&heads, M)) return fail(set_error(SPADE_ERR_OOM, "build: multi sort"));
-    TRYF(cub_call(tmp, st, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortKeys(t, sz, multi, m2, M, 0, 64, st); }), "sort multi");
-    LAUNCH(k_multi_heads, M, st, m2, M, heads);
-    TRYF(cub_call(tmp, st, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, heads, heads, M, st); }), "scan multi");
+    ALLOC(m2, M, "multi sort"); ALLOC(heads, M, "multi sort");
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortKeys(t, sz, multi, m2, M, 0, 64, st); }), "sort multi");
+    LAUNCH(k_multi_heads, M, m2, M, heads);
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, heads, heads, M, st); }), "scan multi");
     int32_t ng32 = 0;
     TRYF(cudaMemcpyAsync(&ng32, heads + M - 1, 4, cudaMemcpyDeviceToHost, st), "NG");
     TRYF(cudaStreamSynchronize(st), "sync multi");
     NG = ng32;
-    if (cudaMalloc(&c->sets, sizeof(int32_t) * M) != cudaSuccess || cudaMalloc(&c->set_rng, sizeof(int2) * NG) != cudaSuccess ||
-        cudaMalloc(&c->runs, sizeof(RunRec) * (NR + NG)) != cudaSuccess)
-      return fail(set_error(SPADE_ERR_OOM, "build: records"));
-    LAUNCH(k_multi_records, M, st, m2, M, heads, NR, c->sets, c->set_rng, c->runs, c->fine);
-  } else {
-    if (cudaMalloc(&c->runs, sizeof(RunRec) * imax64(NR, 1)) != cudaSuccess)
-      return fail(set_error(SPADE_ERR_OOM, "build: records"));
+    ALLOC(csets, M, "corner sets"); ALLOC(crng, NG, "corner sets");
+    LAUNCH(k_multi_sets, M, m2, M, heads, csets, crng, corner);
   }
-  if (NR > 0) { LAUNCH(k_runs, NR, st, NR, g.W, run_end, run_cnt, run_beg, c->fine, c->runs); }
+  tmp.release(multi);
+
+  // --- K-B4 K sets of boundary pixels, records, final canvas ---
+  int32_t *ksize, *kidx; int64_t* koff;
+  ALLOC(ksize, NB, "K sizes"); ALLOC(kidx, NB, "K sizes"); ALLOC(koff, NB + 1, "K offsets");
+  int64_t KT = 0; int64_t NK = 0;
+  if (NB > 0) {
+    LAUNCH(k_kset<0>, NB, NB, pix_of, g, corner, csets, crng, le_beg, le_cnt, c->run_seg, c->run_poly,
+           ksize, nullptr, nullptr, nullptr);
+    cub::TransformInputIterator<int64_t, BigSize, const int32_t*> it_sz(ksize, BigSize());
+    cub::TransformInputIterator<int32_t, BigFlag, const int32_t*> it_b(ksize, BigFlag());
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, it_sz, koff, NB, st); }), "scan K");
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, it_b, kidx, NB, st); }), "scan K idx");
+    int64_t last_off = 0; int32_t last_sz = 0, last_idx = 0;
+    TRYF(cudaMemcpyAsync(&last_off, koff + NB - 1, 8, cudaMemcpyDeviceToHost, st), "K");
+    TRYF(cudaMemcpyAsync(&last_sz, ksize + NB - 1, 4, cudaMemcpyDeviceToHost, st), "K");
+    TRYF(cudaMemcpyAsync(&last_idx, kidx + NB - 1, 4, cudaMemcpyDeviceToHost, st), "K");
+    TRYF(cudaStreamSynchronize(st), "sync K");
+    KT = last_off + (last_sz >= 2 ? last_sz : 0);
+    NK = last_idx + (last_sz >= 2 ? 1 : 0);
+  }
+  // final set storage: [corner owner sets (M entries, NG ranges)] ++ [K sets with |K| >= 2]
+  if (cudaMalloc(&c->sets, sizeof(int32_t) * std::max<int64_t>(M + KT, 1)) != cudaSuccess ||
+      cudaMalloc(&c->set_rng, sizeof(int2) * std::max<int64_t>(NG + NK, 1)) != cudaSuccess ||
+      cudaMalloc(&c->runs, sizeof(RunRec) * std::max<int64_t>(NB + NG, 1)) != cudaSuccess ||
+      cudaMalloc(&c->fine, sizeof(int32_t) * WH) != cudaSuccess)
+    return fail(set_error(SPADE_ERR_OOM, "build: records"));
+  if (M > 0) {
+    TRYF(cudaMemcpyAsync(c->sets, csets, sizeof(int32_t) * M, cudaMemcpyDeviceToDevice, st), "copy sets");
+    TRYF(cudaMemcpyAsync(c->set_rng, crng, sizeof(int2) * NG, cudaMemcpyDeviceToDevice, st), "copy sets");
+  }
+  if (NB > 0) {
+    LAUNCH(k_kset<1>, NB, NB, pix_of, g, corner, csets, crng, le_beg, le_cnt, c->run_seg, c->run_poly,
+           ksize, koff, c->sets + M, c->runs);
+    LAUNCH(k_kset_rng, NB, NB, ksize, koff, kidx, NG, M, c->set_rng, c->runs);
+  }
+  if (NG > 0) LAUNCH(k_multi_recs, NG, NG, NB, c->runs);
+  LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, c->fine);
 
   // --- K-B5 coarse tiles ---
   if (cudaMalloc(&c->coarse, sizeof(uint16_t) * ((int64_t)Wc * Hc + 16)) != cudaSuccess)
     return fail(set_error(SPADE_ERR_OOM, "build: coarse"));
+  TRYF(cudaMemsetAsync(c->coarse, 0, sizeof(uint16_t) * ((int64_t)Wc * Hc + 16), st), "memset");
   TRYF(cudaMemsetAsync(nmulti, 0, 8, st), "memset");
-  LAUNCH(k_coarse, (int64_t)Wc * Hc, st, c->fine, g.W, g.H, b, Wc, Hc, c->coarse, nmulti);
+  LAUNCH(k_coarse, (int64_t)Wc * Hc, c->fine, g.W, g.H, b, Wc, Hc, c->coarse, nmulti);
   unsigned long long h_mixed = 0;
   TRYF(cudaMemcpyAsync(&h_mixed, nmulti, 8, cudaMemcpyDeviceToHost, st), "mixed");
   TRYF(cudaStreamSynchronize(st), "sync coarse");
 #undef TRYF
+#undef ALLOC
+#undef LAUNCH
 
   c->empty = false;
-  c->num_runs = NR;
-  c->num_records = NR + NG;
+  c->num_runs = NB;
+  c->num_records = NB + NG;
   c->num_run_edges = L;
-  c->num_set_entries = M;
+  c->num_set_entries = M + KT;
   c->mixed_tile_frac = (double)h_mixed / ((double)Wc * Hc);
   CanvasDev& d = c->d;
   d.minx = (int32_t)g.minx; d.miny = (int32_t)g.miny;
@@ -568,7 +642,8 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   d.s = s; d.W = g.W; d.H = g.H; d.b = b; d.Wc = Wc; d.Hc = Hc;
   d.fine = c->fine; d.coarse = c->coarse; d.runs = c->runs; d.run_seg = c->run_seg; d.run_poly = c->run_poly;
   d.sets = c->sets; d.set_rng = c->set_rng;
-  (void)rc;
+  if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
+  if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));
   *out = c;
   return SPADE_OK;
 }

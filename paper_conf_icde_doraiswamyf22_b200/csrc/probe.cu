@@ -8,13 +8,13 @@
 // Map output via a unique slot per result + scan.
 //
 // B200 design:
-//   * one persistent CTA per SM, T threads; the coarse canvas (<= 64K uint16 tiles) is copied
-//     into shared memory once per CTA, so ~90% of points are classified by ONE LDS;
+//   * one persistent CTA per SM, T threads; the coarse canvas (<= 80K uint16 tiles) is copied
+//     into shared memory once per CTA, so most points are classified by ONE LDS;
 //   * points stream with 256-bit loads (LDG.E.256, L1::no_allocate, L2::evict_first);
 //   * points in mixed tiles gather one int32 fine pixel from L2 (evict_last policy); all gathers of
 //     a thread's batch are issued before any is consumed (memory-level parallelism);
 //   * boundary points are compacted per warp (ballot) into a shared-memory queue and evaluated
-//     32 at a time (one per lane) against the run's edges (exact int64 crossing test);
+//     32 at a time (one per lane) against the few edges touching their pixel (exact int64 tests);
 //   * COUNT: shared-memory per-polygon histogram (smem atomics), flushed once per CTA with
 //     64-bit global atomics; SELECT/PAIRS: CTA-aggregated output reservation (one global atomic
 //     per CTA batch) and direct stores.
@@ -30,7 +30,7 @@ enum Mode { kCountSmem = 0, kCountGlobal = 1, kSelect = 2, kPairs = 3 };
 constexpr int kQCap = 64;          // per-warp boundary queue entries (drained at >= 32)
 
 struct alignas(32) Vec4 { int4 a, b; };   // 4 points
-struct alignas(16) QEntry { int x, y, run; uint32_t pidx; };
+struct alignas(16) QEntry { int x, y, rec; uint32_t pidx; };
 
 __device__ __forceinline__ Vec4 ld_stream(const Vec4* p) {
   Vec4 r;
@@ -46,24 +46,30 @@ __device__ __forceinline__ uint64_t policy_evict_last() {
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
   return pol;
 }
-__device__ __forceinline__ int ld_fine(const int32_t* p, uint64_t pol) {
-  int r;
+__device__ __forceinline__ uint32_t ld_fine(const int32_t* p, uint64_t pol) {
+  uint32_t r;
   asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
   return r;
 }
 
-struct Params {
-  CanvasDev cv;
-  const int2* xy;
-  int64_t n;
-  int64_t head;               // points before the first 32-byte aligned one (0..3)
-  int64_t nvec;               // aligned 4-point vectors after the head
-  int64_t id_base;            // point id of xy[0]
+// Output side of a launch (what the sinks write).
+struct Out {
   unsigned long long* counts; // COUNT
   unsigned long long* total;  // SELECT/PAIRS: number of results (may exceed capacity)
   int64_t* out_ids;           // SELECT ids / PAIRS point ids
   int32_t* out_poly;          // PAIRS polygon ids
   int64_t cap;
+  int64_t id_base;            // point id of xy[0]
+};
+
+struct Params {
+  CanvasDev cv;
+  const CanvasDev* cvg;       // the same, in global memory (for the out-of-line exact test)
+  const int2* xy;
+  int64_t n;
+  int64_t head;               // points before the first 32-byte aligned one (0..3)
+  int64_t nvec;               // aligned 4-point vectors after the head
+  Out o;
 };
 
 // classification of one point before the fine gather:
@@ -76,112 +82,127 @@ __device__ __forceinline__ uint32_t classify_coarse(const CanvasDev& cv, const u
   if (t != kTileMixed) return t;
   return 0x80000000u | (fy * (uint32_t)cv.W + fx);
 }
-// after the gather: 0 = none, owner+1, or bit31 | record id (boundary run / multi-owner pixel)
+// after the gather: 0 = none, owner+1, or bit31 | record id (boundary pixel / multi-owner pixel)
 __device__ __forceinline__ uint32_t classify_fine(int32_t v) {
   return v >= 0 ? (uint32_t)v + 1u : (v == kEmpty ? 0u : (0x80000000u | (uint32_t)(-2 - v)));
 }
 
-// Exact point-in-polygon for a point on a boundary run (or multi-owner pixel) r:
-//   inside(p, P) = [P in term(r)] XOR parity_P(run edges)      (step 5)
+// Pixel-local exact test of one edge for point p in the pixel whose left side is x = X
+// (DESIGN.md "Canvas"):  cu(X, py) ^ cr(X, py) ^ cr(px, py), where cr is the half-open rightward
+// ray test of reading C1 and cu the upward ray test of the same perturbation.  Both share the
+// cross product o at (X, py).  Exact in int64 (all coordinates in [-2^30, 2^30)).
+__device__ __forceinline__ int local_bit(int4 e, int X, int px, int py) {
+  const int dx = e.z - e.x, dy = e.w - e.y;
+  const long long o = (long long)dx * (py - e.y) - (long long)dy * (X - e.x);
+  const long long o2 = o - (long long)dy * (px - X);
+  const bool ys = (e.y > py) != (e.w > py);
+  const bool xs = (e.x > X) != (e.z > X);
+  const bool crX = ys && (dy > 0 ? o > 0 : o < 0);
+  const bool crP = ys && (dy > 0 ? o2 > 0 : o2 < 0);
+  const bool cuX = xs && (dx > 0 ? (o < 0 || (o == 0 && dy > 0)) : (o > 0 || (o == 0 && dy < 0)));
+  return (int)(crX ^ crP ^ cuX);
+}
+
+// Exact point-in-polygon for a point on boundary pixel (or multi-owner pixel) record `rec`:
+//   inside(p, P) = [P in K] XOR parity_P(local_bit over P's edges touching the pixel)
 // emit(P) is called for every polygon containing the point, in increasing polygon order.
 template <class Emit>
-__device__ __forceinline__ void pip_eval(const CanvasDev& cv, int px, int py, uint32_t rec, Emit&& emit) {
-  const RunRec r = cv.runs[rec];
+__device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
+  const RunRec r = cv->runs[rec];
+  const int X = cv->minx + (int)((((uint32_t)px - (uint32_t)cv->minx) >> cv->s) << cv->s);
   int tn, tb = 0;
   const bool tsingle = r.term >= 0;
   if (tsingle) tn = 1;
   else if (r.term == kEmpty) tn = 0;
-  else { int2 g = cv.set_rng[-2 - r.term]; tb = g.x; tn = g.y; }
-  auto term_at = [&](int i) { return tsingle ? r.term : cv.sets[tb + i]; };
+  else { int2 g = cv->set_rng[-2 - r.term]; tb = g.x; tn = g.y; }
+  const int32_t* sets = cv->sets;
+  auto term_at = [&](int i) { return tsingle ? r.term : sets[tb + i]; };
   int ti = 0;
   auto finalize = [&](int P, int par) {
     while (ti < tn && term_at(ti) < P) emit(term_at(ti++));
     if (ti < tn && term_at(ti) == P) { par ^= 1; ++ti; }
     if (par) emit(P);
   };
+  const int4* seg = cv->run_seg;
+  const int32_t* poly = cv->run_poly;
   int cur = -1, par = 0;
   const int64_t e1 = r.edge_begin + r.edge_cnt;
   for (int64_t e = r.edge_begin; e < e1; ++e) {
-    const int p = __ldg(cv.run_poly + e);
+    const int p = __ldg(poly + e);
     if (p != cur) {
       if (cur >= 0) finalize(cur, par);
       cur = p; par = 0;
     }
-    par ^= edge_crosses(__ldg(cv.run_seg + e), px, py);
+    par ^= local_bit(__ldg(seg + e), X, px, py);
   }
   if (cur >= 0) finalize(cur, par);
   while (ti < tn) emit(term_at(ti++));
 }
 
 template <int MODE>
-struct SinkCtx {
-  unsigned int* hist;         // smem histogram (kCountSmem)
-  const Params* prm;
-};
-
-// Result of a point from the direct (non-queued) path; `owner` >= 0.
-template <int MODE>
-__device__ __forceinline__ void direct_hit_count(SinkCtx<MODE>& sc, int owner) {
-  if (MODE == kCountSmem) atomicAdd(&sc.hist[owner], 1u);
-  else atomicAdd(sc.prm->counts + owner, 1ull);
+__device__ __forceinline__ void count_hit(unsigned int* hist, unsigned long long* counts, int owner) {
+  if (MODE == kCountSmem) atomicAdd(&hist[owner], 1u);
+  else atomicAdd(counts + owner, 1ull);
 }
 
-// Emission from the rare paths (queue drains, unaligned head/tail): per-lane global atomics.
+// Emission from the rare paths (boundary queue drains, unaligned head/tail): per-lane atomics.
 template <int MODE>
-__device__ __forceinline__ void rare_emit_point(SinkCtx<MODE>& sc, const CanvasDev& cv, int x, int y, uint32_t rec,
-                                                int64_t pid) {
-  const Params& P = *sc.prm;
+__device__ __forceinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, const Out& o,
+                                                int x, int y, uint32_t rec, int64_t pid) {
   if (MODE == kCountSmem || MODE == kCountGlobal) {
-    pip_eval(cv, x, y, rec, [&](int p) { direct_hit_count<MODE>(sc, p); });
+    pip_eval(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, o.counts, p); });
   } else if (MODE == kSelect) {
     bool any = false;
-    pip_eval(cv, x, y, rec, [&](int) { any = true; });
+    pip_eval(cvg, x, y, rec, [&](int) { any = true; });
     if (any) {
-      unsigned long long q = atomicAdd(P.total, 1ull);
-      if ((int64_t)q < P.cap) P.out_ids[q] = pid;
+      unsigned long long q = atomicAdd(o.total, 1ull);
+      if ((int64_t)q < o.cap) o.out_ids[q] = pid;
     }
   } else {
-    pip_eval(cv, x, y, rec, [&](int p) {
-      unsigned long long q = atomicAdd(P.total, 1ull);
-      if ((int64_t)q < P.cap) { P.out_ids[q] = pid; P.out_poly[q] = p; }
+    pip_eval(cvg, x, y, rec, [&](int p) {
+      unsigned long long q = atomicAdd(o.total, 1ull);
+      if ((int64_t)q < o.cap) { o.out_ids[q] = pid; o.out_poly[q] = p; }
     });
   }
 }
 
 template <int MODE>
-__device__ __forceinline__ void rare_emit_owner(SinkCtx<MODE>& sc, int owner, int64_t pid) {
-  const Params& P = *sc.prm;
-  if (MODE == kCountSmem || MODE == kCountGlobal) direct_hit_count<MODE>(sc, owner);
+__device__ __forceinline__ void rare_emit_owner(unsigned int* hist, const Out& o, int owner, int64_t pid) {
+  if (MODE == kCountSmem || MODE == kCountGlobal) count_hit<MODE>(hist, o.counts, owner);
   else {
-    unsigned long long q = atomicAdd(P.total, 1ull);
-    if ((int64_t)q < P.cap) {
-      P.out_ids[q] = pid;
-      if (MODE == kPairs) P.out_poly[q] = owner;
+    unsigned long long q = atomicAdd(o.total, 1ull);
+    if ((int64_t)q < o.cap) {
+      o.out_ids[q] = pid;
+      if (MODE == kPairs) o.out_poly[q] = owner;
     }
   }
 }
 
 // One scalar point (unaligned head / tail): classify synchronously.
 template <int MODE>
-__device__ void scalar_point(SinkCtx<MODE>& sc, const CanvasDev& cv, const uint16_t* tiles, int x, int y, int64_t pid) {
+__device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, unsigned int* hist,
+                                          Out o, int x, int y, int64_t pid) {
+  const CanvasDev cv = *cvg;
   uint32_t c = classify_coarse(cv, tiles, x, y);
   if (c & 0x80000000u) c = classify_fine(cv.fine[c & 0x7fffffffu]);
   if (c == 0) return;
-  if (c & 0x80000000u) rare_emit_point<MODE>(sc, cv, x, y, c & 0x7fffffffu, pid);
-  else rare_emit_owner<MODE>(sc, (int)c - 1, pid);
+  if (c & 0x80000000u) rare_emit_point<MODE>(cvg, hist, o, x, y, c & 0x7fffffffu, pid);
+  else rare_emit_owner<MODE>(hist, o, (int)c - 1, pid);
 }
 
-// Evaluate up to 32 queued boundary points (one per lane).
+// Evaluate up to 32 queued boundary points (one per lane).  Out of line: it is the rare path and
+// keeping it out of the streaming loop keeps that loop's register footprint small.
 template <int MODE>
-__device__ __noinline__ void drain(SinkCtx<MODE>& sc, const CanvasDev& cv, QEntry* wq, int cnt, int lane) {
+__device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const QEntry* wq, int cnt, int lane,
+                                   unsigned int* hist, Out o) {
   if (lane < cnt) {
-    QEntry e = wq[lane];
-    rare_emit_point<MODE>(sc, cv, e.x, e.y, (uint32_t)e.run, sc.prm->id_base + (int64_t)e.pidx);
+    const QEntry e = wq[lane];
+    rare_emit_point<MODE>(cvg, hist, o, e.x, e.y, (uint32_t)e.rec, o.id_base + (int64_t)e.pidx);
   }
 }
 
 template <int MODE, int T, int U>
-__global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
+__global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
   const CanvasDev& cv = prm.cv;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -191,15 +212,13 @@ __global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
   uint16_t* tiles = (uint16_t*)smem;
   QEntry* queues = (QEntry*)(smem + tiles_bytes);
   unsigned char* rest = smem + tiles_bytes + NW * kQCap * sizeof(QEntry);
-  SinkCtx<MODE> sc;
-  sc.prm = &prm;
-  sc.hist = (unsigned int*)rest;
-  int* s_scan = (int*)rest;                                 // SELECT/PAIRS: [NW] sums + [NW] bases (int64)
-  long long* s_base = (long long*)(rest + 128 * sizeof(int));
+  unsigned int* hist = (unsigned int*)rest;               // COUNT (smem histogram)
+  int* s_scan = (int*)rest;                               // SELECT/PAIRS: [NW] warp sums
+  long long* s_base = (long long*)(rest + 128 * sizeof(int));   // [NW] warp output bases
 
   for (int i = tid; i < tiles_bytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
   if (MODE == kCountSmem)
-    for (int i = tid; i < cv.num_polys; i += T) sc.hist[i] = 0u;
+    for (int i = tid; i < cv.num_polys; i += T) hist[i] = 0u;
   __syncthreads();
 
   QEntry* wq = queues + warp * kQCap;
@@ -211,12 +230,12 @@ __global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
     const int64_t tail0 = prm.head + 4 * prm.nvec;
     const int64_t ntail = prm.n - tail0;
     if (lane < prm.head) {
-      int2 p = prm.xy[lane];
-      scalar_point<MODE>(sc, cv, tiles, p.x, p.y, prm.id_base + lane);
+      const int2 p = prm.xy[lane];
+      scalar_point<MODE>(prm.cvg, tiles, hist, prm.o, p.x, p.y, prm.o.id_base + lane);
     } else if (lane >= 4 && lane - 4 < ntail) {
-      int64_t i = tail0 + (lane - 4);
-      int2 p = prm.xy[i];
-      scalar_point<MODE>(sc, cv, tiles, p.x, p.y, prm.id_base + i);
+      const int64_t i = tail0 + (lane - 4);
+      const int2 p = prm.xy[i];
+      scalar_point<MODE>(prm.cvg, tiles, hist, prm.o, p.x, p.y, prm.o.id_base + i);
     }
   }
 
@@ -226,49 +245,58 @@ __global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
     Vec4 v[U];
 #pragma unroll
     for (int k = 0; k < U; ++k) {
-      int64_t idx = base + (int64_t)k * T + tid;
+      const int64_t idx = base + (int64_t)k * T + tid;
       if (idx < prm.nvec) v[k] = ld_stream(vp + idx);
-      else { v[k].a = make_int4(0, 0, 0, 0); v[k].b = v[k].a; }
+      else { v[k].a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v[k].b = v[k].a; }
     }
-    // phase A: coarse (shared memory) classification
+    // phase A: coarse (shared memory) classification.  Padding points (INT32_MIN) are outside
+    // every valid extent (vertices are >= -2^30), so they classify as 0.
     uint32_t c[4 * U];
+    uint32_t mix = 0;
 #pragma unroll
     for (int k = 0; k < U; ++k) {
-      const bool valid = base + (int64_t)k * T + tid < prm.nvec;
-      c[4 * k + 0] = valid ? classify_coarse(cv, tiles, v[k].a.x, v[k].a.y) : 0u;
-      c[4 * k + 1] = valid ? classify_coarse(cv, tiles, v[k].a.z, v[k].a.w) : 0u;
-      c[4 * k + 2] = valid ? classify_coarse(cv, tiles, v[k].b.x, v[k].b.y) : 0u;
-      c[4 * k + 3] = valid ? classify_coarse(cv, tiles, v[k].b.z, v[k].b.w) : 0u;
+      c[4 * k + 0] = classify_coarse(cv, tiles, v[k].a.x, v[k].a.y);
+      c[4 * k + 1] = classify_coarse(cv, tiles, v[k].a.z, v[k].a.w);
+      c[4 * k + 2] = classify_coarse(cv, tiles, v[k].b.x, v[k].b.y);
+      c[4 * k + 3] = classify_coarse(cv, tiles, v[k].b.z, v[k].b.w);
     }
+#pragma unroll
+    for (int q = 0; q < 4 * U; ++q) mix |= (c[q] >> 31) << q;
     // phase B: all fine-pixel gathers of the batch in flight together
-    int32_t f[4 * U];
+    if (mix) {
 #pragma unroll
-    for (int q = 0; q < 4 * U; ++q)
-      if (c[q] & 0x80000000u) f[q] = ld_fine(cv.fine + (c[q] & 0x7fffffffu), pol);
+      for (int q = 0; q < 4 * U; ++q)
+        if ((mix >> q) & 1u) c[q] = ld_fine(cv.fine + (c[q] & 0x7fffffffu), pol);
 #pragma unroll
-    for (int q = 0; q < 4 * U; ++q)
-      if (c[q] & 0x80000000u) c[q] = classify_fine(f[q]);
+      for (int q = 0; q < 4 * U; ++q)
+        if ((mix >> q) & 1u) c[q] = classify_fine((int32_t)c[q]);
+    }
     // phase C1: boundary points -> warp queue (ballot compaction), drained 32 at a time
+    uint32_t bnd = 0;
 #pragma unroll
-    for (int q = 0; q < 4 * U; ++q) {
-      const bool isb = (c[q] & 0x80000000u) != 0u;
-      const unsigned m = __ballot_sync(0xffffffffu, isb);
-      if (m) {
-        if (isb) {
-          const int k = q >> 2, h = q & 3;
-          const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
-          const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
-          const int64_t pidx = prm.head + 4 * (base + (int64_t)k * T + tid) + h;
-          wq[qn + __popc(m & ((1u << lane) - 1u))] = QEntry{x, y, (int)(c[q] & 0x7fffffffu), (uint32_t)pidx};
-        }
-        qn += __popc(m);
-        if (qn >= 32) {
-          __syncwarp();
-          drain<MODE>(sc, cv, wq, 32, lane);
-          __syncwarp();
-          if (lane < qn - 32) wq[lane] = wq[32 + lane];
-          __syncwarp();
-          qn -= 32;
+    for (int q = 0; q < 4 * U; ++q) bnd |= (c[q] >> 31) << q;
+    if (__any_sync(0xffffffffu, bnd != 0u)) {
+#pragma unroll
+      for (int q = 0; q < 4 * U; ++q) {
+        const bool isb = (bnd >> q) & 1u;
+        const unsigned m = __ballot_sync(0xffffffffu, isb);
+        if (m) {
+          if (isb) {
+            const int k = q >> 2, h = q & 3;
+            const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
+            const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
+            const int64_t pidx = prm.head + 4 * (base + (int64_t)k * T + tid) + h;
+            wq[qn + __popc(m & ((1u << lane) - 1u))] = QEntry{x, y, (int)(c[q] & 0x7fffffffu), (uint32_t)pidx};
+          }
+          qn += __popc(m);
+          if (qn >= 32) {
+            __syncwarp();
+            drain<MODE>(prm.cvg, wq, 32, lane, hist, prm.o);
+            __syncwarp();
+            if (lane < qn - 32) wq[lane] = wq[32 + lane];
+            __syncwarp();
+            qn -= 32;
+          }
         }
       }
     }
@@ -276,12 +304,12 @@ __global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
     if (MODE == kCountSmem || MODE == kCountGlobal) {
 #pragma unroll
       for (int q = 0; q < 4 * U; ++q)
-        if (c[q] != 0u && !(c[q] & 0x80000000u)) direct_hit_count<MODE>(sc, (int)c[q] - 1);
+        if (c[q] != 0u && !(c[q] >> 31)) count_hit<MODE>(hist, prm.o.counts, (int)c[q] - 1);
     } else {
       // CTA-aggregated reservation of output slots for this batch (Map with a scan)
       int h = 0;
 #pragma unroll
-      for (int q = 0; q < 4 * U; ++q) h += (c[q] != 0u && !(c[q] & 0x80000000u)) ? 1 : 0;
+      for (int q = 0; q < 4 * U; ++q) h += (c[q] != 0u && !(c[q] >> 31)) ? 1 : 0;
       int incl = h;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
@@ -298,7 +326,7 @@ __global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
           if (lane >= o) wincl += t;
         }
         unsigned long long gb = 0;
-        if (lane == 31 && wincl > 0) gb = atomicAdd(prm.total, (unsigned long long)wincl);
+        if (lane == 31 && wincl > 0) gb = atomicAdd(prm.o.total, (unsigned long long)wincl);
         gb = __shfl_sync(0xffffffffu, gb, 31);
         if (lane < NW) s_base[lane] = (long long)gb + (wincl - wsum);
       }
@@ -306,11 +334,11 @@ __global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
       int64_t pos = s_base[warp] + (incl - h);
 #pragma unroll
       for (int q = 0; q < 4 * U; ++q) {
-        if (c[q] != 0u && !(c[q] & 0x80000000u)) {
-          if (pos < prm.cap) {
+        if (c[q] != 0u && !(c[q] >> 31)) {
+          if (pos < prm.o.cap) {
             const int k = q >> 2, hh = q & 3;
-            prm.out_ids[pos] = prm.id_base + prm.head + 4 * (base + (int64_t)k * T + tid) + hh;
-            if (MODE == kPairs) prm.out_poly[pos] = (int)c[q] - 1;
+            prm.o.out_ids[pos] = prm.o.id_base + prm.head + 4 * (base + (int64_t)k * T + tid) + hh;
+            if (MODE == kPairs) prm.o.out_poly[pos] = (int)c[q] - 1;
           }
           ++pos;
         }
@@ -320,12 +348,12 @@ __global__ void __launch_bounds__(T, 1) k_probe(const Params prm) {
   }
   if (qn > 0) {
     __syncwarp();
-    drain<MODE>(sc, cv, wq, qn, lane);
+    drain<MODE>(prm.cvg, wq, qn, lane, hist, prm.o);
   }
   if (MODE == kCountSmem) {
     __syncthreads();
     for (int i = tid; i < cv.num_polys; i += T)
-      if (sc.hist[i]) atomicAdd(prm.counts + i, (unsigned long long)sc.hist[i]);
+      if (hist[i]) atomicAdd(prm.o.counts + i, (unsigned long long)hist[i]);
   }
 }
 
@@ -347,7 +375,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     const uintptr_t addr = (uintptr_t)p.xy;
     p.head = std::min<int64_t>(m, (int64_t)(((32 - (addr & 31)) & 31) / 8));
     p.nvec = (m - p.head) / 4;
-    p.id_base = base.id_base + off;
+    p.o.id_base = base.o.id_base + off;
     const int64_t chunks = (p.nvec + (int64_t)T * U - 1) / ((int64_t)T * U);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(sms, chunks));
     kern<<<grid, T, smem, st>>>(p);
@@ -360,11 +388,12 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
 
 constexpr size_t kSmemBudget = 227 * 1024;
 constexpr int kT = 1024, kU = 2;          // COUNT / SELECT (<= 64 registers per thread)
-constexpr int kTP = 512, kUP = 4;         // PAIRS
+constexpr int kTP = 1024, kUP = 2;        // PAIRS
 
 Params base_params(const spade_canvas* c) {
   Params p{};
   p.cv = c->d;
+  p.cvg = c->d_dev;
   return p;
 }
 
@@ -373,7 +402,7 @@ Params base_params(const spade_canvas* c) {
 int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts, cudaStream_t st) {
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
-  p.counts = (unsigned long long*)counts;
+  p.o.counts = (unsigned long long*)counts;
   const size_t fixed = (((size_t)c->d.Wc * c->d.Hc * 2 + 15) & ~(size_t)15) + (kT / 32) * kQCap * sizeof(QEntry);
   const size_t hist = (size_t)c->d.num_polys * 4;
   if (fixed + hist <= kSmemBudget) return launch<kCountSmem, kT, kU>(c, (const int2*)xy, n, p, hist, st);
@@ -384,7 +413,7 @@ int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t b
                   unsigned long long* d_total, cudaStream_t st) {
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
-  p.id_base = base; p.out_ids = out; p.cap = cap; p.total = d_total;
+  p.o.id_base = base; p.o.out_ids = out; p.o.cap = cap; p.o.total = d_total;
   return launch<kSelect, kT, kU>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
 }
 
@@ -392,7 +421,7 @@ int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t ba
                  int64_t cap, unsigned long long* d_total, cudaStream_t st) {
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
-  p.id_base = base; p.out_ids = opt; p.out_poly = opl; p.cap = cap; p.total = d_total;
+  p.o.id_base = base; p.o.out_ids = opt; p.o.out_poly = opl; p.o.cap = cap; p.o.total = d_total;
   return launch<kPairs, kTP, kUP>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
 }
 

@@ -95,7 +95,7 @@ void spade_canvas_free(spade_canvas* c) {
   if (!c) return;
   cudaDeviceSynchronize();
   cudaFree(c->fine); cudaFree(c->coarse); cudaFree(c->runs); cudaFree(c->run_seg); cudaFree(c->run_poly);
-  cudaFree(c->sets); cudaFree(c->set_rng);
+  cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->d_dev);
   delete c;
 }
 

@@ -12,16 +12,16 @@ namespace spade {
 // Fine canvas pixel (int32), the paper's discrete-canvas pixel (v0, vb) of P:111 reduced to the
 // polygon primitive:  v >= 0  -> the single polygon owning the whole (closed) pixel
 //                     v == -1 -> no polygon
-//                     v <= -2 -> record id  -2 - v  (a boundary run, or a multi-owner pixel)
+//                     v <= -2 -> record id  -2 - v  (a boundary pixel, or a multi-owner pixel)
 constexpr int32_t kEmpty = -1;
 constexpr int32_t kMultiMark = INT32_MIN;     // transient during the fill only
 // Coarse (shared-memory) tile entry, uint16: 0 = empty, 1..0xFFFE = owner+1, 0xFFFF = mixed
 constexpr uint16_t kTileEmpty = 0, kTileMixed = 0xFFFF;
 
-// Boundary-index record.  For a run of boundary pixels: its edges [edge_begin, +edge_cnt) in
-// run_seg/run_poly (sorted by polygon) and the polygon set `term` of the first non-boundary pixel
-// to its right.  For a multi-owner non-boundary pixel: edge_cnt = 0 and term = its owner set.
-// term >= 0: {term};  term == -1: {};  term <= -2: set index m = -2 - term into sets/set_rng.
+// Boundary-index record.  For a boundary pixel: the edges touching the closed pixel,
+// [edge_begin, +edge_cnt) in run_seg/run_poly (sorted by polygon), and the corrected corner set K
+// (`term`).  For a multi-owner non-boundary pixel: edge_cnt = 0 and term =
+// its owner set.  term >= 0: {term};  term == -1: {};  term <= -2: set m = -2 - term (sets/set_rng).
 struct RunRec {
   int64_t edge_begin;
   int32_t edge_cnt;
@@ -38,8 +38,8 @@ struct CanvasDev {            // passed by value to kernels
   int32_t num_polys;
   const int32_t* fine;
   const uint16_t* coarse;
-  const RunRec* runs;
-  const int4* run_seg;        // (ax, ay, bx, by)
+  const RunRec* runs;         // records: boundary pixels, then multi-owner pixels
+  const int4* run_seg;        // (ax, ay, bx, by) of the edges touching each boundary pixel
   const int32_t* run_poly;
   const int32_t* sets;        // concatenated sorted owner sets
   const int2* set_rng;        // (begin, count)
@@ -61,6 +61,7 @@ struct spade_canvas {
   int32_t* run_poly = nullptr;
   int32_t* sets = nullptr;
   int2* set_rng = nullptr;
+  spade::CanvasDev* d_dev = nullptr;   // copy of d in device memory (out-of-line exact test)
 };
 
 namespace spade {
@@ -71,16 +72,6 @@ __host__ __device__ __forceinline__ int64_t floor_div(int64_t a, int64_t b) {
   return (r != 0 && ((r < 0) != (b < 0))) ? q - 1 : q;
 }
 __host__ __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return -floor_div(-a, b); }
-
-// Half-open crossing test of PAPER-reading C1 for one edge (the exact point-edge test that the
-// paper's boundary index performs as a point-triangle test).  Coordinates of a valid
-// canvas are in [-2^30, 2^30) and the point lies inside the extent, so every difference fits in
-// int32 and both products in int64 (two 32x32->64 widening multiplies).
-__device__ __forceinline__ int edge_crosses(int4 e, int px, int py) {
-  if ((e.y > py) == (e.w > py)) return 0;
-  long long o = (long long)(e.z - e.x) * (long long)(py - e.y) - (long long)(e.w - e.y) * (long long)(px - e.x);
-  return e.w > e.y ? (o > 0) : (o < 0);
-}
 
 // error plumbing (spade_api.cu)
 int set_error(int code, const char* fmt, ...);
