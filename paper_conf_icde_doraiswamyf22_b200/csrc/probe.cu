@@ -20,6 +20,7 @@
 //     per CTA batch) and direct stores.
 #include <cstdint>
 #include <algorithm>
+#include <cstdlib>
 #include "spade_internal.cuh"
 
 namespace spade {
@@ -27,10 +28,9 @@ namespace spade {
 namespace {
 
 enum Mode { kCountSmem = 0, kCountGlobal = 1, kSelect = 2, kPairs = 3 };
-constexpr int kQCap = 64;          // per-warp boundary queue entries (drained at >= 32)
 
 struct alignas(32) Vec4 { int4 a, b; };   // 4 points
-struct alignas(16) QEntry { int x, y, rec; uint32_t pidx; };
+struct alignas(8) QEntry { uint32_t rec, pidx; };   // boundary point: its record and index
 
 __device__ __forceinline__ Vec4 ld_stream(const Vec4* p) {
   Vec4 r;
@@ -82,10 +82,10 @@ __device__ __forceinline__ uint32_t classify_coarse(const CanvasDev& cv, const u
   if (t != kTileMixed) return t;
   return 0x80000000u | (fy * (uint32_t)cv.W + fx);
 }
-// after the gather: 0 = none, owner+1, or bit31 | record id (boundary pixel / multi-owner pixel)
-__device__ __forceinline__ uint32_t classify_fine(int32_t v) {
-  return v >= 0 ? (uint32_t)v + 1u : (v == kEmpty ? 0u : (0x80000000u | (uint32_t)(-2 - v)));
-}
+// Point class c after the fine gather: c = fine pixel value + 1, i.e. 0 = no polygon,
+// 1 .. 2^31-1 = owner + 1, and >= 2^31 = record ~c (boundary / multi-owner pixel).  Uniform
+// coarse tiles give the same encoding directly (tile value = owner + 1, 0 = empty).
+__device__ __forceinline__ uint32_t classify_fine(int32_t v) { return (uint32_t)v + 1u; }
 
 // Pixel-local exact test of one edge for point p in the pixel whose left side is x = X
 // (DESIGN.md "Canvas"):  cu(X, py) ^ cr(X, py) ^ cr(px, py), where cr is the half-open rightward
@@ -186,43 +186,61 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
   uint32_t c = classify_coarse(cv, tiles, x, y);
   if (c & 0x80000000u) c = classify_fine(cv.fine[c & 0x7fffffffu]);
   if (c == 0) return;
-  if (c & 0x80000000u) rare_emit_point<MODE>(cvg, hist, o, x, y, c & 0x7fffffffu, pid);
+  if (c & 0x80000000u) rare_emit_point<MODE>(cvg, hist, o, x, y, ~c, pid);
   else rare_emit_owner<MODE>(hist, o, (int)c - 1, pid);
 }
 
-// Evaluate up to 32 queued boundary points (one per lane).  Out of line: it is the rare path and
-// keeping it out of the streaming loop keeps that loop's register footprint small.
+// Evaluate up to 32 queued boundary points (one per lane); the point is re-read here (L2) so the
+// streaming loop never waits on it.  Out of line: it is the rare path and keeping it out of the
+// streaming loop keeps that loop's register footprint small.
 template <int MODE>
-__device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const QEntry* wq, int cnt, int lane,
-                                   unsigned int* hist, Out o) {
+__device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const int2* __restrict__ xy, const QEntry* wq,
+                                   int cnt, int lane, unsigned int* hist, Out o) {
   if (lane < cnt) {
     const QEntry e = wq[lane];
-    rare_emit_point<MODE>(cvg, hist, o, e.x, e.y, (uint32_t)e.rec, o.id_base + (int64_t)e.pidx);
+    const int2 p = __ldg(xy + e.pidx);
+    rare_emit_point<MODE>(cvg, hist, o, p.x, p.y, e.rec, o.id_base + (int64_t)e.pidx);
   }
 }
 
-template <int MODE, int T, int U>
+// Per-CTA shared-memory layout (bytes, in order):
+//   tiles   (Wc*Hc + 1) uint16, rounded up to 16 B; entry Wc*Hc is an always-empty sentinel
+//   queues  NW * QCAP QEntry (boundary points per warp; QCAP = 32 + 32 * points per thread)
+//   COUNT   kHC copies of (P + 1) uint32 bins (bin P = "no polygon" trash bin)
+//   SELECT/PAIRS: 128 int warp sums + 32 int64 warp bases
+constexpr int kHC = 8;             // histogram copies (lane & 7): spreads same-polygon atomics
+
+__host__ __device__ constexpr int qcap_for(int U) { return 32 + 32 * 4 * U; }
+__host__ __device__ __forceinline__ size_t tiles_bytes_for(int ntiles) { return (((size_t)ntiles + 1) * 2 + 15) & ~(size_t)15; }
+
+template <int MODE, int T, int U, int PF>
 __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
   const CanvasDev& cv = prm.cv;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int NW = T / 32;
-  const int ntiles = cv.Wc * cv.Hc;
-  const int tiles_bytes = ((ntiles * 2) + 15) & ~15;
+  constexpr int NPT = 4 * U;                      // points per thread per batch
+  constexpr int QCAP = 32 + 32 * NPT;             // < 32 left over + one full batch
+  const uint32_t ntiles = (uint32_t)(cv.Wc * cv.Hc);
+  const uint32_t tbytes = (uint32_t)tiles_bytes_for((int)ntiles);
   uint16_t* tiles = (uint16_t*)smem;
-  QEntry* queues = (QEntry*)(smem + tiles_bytes);
-  unsigned char* rest = smem + tiles_bytes + NW * kQCap * sizeof(QEntry);
-  unsigned int* hist = (unsigned int*)rest;               // COUNT (smem histogram)
-  int* s_scan = (int*)rest;                               // SELECT/PAIRS: [NW] warp sums
-  long long* s_base = (long long*)(rest + 128 * sizeof(int));   // [NW] warp output bases
+  QEntry* queues = (QEntry*)(smem + tbytes);
+  unsigned char* rest = smem + tbytes + NW * QCAP * sizeof(QEntry);
+  const uint32_t P = (uint32_t)cv.num_polys;
+  unsigned int* hist = (unsigned int*)rest;                       // COUNT
+  unsigned int* myhist = hist + (lane & (kHC - 1)) * (P + 1);
+  int* s_scan = (int*)rest;                                       // SELECT/PAIRS
+  long long* s_base = (long long*)(rest + 128 * sizeof(int));
 
-  for (int i = tid; i < tiles_bytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
+  for (uint32_t i = tid; i < tbytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
   if (MODE == kCountSmem)
-    for (int i = tid; i < cv.num_polys; i += T) hist[i] = 0u;
+    for (uint32_t i = tid; i < kHC * (P + 1); i += T) hist[i] = 0u;
   __syncthreads();
 
-  QEntry* wq = queues + warp * kQCap;
-  int qn = 0;                                   // warp-uniform
+  QEntry* wq = queues + warp * QCAP;
+  __shared__ int s_qn[NW];                      // per-warp queue fill
+  if (lane == 0) s_qn[warp] = 0;
+  __syncwarp();
   const uint64_t pol = policy_evict_last();
 
   // unaligned head and tail (< 8 points): CTA 0, warp 0
@@ -231,85 +249,107 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
     const int64_t ntail = prm.n - tail0;
     if (lane < prm.head) {
       const int2 p = prm.xy[lane];
-      scalar_point<MODE>(prm.cvg, tiles, hist, prm.o, p.x, p.y, prm.o.id_base + lane);
+      scalar_point<MODE>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + lane);
     } else if (lane >= 4 && lane - 4 < ntail) {
       const int64_t i = tail0 + (lane - 4);
       const int2 p = prm.xy[i];
-      scalar_point<MODE>(prm.cvg, tiles, hist, prm.o, p.x, p.y, prm.o.id_base + i);
+      scalar_point<MODE>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + i);
     }
   }
 
   const Vec4* vp = (const Vec4*)(prm.xy + prm.head);
-  const int64_t chunk = (int64_t)T * U;
-  for (int64_t base = (int64_t)blockIdx.x * chunk; base < prm.nvec; base += (int64_t)gridDim.x * chunk) {
-    Vec4 v[U];
+  const uint32_t nvec = (uint32_t)prm.nvec;      // launches hold < 2^31 points
+  const uint32_t chunk = (uint32_t)(T * U);
+  const uint32_t minx = (uint32_t)cv.minx, miny = (uint32_t)cv.miny;
+  const uint32_t extw = cv.extw, exth = cv.exth;
+  const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
+  auto load_batch = [&](Vec4 (&v)[U], uint32_t base) {
+    if (base + chunk <= nvec) {                  // CTA-uniform: full batch, no bounds checks
 #pragma unroll
-    for (int k = 0; k < U; ++k) {
-      const int64_t idx = base + (int64_t)k * T + tid;
-      if (idx < prm.nvec) v[k] = ld_stream(vp + idx);
-      else { v[k].a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v[k].b = v[k].a; }
-    }
-    // phase A: coarse (shared memory) classification.  Padding points (INT32_MIN) are outside
-    // every valid extent (vertices are >= -2^30), so they classify as 0.
-    uint32_t c[4 * U];
-    uint32_t mix = 0;
+      for (int k = 0; k < U; ++k) v[k] = ld_stream(vp + base + k * T + tid);
+    } else {
 #pragma unroll
-    for (int k = 0; k < U; ++k) {
-      c[4 * k + 0] = classify_coarse(cv, tiles, v[k].a.x, v[k].a.y);
-      c[4 * k + 1] = classify_coarse(cv, tiles, v[k].a.z, v[k].a.w);
-      c[4 * k + 2] = classify_coarse(cv, tiles, v[k].b.x, v[k].b.y);
-      c[4 * k + 3] = classify_coarse(cv, tiles, v[k].b.z, v[k].b.w);
-    }
-#pragma unroll
-    for (int q = 0; q < 4 * U; ++q) mix |= (c[q] >> 31) << q;
-    // phase B: all fine-pixel gathers of the batch in flight together
-    if (mix) {
-#pragma unroll
-      for (int q = 0; q < 4 * U; ++q)
-        if ((mix >> q) & 1u) c[q] = ld_fine(cv.fine + (c[q] & 0x7fffffffu), pol);
-#pragma unroll
-      for (int q = 0; q < 4 * U; ++q)
-        if ((mix >> q) & 1u) c[q] = classify_fine((int32_t)c[q]);
-    }
-    // phase C1: boundary points -> warp queue (ballot compaction), drained 32 at a time
-    uint32_t bnd = 0;
-#pragma unroll
-    for (int q = 0; q < 4 * U; ++q) bnd |= (c[q] >> 31) << q;
-    if (__any_sync(0xffffffffu, bnd != 0u)) {
-#pragma unroll
-      for (int q = 0; q < 4 * U; ++q) {
-        const bool isb = (bnd >> q) & 1u;
-        const unsigned m = __ballot_sync(0xffffffffu, isb);
-        if (m) {
-          if (isb) {
-            const int k = q >> 2, h = q & 3;
-            const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
-            const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
-            const int64_t pidx = prm.head + 4 * (base + (int64_t)k * T + tid) + h;
-            wq[qn + __popc(m & ((1u << lane) - 1u))] = QEntry{x, y, (int)(c[q] & 0x7fffffffu), (uint32_t)pidx};
-          }
-          qn += __popc(m);
-          if (qn >= 32) {
-            __syncwarp();
-            drain<MODE>(prm.cvg, wq, 32, lane, hist, prm.o);
-            __syncwarp();
-            if (lane < qn - 32) wq[lane] = wq[32 + lane];
-            __syncwarp();
-            qn -= 32;
-          }
-        }
+      for (int k = 0; k < U; ++k) {
+        const uint32_t idx = base + k * T + tid;
+        if (idx < nvec) v[k] = ld_stream(vp + idx);
+        else { v[k].a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v[k].b = v[k].a; }
       }
     }
-    // phase C2: direct hits
-    if (MODE == kCountSmem || MODE == kCountGlobal) {
+  };
+  const uint32_t stride = gridDim.x * chunk;
+  Vec4 nxt[U];
+  if (PF && blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
+  for (uint32_t base = blockIdx.x * chunk; base < nvec; base += stride) {
+    Vec4 v[U];
+    if (PF) {
 #pragma unroll
-      for (int q = 0; q < 4 * U; ++q)
-        if (c[q] != 0u && !(c[q] >> 31)) count_hit<MODE>(hist, prm.o.counts, (int)c[q] - 1);
+      for (int k = 0; k < U; ++k) v[k] = nxt[k];
+      if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight while this one is processed
+    } else {
+      load_batch(v, base);
+    }
+    // phase A: coarse (shared memory) lookup, branch-free; points outside the extent read the
+    // always-empty sentinel tile.  c = 0 (none) | owner + 1 | fine pixel index (mixed tile)
+    uint32_t c[NPT];
+    uint32_t mix = 0;
+#pragma unroll
+    for (int q = 0; q < NPT; ++q) {
+      const int k = q >> 2, h = q & 3;
+      const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
+      const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
+      const uint32_t ux = (uint32_t)x - minx, uy = (uint32_t)y - miny;
+      uint32_t ti = (uy >> sb) * Wc + (ux >> sb);
+      ti = (ux <= extw && uy <= exth) ? ti : ntiles;
+      const uint32_t t = tiles[ti];
+      const bool m = t == kTileMixed;
+      c[q] = m ? (uy >> s) * W + (ux >> s) : t;
+      mix |= (m ? 1u : 0u) << q;
+    }
+    // phase B: fine pixels of mixed tiles; all gathers of the batch in flight together
+#pragma unroll
+    for (int q = 0; q < NPT; ++q)
+      if ((mix >> q) & 1u) c[q] = classify_fine((int32_t)ld_fine(cv.fine + c[q], pol));
+    // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
+    uint32_t bnd = 0;
+#pragma unroll
+    for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
+    // phase C1: boundary points -> warp queue (smem atomic reservation), drained 32 at a time
+    if (__any_sync(0xffffffffu, bnd != 0u)) {
+      if (bnd) {
+        int pos = atomicAdd(&s_qn[warp], __popc(bnd));
+#pragma unroll
+        for (int q = 0; q < NPT; ++q)
+          if ((bnd >> q) & 1u) {
+            const int k = q >> 2, h = q & 3;
+            wq[pos++] = QEntry{~c[q], (uint32_t)prm.head + 4 * (base + k * T + tid) + h};
+          }
+      }
+      __syncwarp();
+      int qn = s_qn[warp];
+      if (qn >= 32) {
+        do {
+          drain<MODE>(prm.cvg, prm.xy, wq + qn - 32, 32, lane, myhist, prm.o);
+          qn -= 32;
+        } while (qn >= 32);
+        __syncwarp();
+        if (lane == 0) s_qn[warp] = qn;
+      }
+      __syncwarp();
+    }
+    // phase C2: direct hits
+    if (MODE == kCountSmem) {
+      // branch-free: non-hits (0 - 1 = 0xFFFFFFFF, boundary >= 2^31 - 1) go to the trash bin P
+#pragma unroll
+      for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P)], 1u);
+    } else if (MODE == kCountGlobal) {
+#pragma unroll
+      for (int q = 0; q < NPT; ++q)
+        if (c[q] != 0u && !(c[q] >> 31)) atomicAdd(prm.o.counts + (c[q] - 1u), 1ull);
     } else {
       // CTA-aggregated reservation of output slots for this batch (Map with a scan)
       int h = 0;
 #pragma unroll
-      for (int q = 0; q < 4 * U; ++q) h += (c[q] != 0u && !(c[q] >> 31)) ? 1 : 0;
+      for (int q = 0; q < NPT; ++q) h += (c[q] != 0u && !(c[q] >> 31)) ? 1 : 0;
       int incl = h;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
@@ -333,11 +373,11 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
       __syncthreads();
       int64_t pos = s_base[warp] + (incl - h);
 #pragma unroll
-      for (int q = 0; q < 4 * U; ++q) {
+      for (int q = 0; q < NPT; ++q) {
         if (c[q] != 0u && !(c[q] >> 31)) {
           if (pos < prm.o.cap) {
             const int k = q >> 2, hh = q & 3;
-            prm.o.out_ids[pos] = prm.o.id_base + prm.head + 4 * (base + (int64_t)k * T + tid) + hh;
+            prm.o.out_ids[pos] = prm.o.id_base + prm.head + 4 * (int64_t)(base + k * T + tid) + hh;
             if (MODE == kPairs) prm.o.out_poly[pos] = (int)c[q] - 1;
           }
           ++pos;
@@ -346,27 +386,29 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
       __syncthreads();   // s_scan / s_base reuse next batch
     }
   }
-  if (qn > 0) {
-    __syncwarp();
-    drain<MODE>(prm.cvg, wq, qn, lane, hist, prm.o);
-  }
+  __syncwarp();
+  if (s_qn[warp] > 0) drain<MODE>(prm.cvg, prm.xy, wq, s_qn[warp], lane, myhist, prm.o);
   if (MODE == kCountSmem) {
     __syncthreads();
-    for (int i = tid; i < cv.num_polys; i += T)
-      if (hist[i]) atomicAdd(prm.o.counts + i, (unsigned long long)hist[i]);
+    for (uint32_t i = tid; i < P; i += T) {
+      unsigned long long sum = 0;
+#pragma unroll
+      for (int k = 0; k < kHC; ++k) sum += hist[k * (P + 1) + i];
+      if (sum) atomicAdd(prm.o.counts + i, sum);
+    }
   }
 }
 
-template <int MODE, int T, int U>
+template <int MODE, int T, int U, int PF>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
   const int ntiles = c->d.Wc * c->d.Hc;
-  const size_t smem = (((size_t)ntiles * 2 + 15) & ~(size_t)15) + (T / 32) * kQCap * sizeof(QEntry) + extra_smem;
-  auto kern = k_probe<MODE, T, U>;
+  const size_t smem = tiles_bytes_for(ntiles) + (T / 32) * qcap_for(U) * sizeof(QEntry) + extra_smem;
+  auto kern = k_probe<MODE, T, U, PF>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
   const int sms = device_sm_count();
-  // launches of at most 2^31 points (queue entries hold 32-bit point offsets)
-  const int64_t kMax = 1ll << 31;
+  // launches of fewer than 2^31 points (32-bit vector indices and queue point offsets)
+  const int64_t kMax = (1ll << 31) - 64;
   for (int64_t off = 0; off < n; off += kMax) {
     const int64_t m = std::min(kMax, n - off);
     Params p = base;
@@ -387,8 +429,38 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
 }
 
 constexpr size_t kSmemBudget = 227 * 1024;
-constexpr int kT = 1024, kU = 2;          // COUNT / SELECT (<= 64 registers per thread)
-constexpr int kTP = 1024, kUP = 2;        // PAIRS
+
+// Launch-shape variants of the probe (threads per CTA, 4-point vectors per thread per batch,
+// register double-buffered prefetch of the next batch).  SPADE_PROBE_VARIANT=<i> overrides the
+// default for tuning runs; the default is the measured best.
+struct Variant { int T, U, PF; };
+constexpr Variant kVariants[] = {{1024, 2, 0}, {768, 2, 1}, {512, 4, 1}, {1024, 1, 1}, {512, 2, 1}};
+constexpr int kDefaultVariant = 3;
+
+int variant_index() {
+  static int v = [] {
+    const char* e = getenv("SPADE_PROBE_VARIANT");
+    int i = e ? atoi(e) : kDefaultVariant;
+    return (i >= 0 && i < (int)(sizeof(kVariants) / sizeof(kVariants[0]))) ? i : kDefaultVariant;
+  }();
+  return v;
+}
+
+template <int MODE>
+int launch_variant(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
+  switch (variant_index()) {
+    case 0: return launch<MODE, 1024, 2, 0>(c, xy, n, p, extra, st);
+    case 1: return launch<MODE, 768, 2, 1>(c, xy, n, p, extra, st);
+    case 2: return launch<MODE, 512, 4, 1>(c, xy, n, p, extra, st);
+    case 3: return launch<MODE, 1024, 1, 1>(c, xy, n, p, extra, st);
+    default: return launch<MODE, 512, 2, 1>(c, xy, n, p, extra, st);
+  }
+}
+
+size_t fixed_smem(const spade_canvas* c) {
+  const Variant v = kVariants[variant_index()];
+  return tiles_bytes_for(c->d.Wc * c->d.Hc) + (v.T / 32) * qcap_for(v.U) * sizeof(QEntry);
+}
 
 Params base_params(const spade_canvas* c) {
   Params p{};
@@ -403,10 +475,9 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.counts = (unsigned long long*)counts;
-  const size_t fixed = (((size_t)c->d.Wc * c->d.Hc * 2 + 15) & ~(size_t)15) + (kT / 32) * kQCap * sizeof(QEntry);
-  const size_t hist = (size_t)c->d.num_polys * 4;
-  if (fixed + hist <= kSmemBudget) return launch<kCountSmem, kT, kU>(c, (const int2*)xy, n, p, hist, st);
-  return launch<kCountGlobal, kT, kU>(c, (const int2*)xy, n, p, 0, st);
+  const size_t hist = (size_t)kHC * (c->d.num_polys + 1) * 4;
+  if (fixed_smem(c) + hist <= kSmemBudget) return launch_variant<kCountSmem>(c, (const int2*)xy, n, p, hist, st);
+  return launch_variant<kCountGlobal>(c, (const int2*)xy, n, p, 0, st);
 }
 
 int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* out, int64_t cap,
@@ -414,7 +485,7 @@ int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t b
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = out; p.o.cap = cap; p.o.total = d_total;
-  return launch<kSelect, kT, kU>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
+  return launch_variant<kSelect>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
 }
 
 int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* opt, int32_t* opl,
@@ -422,7 +493,7 @@ int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t ba
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = opt; p.o.out_poly = opl; p.o.cap = cap; p.o.total = d_total;
-  return launch<kPairs, kTP, kUP>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
+  return launch_variant<kPairs>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
 }
 
 }  // namespace spade
