@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU oracle sample time")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu/clocks)")
+    ap.add_argument("--dense", action="store_true", help="force the dense fine-canvas layout (A/B runs)")
     return ap.parse_args()
 
 
@@ -205,7 +206,7 @@ def main():
     # canvas build (timed separately; not part of a step)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    cv = sp.Canvas(w.polys, max_dim=w.max_dim)
+    cv = sp.Canvas(w.polys, max_dim=w.max_dim, dense=a.dense)
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
     info = cv.info()

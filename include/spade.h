@@ -60,7 +60,12 @@ enum {
 typedef struct {
     int32_t log2_pixel;   /* -1 = auto                                    */
     int32_t max_dim;      /* used when log2_pixel == -1; 0 means 4096     */
+    int32_t flags;        /* SPADE_CANVAS_* bits; 0 = defaults            */
 } spade_canvas_params;
+
+/* flags: keep the dense W x H fine canvas as the probe's second level even when the compact
+ * mixed-tile layout applies (for tests / comparisons; results are identical). */
+#define SPADE_CANVAS_DENSE 1
 
 /* Build the discrete canvas + boundary index for a polygon set (P:113-123 canvas creation,
  * Sec. 4.2; P:146 and P:268 boundary index, Sec. 4.3 / 5.5).
@@ -72,7 +77,7 @@ typedef struct {
  *                        several outer rings, self-intersections and degenerate rings
  *                        (even-odd over all rings, reading C2); polygons may overlap (C3).
  *   num_polys     P >= 0
- *   prm           NULL = defaults {-1, 4096}
+ *   prm           NULL = defaults {-1, 4096, 0}
  *   out           receives the canvas handle (NULL on error)
  * The input buffers may be freed once this returns.  Synchronises `stream` (a few times: sizes
  * are data dependent).  Errors: INVALID_ARG, COORD_RANGE, OOM, CUDA. */

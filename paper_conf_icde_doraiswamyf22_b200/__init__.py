@@ -41,7 +41,10 @@ class CapacityError(SpadeError):
 
 
 class CanvasParams(ctypes.Structure):
-    _fields_ = [("log2_pixel", ctypes.c_int32), ("max_dim", ctypes.c_int32)]
+    _fields_ = [("log2_pixel", ctypes.c_int32), ("max_dim", ctypes.c_int32), ("flags", ctypes.c_int32)]
+
+
+SPADE_CANVAS_DENSE = 1
 
 
 def load(path: str | None = None):
@@ -119,14 +122,14 @@ def launch_count() -> int:
 class Canvas:
     """Discrete canvas + boundary index of a polygon set (owns device memory)."""
 
-    def __init__(self, polys, log2_pixel: int = -1, max_dim: int = 4096, stream=None):
+    def __init__(self, polys, log2_pixel: int = -1, max_dim: int = 4096, dense: bool = False, stream=None):
         torch = _torch()
         lib = load()
         ring_xy = _dev(polys["ring_xy"], torch.int32, 2)
         ring_off = _dev(polys["ring_off"], torch.int64)
         poly_ring_off = _dev(polys["poly_ring_off"], torch.int64)
         self.num_polys = int(poly_ring_off.numel()) - 1
-        prm = CanvasParams(log2_pixel, max_dim)
+        prm = CanvasParams(log2_pixel, max_dim, SPADE_CANVAS_DENSE if dense else 0)
         h = ctypes.c_void_p()
         rc = lib.spade_build_canvas(ctypes.c_void_p(ring_xy.data_ptr()), ctypes.c_void_p(ring_off.data_ptr()),
                                     ctypes.c_void_p(poly_ring_off.data_ptr()), self.num_polys, ctypes.byref(prm),

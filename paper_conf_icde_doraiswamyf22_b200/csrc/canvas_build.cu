@@ -331,8 +331,9 @@ __global__ void k_multi_recs(int64_t NG, int64_t NB, RunRec* __restrict__ recs) 
     recs[NB + g] = RunRec{0, 0, (int32_t)(-2 - g)};
 }
 
+// K-B5: tile summary.  tval = owner + 1 / 0 for uniform tiles; mixed tiles flagged in tmix.
 __global__ void k_coarse(const int32_t* __restrict__ fine, int W, int H, int b, int Wc, int Hc,
-                         uint16_t* __restrict__ coarse, unsigned long long* __restrict__ nmixed) {
+                         int32_t* __restrict__ tval, int32_t* __restrict__ tmix) {
   int64_t NT = (int64_t)Wc * Hc;
   const int B = 1 << b;
   for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < NT; t += (int64_t)gridDim.x * kBT) {
@@ -344,10 +345,39 @@ __global__ void k_coarse(const int32_t* __restrict__ fine, int W, int H, int b, 
     for (int j = j0; j < j1 && uni; ++j)
       for (int i = i0; i < i1; ++i)
         if (fine[(int64_t)j * W + i] != v0) { uni = false; break; }
-    uint16_t c;
-    if (uni && (int64_t)v0 + 1 < (int64_t)kTileMixed) c = (uint16_t)(v0 + 1);
-    else { c = kTileMixed; atomicAdd(nmixed, 1ull); }
-    coarse[t] = c;
+    tval[t] = uni ? v0 + 1 : -1;
+    tmix[t] = uni ? 0 : 1;
+  }
+}
+
+// coarse entries; compact layout copies each mixed tile's pixels into block m = mscan[t]
+__global__ void k_coarse_final(const int32_t* __restrict__ tval, const int32_t* __restrict__ mscan, int Wc, int Hc,
+                               int compact, uint32_t owner_lim, uint16_t* __restrict__ coarse) {
+  const int64_t NT1 = (int64_t)(Wc + 1) * (Hc + 1);          // with the sentinel column and row
+  for (int64_t u = blockIdx.x * (int64_t)kBT + threadIdx.x; u < NT1; u += (int64_t)gridDim.x * kBT) {
+    const int tx = (int)(u % (Wc + 1)), ty = (int)(u / (Wc + 1));
+    uint16_t e = kTileEmpty;
+    if (tx < Wc && ty < Hc) {
+      const int64_t t = (int64_t)ty * Wc + tx;
+      const int32_t v = tval[t];
+      if (v >= 0 && (uint32_t)v < owner_lim) e = (uint16_t)v;
+      else e = compact ? (uint16_t)(kTileMixedCompact | (uint32_t)mscan[t]) : kTileMixed;
+    }
+    coarse[u] = e;
+  }
+}
+
+__global__ void k_compact(const int32_t* __restrict__ fine, int W, int H, int b, int Wc, const int32_t* __restrict__ tval,
+                          const int32_t* __restrict__ mscan, int64_t NT, uint32_t owner_lim, int32_t* __restrict__ cfine) {
+  const int B = 1 << b;
+  const int64_t NP = NT << (2 * b);
+  for (int64_t q = blockIdx.x * (int64_t)kBT + threadIdx.x; q < NP; q += (int64_t)gridDim.x * kBT) {
+    const int64_t t = q >> (2 * b);
+    const int32_t v = tval[t];
+    if (v >= 0 && (uint32_t)v < owner_lim) continue;       // uniform tile: not stored
+    const int within = (int)(q & ((1 << (2 * b)) - 1));
+    const int i = (int)(t % Wc) * B + (within & (B - 1)), j = (int)(t / Wc) * B + (within >> b);
+    cfine[((int64_t)mscan[t] << (2 * b)) + within] = (i < W && j < H) ? fine[(int64_t)j * W + i] : kEmpty;
   }
 }
 
@@ -466,17 +496,24 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
     s = 0;
     while (std::max((ew >> s) + 1, (eh >> s) + 1) > max_dim) ++s;
   }
+  s = std::min(s, 29);
   Geo g;
   g.minx = h_ext[0]; g.miny = h_ext[1]; g.s = s; g.S = 1ll << s;
-  int64_t W64 = (ew >> s) + 1, H64 = (eh >> s) + 1;
+  const int64_t W0 = (ew >> s) + 1, H0 = (eh >> s) + 1;
+  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (160 KB),
+  // including one sentinel column and row of always-empty tiles (the probe clamps tile
+  // coordinates into them instead of testing the extent); tile side 2^b pixels, s + b <= 30
+  const int64_t kMaxTiles = 81920;
+  int b = 0;
+  while ((((W0 + (1 << b) - 1) >> b) + 1) * (((H0 + (1 << b) - 1) >> b) + 1) > kMaxTiles) ++b;
+  if (s + b > 30) return fail(set_error(SPADE_ERR_INVALID_ARG, "canvas tiles too coarse (s=%d, b=%d)", s, b));
+  const int Wc = (int)((W0 + (1 << b) - 1) >> b), Hc = (int)((H0 + (1 << b) - 1) >> b);
+  // the canvas itself is padded to whole tiles: pixels beyond the extent are ordinary pixels
+  // (no edge touches them, no crossing lies right of their corner, so they come out empty)
+  const int64_t W64 = (int64_t)Wc << b, H64 = (int64_t)Hc << b;
   if (W64 * H64 > (1ll << 31) - 4) return fail(set_error(SPADE_ERR_INVALID_ARG, "canvas too large (%lld x %lld)", (long long)W64, (long long)H64));
   g.W = (int)W64; g.H = (int)H64;
   const int64_t WH = (int64_t)g.W * g.H;
-  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (160 KB)
-  const int64_t kMaxTiles = 81920;
-  int b = 0;
-  while (((int64_t)(g.W + (1 << b) - 1) >> b) * ((int64_t)(g.H + (1 << b) - 1) >> b) > kMaxTiles) ++b;
-  int Wc = (g.W + (1 << b) - 1) >> b, Hc = (g.H + (1 << b) - 1) >> b;
 
   // --- K-B1 counts, scans, emit ---
   int64_t *nfrag, *nev, *frag_off, *ev_off;
@@ -617,15 +654,30 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   if (NG > 0) LAUNCH(k_multi_recs, NG, NG, NB, c->runs);
   LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, c->fine);
 
-  // --- K-B5 coarse tiles ---
-  if (cudaMalloc(&c->coarse, sizeof(uint16_t) * ((int64_t)Wc * Hc + 16)) != cudaSuccess)
-    return fail(set_error(SPADE_ERR_OOM, "build: coarse"));
-  TRYF(cudaMemsetAsync(c->coarse, 0, sizeof(uint16_t) * ((int64_t)Wc * Hc + 16), st), "memset");
-  TRYF(cudaMemsetAsync(nmulti, 0, 8, st), "memset");
-  LAUNCH(k_coarse, (int64_t)Wc * Hc, c->fine, g.W, g.H, b, Wc, Hc, c->coarse, nmulti);
-  unsigned long long h_mixed = 0;
-  TRYF(cudaMemcpyAsync(&h_mixed, nmulti, 8, cudaMemcpyDeviceToHost, st), "mixed");
+  // --- K-B5 coarse tiles (+ compact fine layout) ---
+  const int64_t NT = (int64_t)Wc * Hc;
+  int32_t *tval, *tmix, *mscan;
+  ALLOC(tval, NT, "tiles"); ALLOC(tmix, NT, "tiles"); ALLOC(mscan, NT, "tiles");
+  LAUNCH(k_coarse, NT, c->fine, g.W, g.H, b, Wc, Hc, tval, tmix);
+  TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, tmix, mscan, NT, st); }), "scan tiles");
+  int32_t last_scan = 0, last_mix = 0;
+  TRYF(cudaMemcpyAsync(&last_scan, mscan + NT - 1, 4, cudaMemcpyDeviceToHost, st), "mixed");
+  TRYF(cudaMemcpyAsync(&last_mix, tmix + NT - 1, 4, cudaMemcpyDeviceToHost, st), "mixed");
   TRYF(cudaStreamSynchronize(st), "sync coarse");
+  const int64_t h_mixed = (int64_t)last_scan + last_mix;
+  const bool compact = P < (int32_t)kTileMixedCompact - 1 && h_mixed <= 32768 && !(prm && (prm->flags & SPADE_CANVAS_DENSE));
+  const uint32_t owner_lim = compact ? kTileMixedCompact : kTileMixed;     // tile values v+1 below this are uniform
+  const int64_t NT1 = (int64_t)(Wc + 1) * (Hc + 1);
+  if (cudaMalloc(&c->coarse, sizeof(uint16_t) * (NT1 + 16)) != cudaSuccess)
+    return fail(set_error(SPADE_ERR_OOM, "build: coarse"));
+  TRYF(cudaMemsetAsync(c->coarse, 0, sizeof(uint16_t) * (NT1 + 16), st), "memset");
+  LAUNCH(k_coarse_final, NT1, tval, mscan, Wc, Hc, compact ? 1 : 0, owner_lim, c->coarse);
+  if (compact && h_mixed > 0) {
+    if (cudaMalloc(&c->cfine, sizeof(int32_t) * (h_mixed << (2 * b))) != cudaSuccess)
+      return fail(set_error(SPADE_ERR_OOM, "build: compact canvas"));
+    LAUNCH(k_compact, NT << (2 * b), c->fine, g.W, g.H, b, Wc, tval, mscan, NT, owner_lim, c->cfine);
+  }
+  TRYF(cudaStreamSynchronize(st), "sync compact");
 #undef TRYF
 #undef ALLOC
 #undef LAUNCH
@@ -640,6 +692,9 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   d.minx = (int32_t)g.minx; d.miny = (int32_t)g.miny;
   d.extw = (uint32_t)ew; d.exth = (uint32_t)eh;
   d.s = s; d.W = g.W; d.H = g.H; d.b = b; d.Wc = Wc; d.Hc = Hc;
+  d.compact = compact ? 1 : 0;
+  d.mix_min = compact ? kTileMixedCompact : kTileMixed;
+  d.cfine = c->cfine;
   d.fine = c->fine; d.coarse = c->coarse; d.runs = c->runs; d.run_seg = c->run_seg; d.run_poly = c->run_poly;
   d.sets = c->sets; d.set_rng = c->set_rng;
   if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));

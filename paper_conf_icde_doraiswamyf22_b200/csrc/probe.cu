@@ -30,7 +30,7 @@ namespace {
 enum Mode { kCountSmem = 0, kCountGlobal = 1, kSelect = 2, kPairs = 3 };
 
 struct alignas(32) Vec4 { int4 a, b; };   // 4 points
-struct alignas(8) QEntry { uint32_t rec, pidx; };   // boundary point: its record and index
+struct alignas(8) QEntry { uint32_t rec, pidx; };   // boundary point: record and point index
 
 __device__ __forceinline__ Vec4 ld_stream(const Vec4* p) {
   Vec4 r;
@@ -72,16 +72,6 @@ struct Params {
   Out o;
 };
 
-// classification of one point before the fine gather:
-//   0 = no polygon, 1..2^31-1 = owner + 1, bit31 set = needs the fine pixel (index in low 31 bits)
-__device__ __forceinline__ uint32_t classify_coarse(const CanvasDev& cv, const uint16_t* tiles, int x, int y) {
-  uint32_t ux = (uint32_t)x - (uint32_t)cv.minx, uy = (uint32_t)y - (uint32_t)cv.miny;
-  if (ux > cv.extw || uy > cv.exth) return 0u;
-  uint32_t fx = ux >> cv.s, fy = uy >> cv.s;
-  uint32_t t = tiles[(fy >> cv.b) * (uint32_t)cv.Wc + (fx >> cv.b)];
-  if (t != kTileMixed) return t;
-  return 0x80000000u | (fy * (uint32_t)cv.W + fx);
-}
 // Point class c after the fine gather: c = fine pixel value + 1, i.e. 0 = no polygon,
 // 1 .. 2^31-1 = owner + 1, and >= 2^31 = record ~c (boundary / multi-owner pixel).  Uniform
 // coarse tiles give the same encoding directly (tile value = owner + 1, 0 = empty).
@@ -183,49 +173,55 @@ template <int MODE>
 __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, unsigned int* hist,
                                           Out o, int x, int y, int64_t pid) {
   const CanvasDev cv = *cvg;
-  uint32_t c = classify_coarse(cv, tiles, x, y);
-  if (c & 0x80000000u) c = classify_fine(cv.fine[c & 0x7fffffffu]);
+  const uint32_t ux = (uint32_t)x - (uint32_t)cv.minx, uy = (uint32_t)y - (uint32_t)cv.miny;
+  if (ux > cv.extw || uy > cv.exth) return;
+  const uint32_t fx = ux >> cv.s, fy = uy >> cv.s;
+  uint32_t c = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
+  if (c >= cv.mix_min) c = classify_fine(*fine_ptr(cv, c, fx, fy));
   if (c == 0) return;
   if (c & 0x80000000u) rare_emit_point<MODE>(cvg, hist, o, x, y, ~c, pid);
   else rare_emit_owner<MODE>(hist, o, (int)c - 1, pid);
 }
 
-// Evaluate up to 32 queued boundary points (one per lane); the point is re-read here (L2) so the
-// streaming loop never waits on it.  Out of line: it is the rare path and keeping it out of the
-// streaming loop keeps that loop's register footprint small.
+// Evaluate up to 32 queued boundary points (one per lane).  Out of line: it is the rare path and
+// keeping it out of the streaming loop keeps that loop's register footprint small.  Queue entries
+// are 8 B (record, point index): a small queue leaves more of the SM's 256 KB for L1, which caches
+// the fine-pixel gathers of clustered points.
 template <int MODE>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const int2* __restrict__ xy, const QEntry* wq,
                                    int cnt, int lane, unsigned int* hist, Out o) {
   if (lane < cnt) {
     const QEntry e = wq[lane];
-    const int2 p = __ldg(xy + e.pidx);
+    const int2 p = __ldg(xy + e.pidx);        // re-read here (rare) so the streaming loop never waits
     rare_emit_point<MODE>(cvg, hist, o, p.x, p.y, e.rec, o.id_base + (int64_t)e.pidx);
   }
 }
 
 // Per-CTA shared-memory layout (bytes, in order):
-//   tiles   (Wc*Hc + 1) uint16, rounded up to 16 B; entry Wc*Hc is an always-empty sentinel
-//   queues  NW * QCAP QEntry (boundary points per warp; QCAP = 32 + 32 * points per thread)
+//   tiles   (Wc+1) x (Hc+1) uint16 (pitch Wc+1), rounded up to 16 B; the last column and row are
+//           always-empty sentinels: tile coordinates are clamped into them (no extent test)
+//   queues  NW * (32 + 128 U) QEntry (8 B; boundary points per warp).  Keep the total <= ~196 KB:
+//           measured, the probe loses ~35% when the L1 carve-out left over drops below ~60 KB.
 //   COUNT   kHC copies of (P + 1) uint32 bins (bin P = "no polygon" trash bin)
 //   SELECT/PAIRS: 128 int warp sums + 32 int64 warp bases
 constexpr int kHC = 8;             // histogram copies (lane & 7): spreads same-polygon atomics
 
 __host__ __device__ constexpr int qcap_for(int U) { return 32 + 32 * 4 * U; }
-__host__ __device__ __forceinline__ size_t tiles_bytes_for(int ntiles) { return (((size_t)ntiles + 1) * 2 + 15) & ~(size_t)15; }
+// tile array incl. the sentinel column and row, rounded up to 16 B
+__host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
 
-template <int MODE, int T, int U, int PF>
+template <int MODE, int T, int U, int PF, int COMPACT>
 __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
   const CanvasDev& cv = prm.cv;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int NW = T / 32;
   constexpr int NPT = 4 * U;                      // points per thread per batch
-  constexpr int QCAP = 32 + 32 * NPT;             // < 32 left over + one full batch
-  const uint32_t ntiles = (uint32_t)(cv.Wc * cv.Hc);
-  const uint32_t tbytes = (uint32_t)tiles_bytes_for((int)ntiles);
+
+  const uint32_t tbytes = (uint32_t)tiles_bytes_for(cv.Wc, cv.Hc);
   uint16_t* tiles = (uint16_t*)smem;
   QEntry* queues = (QEntry*)(smem + tbytes);
-  unsigned char* rest = smem + tbytes + NW * QCAP * sizeof(QEntry);
+  unsigned char* rest = smem + tbytes + NW * qcap_for(U) * sizeof(QEntry);
   const uint32_t P = (uint32_t)cv.num_polys;
   unsigned int* hist = (unsigned int*)rest;                       // COUNT
   unsigned int* myhist = hist + (lane & (kHC - 1)) * (P + 1);
@@ -237,7 +233,7 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
     for (uint32_t i = tid; i < kHC * (P + 1); i += T) hist[i] = 0u;
   __syncthreads();
 
-  QEntry* wq = queues + warp * QCAP;
+  QEntry* wq = queues + warp * qcap_for(U);
   __shared__ int s_qn[NW];                      // per-warp queue fill
   if (lane == 0) s_qn[warp] = 0;
   __syncwarp();
@@ -261,8 +257,10 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
   const uint32_t nvec = (uint32_t)prm.nvec;      // launches hold < 2^31 points
   const uint32_t chunk = (uint32_t)(T * U);
   const uint32_t minx = (uint32_t)cv.minx, miny = (uint32_t)cv.miny;
-  const uint32_t extw = cv.extw, exth = cv.exth;
   const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
+  const uint32_t Hc = (uint32_t)cv.Hc, Wc1 = Wc + 1u;
+  const uint32_t b = (uint32_t)cv.b, bm = (1u << cv.b) - 1u, mixmin = cv.mix_min;
+  const int32_t* __restrict__ finep = COMPACT ? cv.cfine : cv.fine;
   auto load_batch = [&](Vec4 (&v)[U], uint32_t base) {
     if (base + chunk <= nvec) {                  // CTA-uniform: full batch, no bounds checks
 #pragma unroll
@@ -288,33 +286,43 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
     } else {
       load_batch(v, base);
     }
-    // phase A: coarse (shared memory) lookup, branch-free; points outside the extent read the
-    // always-empty sentinel tile.  c = 0 (none) | owner + 1 | fine pixel index (mixed tile)
+    // phase A: coarse (shared memory) lookup, branch-free.  Offsets from the extent origin are
+    // unsigned; points left of / below the origin wrap to huge values and, like points right of /
+    // above the canvas, clamp into the always-empty sentinel column / row (exact because
+    // 2^(s+b) <= 2^30, see canvas_build.cu).  c = 0 (none) | owner + 1 | tile value (mixed).
     uint32_t c[NPT];
-    uint32_t mix = 0;
 #pragma unroll
     for (int q = 0; q < NPT; ++q) {
       const int k = q >> 2, h = q & 3;
       const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
       const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
       const uint32_t ux = (uint32_t)x - minx, uy = (uint32_t)y - miny;
-      uint32_t ti = (uy >> sb) * Wc + (ux >> sb);
-      ti = (ux <= extw && uy <= exth) ? ti : ntiles;
-      const uint32_t t = tiles[ti];
-      const bool m = t == kTileMixed;
-      c[q] = m ? (uy >> s) * W + (ux >> s) : t;
-      mix |= (m ? 1u : 0u) << q;
+      const uint32_t ti = min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc);
+      c[q] = tiles[ti];
     }
     // phase B: fine pixels of mixed tiles; all gathers of the batch in flight together
 #pragma unroll
-    for (int q = 0; q < NPT; ++q)
-      if ((mix >> q) & 1u) c[q] = classify_fine((int32_t)ld_fine(cv.fine + c[q], pol));
+    for (int q = 0; q < NPT; ++q) {
+      if (c[q] >= mixmin) {
+        const int k = q >> 2, h = q & 3;
+        const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
+        const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
+        const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
+        const uint32_t fidx = COMPACT ? ((((c[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
+        c[q] = classify_fine((int32_t)ld_fine(finep + fidx, pol));
+      }
+    }
     // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
-    uint32_t bnd = 0;
+    uint32_t orc = 0;
 #pragma unroll
-    for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
-    // phase C1: boundary points -> warp queue (smem atomic reservation), drained 32 at a time
-    if (__any_sync(0xffffffffu, bnd != 0u)) {
+    for (int q = 0; q < NPT; ++q) orc |= c[q];
+    // phase C1: boundary points -> warp queue (one smem atomic per lane that has any), drained 32
+    // at a time from the top.  Capacity 160 = < 32 left over + 32 lanes x 4 points.
+    static_assert(NPT <= 4, "queue capacity assumes <= 4 points per thread per batch");
+    if (__any_sync(0xffffffffu, (int)orc < 0)) {
+      uint32_t bnd = 0;
+#pragma unroll
+      for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
       if (bnd) {
         int pos = atomicAdd(&s_qn[warp], __popc(bnd));
 #pragma unroll
@@ -399,11 +407,10 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
   }
 }
 
-template <int MODE, int T, int U, int PF>
+template <int MODE, int T, int U, int PF, int COMPACT>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
-  const int ntiles = c->d.Wc * c->d.Hc;
-  const size_t smem = tiles_bytes_for(ntiles) + (T / 32) * qcap_for(U) * sizeof(QEntry) + extra_smem;
-  auto kern = k_probe<MODE, T, U, PF>;
+  const size_t smem = tiles_bytes_for(c->d.Wc, c->d.Hc) + (T / 32) * qcap_for(U) * sizeof(QEntry) + extra_smem;
+  auto kern = k_probe<MODE, T, U, PF, COMPACT>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
   const int sms = device_sm_count();
@@ -434,8 +441,8 @@ constexpr size_t kSmemBudget = 227 * 1024;
 // register double-buffered prefetch of the next batch).  SPADE_PROBE_VARIANT=<i> overrides the
 // default for tuning runs; the default is the measured best.
 struct Variant { int T, U, PF; };
-constexpr Variant kVariants[] = {{1024, 2, 0}, {768, 2, 1}, {512, 4, 1}, {1024, 1, 1}, {512, 2, 1}};
-constexpr int kDefaultVariant = 3;
+constexpr Variant kVariants[] = {{1024, 1, 1}, {768, 1, 1}, {512, 1, 1}};
+constexpr int kDefaultVariant = 0;
 
 int variant_index() {
   static int v = [] {
@@ -446,20 +453,23 @@ int variant_index() {
   return v;
 }
 
+template <int MODE, int COMPACT>
+int launch_variant2(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
+  switch (variant_index()) {
+    case 1: return launch<MODE, 768, 1, 1, COMPACT>(c, xy, n, p, extra, st);
+    case 2: return launch<MODE, 512, 1, 1, COMPACT>(c, xy, n, p, extra, st);
+    default: return launch<MODE, 1024, 1, 1, COMPACT>(c, xy, n, p, extra, st);
+  }
+}
+
 template <int MODE>
 int launch_variant(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
-  switch (variant_index()) {
-    case 0: return launch<MODE, 1024, 2, 0>(c, xy, n, p, extra, st);
-    case 1: return launch<MODE, 768, 2, 1>(c, xy, n, p, extra, st);
-    case 2: return launch<MODE, 512, 4, 1>(c, xy, n, p, extra, st);
-    case 3: return launch<MODE, 1024, 1, 1>(c, xy, n, p, extra, st);
-    default: return launch<MODE, 512, 2, 1>(c, xy, n, p, extra, st);
-  }
+  return c->d.compact ? launch_variant2<MODE, 1>(c, xy, n, p, extra, st) : launch_variant2<MODE, 0>(c, xy, n, p, extra, st);
 }
 
 size_t fixed_smem(const spade_canvas* c) {
   const Variant v = kVariants[variant_index()];
-  return tiles_bytes_for(c->d.Wc * c->d.Hc) + (v.T / 32) * qcap_for(v.U) * sizeof(QEntry);
+  return tiles_bytes_for(c->d.Wc, c->d.Hc) + (v.T / 32) * qcap_for(v.U) * sizeof(QEntry);
 }
 
 Params base_params(const spade_canvas* c) {

@@ -15,8 +15,11 @@ namespace spade {
 //                     v <= -2 -> record id  -2 - v  (a boundary pixel, or a multi-owner pixel)
 constexpr int32_t kEmpty = -1;
 constexpr int32_t kMultiMark = INT32_MIN;     // transient during the fill only
-// Coarse (shared-memory) tile entry, uint16: 0 = empty, 1..0xFFFE = owner+1, 0xFFFF = mixed
-constexpr uint16_t kTileEmpty = 0, kTileMixed = 0xFFFF;
+// Coarse (shared-memory) tile entry, uint16: 0 = empty, owner+1 for a uniform tile, and a mixed
+// tile is >= mix_min.  Dense layout (mix_min = 0xFFFF): the fine pixel is fine[fy*W + fx].
+// Compact layout (mix_min = 0x8000, needs P < 32767 and < 32768 mixed tiles): entry 0x8000|m and
+// the tile's pixels are the m-th block of 2^b x 2^b int32 in cfine (only mixed tiles stored).
+constexpr uint16_t kTileEmpty = 0, kTileMixed = 0xFFFF, kTileMixedCompact = 0x8000;
 
 // Boundary-index record.  For a boundary pixel: the edges touching the closed pixel,
 // [edge_begin, +edge_cnt) in run_seg/run_poly (sorted by polygon), and the corrected corner set K
@@ -32,11 +35,15 @@ struct CanvasDev {            // passed by value to kernels
   int32_t minx, miny;         // extent origin
   uint32_t extw, exth;        // maxx - minx, maxy - miny (points with larger offsets are outside)
   int32_t s;                  // log2 pixel size
-  int32_t W, H;               // fine canvas size
+  int32_t W, H;               // fine canvas size (padded to whole tiles: W = Wc << b)
   int32_t b;                  // log2 tile size in fine pixels
-  int32_t Wc, Hc;             // coarse grid
+  int32_t Wc, Hc;             // coarse grid; the smem array has pitch Wc + 1 and Hc + 1 rows
+                              // (last column and row: always-empty sentinel tiles)
   int32_t num_polys;
-  const int32_t* fine;
+  int32_t compact;            // 1: compact fine layout (cfine), 0: dense (fine)
+  uint32_t mix_min;           // tile entries >= mix_min are mixed
+  const int32_t* fine;        // dense W x H canvas (always present)
+  const int32_t* cfine;       // compact mixed-tile blocks (compact layout only)
   const uint16_t* coarse;
   const RunRec* runs;         // records: boundary pixels, then multi-owner pixels
   const int4* run_seg;        // (ax, ay, bx, by) of the edges touching each boundary pixel
@@ -55,6 +62,7 @@ struct spade_canvas {
   double mixed_tile_frac = 0.0;
   // owned device allocations
   int32_t* fine = nullptr;
+  int32_t* cfine = nullptr;
   uint16_t* coarse = nullptr;
   spade::RunRec* runs = nullptr;
   int4* run_seg = nullptr;
@@ -65,6 +73,15 @@ struct spade_canvas {
 };
 
 namespace spade {
+
+// Fine pixel index of pixel (fx, fy) whose coarse tile entry is the mixed value t.
+__host__ __device__ __forceinline__ const int32_t* fine_ptr(const CanvasDev& cv, uint32_t t, uint32_t fx, uint32_t fy) {
+  if (cv.compact) {
+    const uint32_t bm = (1u << cv.b) - 1u;
+    return cv.cfine + ((((t & 0x7fffu) << cv.b) | (fy & bm)) << cv.b | (fx & bm));
+  }
+  return cv.fine + ((size_t)fy * (uint32_t)cv.W + fx);
+}
 
 // ---- exact integer helpers (host + device) --------------------------------------------------
 __host__ __device__ __forceinline__ int64_t floor_div(int64_t a, int64_t b) {

@@ -25,9 +25,9 @@ def spade():
     return sp
 
 
-def gpu_all(sp, polys, xy, s=-1, max_dim=4096, base=0):
+def gpu_all(sp, polys, xy, s=-1, max_dim=4096, base=0, dense=False):
     import torch
-    cv = sp.Canvas(polys, log2_pixel=s, max_dim=max_dim)
+    cv = sp.Canvas(polys, log2_pixel=s, max_dim=max_dim, dense=dense)
     xy_d = torch.as_tensor(np.ascontiguousarray(xy, np.int32)).cuda()
     counts = sp.join_count(cv, xy_d).cpu().numpy()
     pt, pl = sp.join_pairs(cv, xy_d, point_id_base=base)
@@ -36,8 +36,8 @@ def gpu_all(sp, polys, xy, s=-1, max_dim=4096, base=0):
     return cv, counts, sorted_pairs(pt.cpu().numpy(), pl.cpu().numpy()), np.sort(ids.cpu().numpy())
 
 
-def check_all(sp, polys, xy, s=-1, max_dim=4096, base=0):
-    cv, counts, (pt, pl), ids = gpu_all(sp, polys, xy, s, max_dim, base)
+def check_all(sp, polys, xy, s=-1, max_dim=4096, base=0, dense=False):
+    cv, counts, (pt, pl), ids = gpu_all(sp, polys, xy, s, max_dim, base, dense)
     ocounts = oracle.join_count(xy, polys)
     opt, opl = oracle.join_pairs(xy, polys, point_id_base=base)
     oids = oracle.select(xy, polys, point_id_base=base)
@@ -48,11 +48,12 @@ def check_all(sp, polys, xy, s=-1, max_dim=4096, base=0):
     return cv
 
 
+@pytest.mark.parametrize("dense", [False, True])
 @pytest.mark.parametrize("s", [-1, 0, 1, 3, 5, 8, 10])
-def test_c1_all_ops_all_resolutions(spade, s):
+def test_c1_all_ops_all_resolutions(spade, s, dense):
     w = configs.c1()
     xy = np.concatenate([gen.points_host(w.points, w.point_seed, 0, w.n_points), configs.c1_edge_points(w.polys)])
-    check_all(spade, w.polys, xy, s=s, max_dim=w.max_dim, base=1000)
+    check_all(spade, w.polys, xy, s=s, max_dim=w.max_dim, base=1000, dense=dense)
 
 
 @pytest.mark.parametrize("seed", range(12))
@@ -61,7 +62,7 @@ def test_tiny_lattice_bruteforce(spade, seed):
     polys = random_polyset(rng, 0, 40, int(rng.integers(1, 7)))
     xy = lattice(-2, -2, 42, 42)
     for s in (0, 1, 2, 3, 4, 6):
-        check_all(spade, polys, xy, s=s)
+        check_all(spade, polys, xy, s=s, dense=bool(seed & 1))
 
 
 def test_grid_tiling_closed_form(spade):
