@@ -35,8 +35,9 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--workload", default="c3", choices=["c3", "c5"])
-    ap.add_argument("--points-per-gpu", type=int, default=1_000_000_000)
+    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5"],
+                    help="c3 (default) = the metric's join+COUNT config; c2 select, c4 pairs, c5 40k polygons")
+    ap.add_argument("--points-per-gpu", type=int, default=None, help="default: the config's size (1B; C2 100M)")
     ap.add_argument("--impl", default="spade", choices=["spade", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
@@ -44,6 +45,7 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU oracle sample time")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu/clocks)")
     ap.add_argument("--dense", action="store_true", help="force the dense fine-canvas layout (A/B runs)")
+    ap.add_argument("--max-dim", type=int, default=None, help="override the workload's canvas max_dim")
     return ap.parse_args()
 
 
@@ -54,9 +56,18 @@ def dist_env():
     return ws, rank, local
 
 
+METRICS = {
+    "count": METRIC,
+    "select": "points/sec for spatial selection (ids of points inside the query polygon)",
+    "pairs": "points/sec for point-polygon join emitting (point_id, polygon_id) pairs",
+}
+
+
 def workload(name, n_per_gpu):
     from gen import configs
-    return configs.c3(n_per_gpu) if name == "c3" else configs.c5(n_per_gpu)
+    if name in ("c1", "c2"):
+        return getattr(configs, name)() if n_per_gpu is None else getattr(configs, name)(n_per_gpu)
+    return getattr(configs, name)(n_per_gpu or 1_000_000_000)
 
 
 def measured_peak():
@@ -206,7 +217,7 @@ def main():
     # canvas build (timed separately; not part of a step)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    cv = sp.Canvas(w.polys, max_dim=w.max_dim, dense=a.dense)
+    cv = sp.Canvas(w.polys, max_dim=a.max_dim or w.max_dim, dense=a.dense)
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
     info = cv.info()
@@ -215,16 +226,27 @@ def main():
     xy = torch.empty((n, 2), dtype=torch.int32, device=dev)
     gen.points_device(w.points, w.point_seed, rank * n, n, out=xy)
     counts = torch.zeros(P, dtype=torch.int64, device=dev)
+    op = w.op
+    out_sel = torch.empty(n, dtype=torch.int64, device=dev) if op == "select" else None
+    out_pairs = (torch.empty(n, dtype=torch.int64, device=dev), torch.empty(n, dtype=torch.int32, device=dev)) \
+        if op == "pairs" else None
     torch.cuda.synchronize()
+    n_results = [0]
 
     def step(ev_k0=None, ev_k1=None):
-        counts.zero_()
+        if op == "count":
+            counts.zero_()
         if ev_k0 is not None:
             ev_k0.record(stream)
-        sp.join_count(cv, xy, counts)
+        if op == "count":
+            sp.join_count(cv, xy, counts)
+        elif op == "select":
+            n_results[0] = sp.select(cv, xy, point_id_base=rank * n, out=out_sel).numel()
+        else:
+            n_results[0] = sp.join_pairs(cv, xy, point_id_base=rank * n, out=out_pairs)[0].numel()
         if ev_k1 is not None:
             ev_k1.record(stream)
-        if ws > 1:
+        if ws > 1 and op == "count":
             dist.all_reduce(counts)
 
     for _ in range(max(3, a.warmup)):
@@ -258,17 +280,26 @@ def main():
     total_pts = n * ws
     value = total_pts * a.steps / (t_max / 1e3)
     # correctness guard: tilings cover the whole domain, every point is counted exactly once
-    ok = int(counts.sum().item()) == total_pts
+    if op == "count":
+        check = {"sum_counts_equals_points": int(counts.sum().item()) == total_pts}
+    elif op == "pairs":
+        check = {"one_pair_per_point": n_results[0] == n}
+    else:
+        check = {"selected": n_results[0], "selectivity": n_results[0] / n}
 
     kavg = statistics.mean(kern_ms)
     peak, peak_src = measured_peak()
-    achieved = n * 8 / (kavg / 1e3) / 1e9
+    # algorithmic bytes per launch: the int2 stream, plus the results written (select: 8 B id per
+    # selected point; pairs: 8 B id + 4 B polygon id per pair); counts are 8*P bytes, negligible
+    out_bytes = {"count": 0, "select": 8 * n_results[0], "pairs": 12 * n_results[0]}[op]
+    alg_bytes = n * 8 + out_bytes
+    achieved = alg_bytes / (kavg / 1e3) / 1e9
     traffic, traffic_src = ncu_traffic(w.name)
 
     line = None
     if rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": ws, "steps": a.steps,
+            "metric": METRICS[op], "value": value, "unit": "points/s", "n_gpus": ws, "steps": a.steps,
             "warmup": max(3, a.warmup), "ms_per_step": t_max / a.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {
@@ -279,17 +310,20 @@ def main():
             },
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "k_probe<COUNT> (spade_join_count)", "kernel_ms": kavg,
-                         "algorithmic_bytes_per_launch": n * 8, "peak_source": peak_src,
+                         "kernel": {"count": "k_probe<COUNT> (spade_join_count)",
+                                    "select": "k_probe<SELECT> (spade_select; includes its n_out readback)",
+                                    "pairs": "k_probe<PAIRS> (spade_join_pairs; includes its n_out readback)"}[op],
+                         "kernel_ms": kavg, "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
                          "traffic_source": traffic_src},
             "gpu_launches": int(l1 - l0),
-            "check": {"sum_counts_equals_points": ok},
+            "check": check,
         }
         if clocks:
             line["clocks"] = clocks
 
-    # end-to-end through the public API from pinned host memory (H2D + D2H inside the timing)
-    if rank == 0 and not a.no_e2e and not a.profile and ws == 1:
+    # end-to-end through the public API from pinned host memory (H2D + D2H inside the timing):
+    # every rank streams its own shard from host memory, then the counts all_reduce; max over ranks
+    if not a.no_e2e and not a.profile and op == "count":
         host = torch.empty((n, 2), dtype=torch.int32, pin_memory=True)
         host.copy_(xy)
         del xy
@@ -299,13 +333,27 @@ def main():
         times = []
         for _ in range(a.e2e_steps):
             hc[:] = 0
+            if ws > 1:
+                dist.barrier()
             torch.cuda.synchronize()
             s0 = time.perf_counter()
             sp.join_count_host(cv, host, hc)
-            times.append(time.perf_counter() - s0)
-        line["e2e"] = {"value": n / statistics.median(times), "unit": "points/s", "h2d_bytes_per_step": n * 8,
-                       "d2h_bytes_per_step": P * 8, "api": "spade_join_count_host (pinned host buffer)",
-                       "steps": a.e2e_steps, "ok": int(hc.sum()) == n}
+            if ws > 1:
+                ct = torch.from_numpy(hc).to(dev)
+                dist.all_reduce(ct)
+                hc[:] = ct.cpu().numpy()
+            dt = time.perf_counter() - s0
+            if ws > 1:
+                tt = torch.tensor([dt], dtype=torch.float64, device=dev)
+                dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+                dt = tt.item()
+            times.append(dt)
+        if rank == 0:
+            line["e2e"] = {"value": total_pts / statistics.median(times), "unit": "points/s",
+                           "h2d_bytes_per_step": n * 8, "d2h_bytes_per_step": P * 8,
+                           "api": "spade_join_count_host (pinned host buffer per rank) + all_reduce",
+                           "steps": a.e2e_steps, "ok": int(hc.sum()) == total_pts,
+                           "timing": "host wall clock around the synchronous API call, max over ranks"}
     elif rank == 0 and not a.profile:
         line["e2e"] = None
     if rank == 0 and not a.no_cpu_baseline and not a.profile and ws == 1:

@@ -183,15 +183,16 @@ def join_count(canvas: Canvas, xy, counts=None, stream=None):
     return counts
 
 
-def select(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = None, stream=None):
+def select(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = None, stream=None, out=None):
     """int64 CUDA tensor of the ids of points inside >= 1 polygon (order unspecified).
     capacity=None uses n_max = n (1-pass Map); a too-small capacity retries once with the
-    reported size (2-pass Map)."""
+    reported size (2-pass Map).  `out` (int64 CUDA, >= capacity) avoids the allocation."""
     torch = _torch()
     xy, n = _points(xy)
     cap = n if capacity is None else capacity
-    for _ in range(2):
-        out = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+    for attempt in range(2):
+        if out is None or attempt > 0 or out.numel() < max(cap, 1):
+            out = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
         n_out = ctypes.c_int64()
         rc = load().spade_select(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n, point_id_base,
                                  ctypes.c_void_p(out.data_ptr()), cap, ctypes.byref(n_out), _stream(stream))
@@ -203,14 +204,18 @@ def select(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = No
     raise SpadeError(SPADE_ERR_CAPACITY, "select: capacity retry failed")
 
 
-def join_pairs(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = None, stream=None):
-    """(point_ids int64, poly_ids int32) CUDA tensors, order unspecified."""
+def join_pairs(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = None, stream=None, out=None):
+    """(point_ids int64, poly_ids int32) CUDA tensors, order unspecified.  `out` = (pt, pl)
+    preallocated CUDA tensors (>= capacity) avoids the allocation."""
     torch = _torch()
     xy, n = _points(xy)
     cap = n if capacity is None else capacity
-    for _ in range(2):
-        pt = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
-        pl = torch.empty(max(cap, 1), dtype=torch.int32, device="cuda")
+    for attempt in range(2):
+        if out is not None and attempt == 0 and out[0].numel() >= max(cap, 1) and out[1].numel() >= max(cap, 1):
+            pt, pl = out
+        else:
+            pt = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+            pl = torch.empty(max(cap, 1), dtype=torch.int32, device="cuda")
         n_out = ctypes.c_int64()
         rc = load().spade_join_pairs(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n, point_id_base,
                                      ctypes.c_void_p(pt.data_ptr()), ctypes.c_void_p(pl.data_ptr()), cap,

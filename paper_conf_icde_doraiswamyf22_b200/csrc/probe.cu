@@ -21,6 +21,7 @@
 #include <cstdint>
 #include <algorithm>
 #include <cstdlib>
+#include <cub/block/block_scan.cuh>
 #include "spade_internal.cuh"
 
 namespace spade {
@@ -62,8 +63,15 @@ struct Out {
   int64_t id_base;            // point id of xy[0]
 };
 
+// Deferred boundary point (the exact test runs in a second, load-balanced kernel).
+struct alignas(16) DEntry { int x, y; uint32_t rec, pidx; };
+constexpr uint32_t kHole = 0xffffffffu;   // DEntry.rec of a reserved-but-unused slot
+
 struct Params {
   CanvasDev cv;
+  DEntry* defer;              // per-CTA regions of defer_cap entries (nullptr: drain in-loop)
+  uint32_t defer_cap;
+  unsigned int* defer_fill;   // [grid] entries used per CTA region
   const CanvasDev* cvg;       // the same, in global memory (for the out-of-line exact test)
   const int2* xy;
   int64_t n;
@@ -190,10 +198,44 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
 template <int MODE>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const int2* __restrict__ xy, const QEntry* wq,
                                    int cnt, int lane, unsigned int* hist, Out o) {
-  if (lane < cnt) {
-    const QEntry e = wq[lane];
-    const int2 p = __ldg(xy + e.pidx);        // re-read here (rare) so the streaming loop never waits
-    rare_emit_point<MODE>(cvg, hist, o, p.x, p.y, e.rec, o.id_base + (int64_t)e.pidx);
+  const bool active = lane < cnt;
+  QEntry e{0u, 0u};
+  int2 p = make_int2(0, 0);
+  if (active) {
+    e = wq[lane];
+    p = __ldg(xy + e.pidx);                     // re-read here (rare) so the streaming loop never waits
+  }
+  const int64_t pid = o.id_base + (int64_t)e.pidx;
+  if (MODE == kCountSmem || MODE == kCountGlobal) {
+    if (active) pip_eval(cvg, p.x, p.y, e.rec, [&](int q) { count_hit<MODE>(hist, o.counts, q); });
+    return;
+  }
+  // SELECT / PAIRS: count this lane's results, reserve all of the warp's slots with ONE global
+  // atomic (a per-result atomic on the single counter serialises badly), then write them.
+  int nres = 0;
+  if (active) {
+    if (MODE == kSelect) { bool any = false; pip_eval(cvg, p.x, p.y, e.rec, [&](int) { any = true; }); nres = any; }
+    else pip_eval(cvg, p.x, p.y, e.rec, [&](int) { ++nres; });
+  }
+  int incl = nres;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int t = __shfl_up_sync(0xffffffffu, incl, d);
+    if (lane >= d) incl += t;
+  }
+  unsigned long long gb = 0;
+  if (lane == 31 && incl > 0) gb = atomicAdd(o.total, (unsigned long long)incl);
+  gb = __shfl_sync(0xffffffffu, gb, 31);
+  int64_t pos = (int64_t)gb + (incl - nres);
+  if (nres) {
+    if (MODE == kSelect) {
+      if (pos < o.cap) o.out_ids[pos] = pid;
+    } else {
+      pip_eval(cvg, p.x, p.y, e.rec, [&](int q) {
+        if (pos < o.cap) { o.out_ids[pos] = pid; o.out_poly[pos] = q; }
+        ++pos;
+      });
+    }
   }
 }
 
@@ -235,8 +277,11 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
 
   QEntry* wq = queues + warp * qcap_for(U);
   __shared__ int s_qn[NW];                      // per-warp queue fill
+  __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
   if (lane == 0) s_qn[warp] = 0;
-  __syncwarp();
+  if (tid == 0) s_dfill = 0;
+  __syncthreads();
+  DEntry* const dreg = prm.defer ? prm.defer + (size_t)blockIdx.x * prm.defer_cap : nullptr;
   const uint64_t pol = policy_evict_last();
 
   // unaligned head and tail (< 8 points): CTA 0, warp 0
@@ -323,6 +368,25 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
       uint32_t bnd = 0;
 #pragma unroll
       for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
+      if (dreg != nullptr && bnd) {
+        // defer to the second kernel: one smem atomic per lane, a 16-B store per point
+        const uint32_t nb = __popc(bnd);
+        const uint32_t dpos = atomicAdd(&s_dfill, nb);
+        const bool fits = dpos + nb <= prm.defer_cap;
+        uint32_t d = dpos;
+#pragma unroll
+        for (int q = 0; q < NPT; ++q)
+          if ((bnd >> q) & 1u) {
+            const int k = q >> 2, h = q & 3;
+            const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
+            const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
+            if (fits) dreg[d] = DEntry{x, y, ~c[q], (uint32_t)prm.head + 4 * (base + k * T + tid) + h};
+            else if (d < prm.defer_cap) dreg[d] = DEntry{0, 0, kHole, 0u};   // region full: hole
+            ++d;
+          }
+        if (fits) bnd = 0;                                  // else: fall back to the warp queue
+      }
+      if (__any_sync(0xffffffffu, bnd != 0u)) {
       if (bnd) {
         int pos = atomicAdd(&s_qn[warp], __popc(bnd));
 #pragma unroll
@@ -343,6 +407,7 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
         if (lane == 0) s_qn[warp] = qn;
       }
       __syncwarp();
+      }
     }
     // phase C2: direct hits
     if (MODE == kCountSmem) {
@@ -354,17 +419,17 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
       for (int q = 0; q < NPT; ++q)
         if (c[q] != 0u && !(c[q] >> 31)) atomicAdd(prm.o.counts + (c[q] - 1u), 1ull);
     } else {
-      // CTA-aggregated reservation of output slots for this batch (Map with a scan)
-      int h = 0;
+      // CTA-aggregated reservation of output slots for this batch (Map with a scan).
+      // Within the warp the results are laid out slot-major (all lanes' slot 0 hits, then slot 1,
+      // ...), so every store instruction writes one contiguous run: coalesced 8-B / 4-B stores.
+      unsigned hm[NPT];
+      int wtot = 0;
 #pragma unroll
-      for (int q = 0; q < NPT; ++q) h += (c[q] != 0u && !(c[q] >> 31)) ? 1 : 0;
-      int incl = h;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int t = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += t;
+      for (int q = 0; q < NPT; ++q) {
+        hm[q] = __ballot_sync(0xffffffffu, c[q] != 0u && !(c[q] >> 31));
+        wtot += __popc(hm[q]);
       }
-      if (lane == 31) s_scan[warp] = incl;
+      if (lane == 0) s_scan[warp] = wtot;
       __syncthreads();
       if (warp == 0) {
         int wsum = lane < NW ? s_scan[lane] : 0, wincl = wsum;
@@ -379,23 +444,29 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
         if (lane < NW) s_base[lane] = (long long)gb + (wincl - wsum);
       }
       __syncthreads();
-      int64_t pos = s_base[warp] + (incl - h);
+      int64_t wpos = s_base[warp];
+      const unsigned lt = (1u << lane) - 1u;
 #pragma unroll
       for (int q = 0; q < NPT; ++q) {
-        if (c[q] != 0u && !(c[q] >> 31)) {
+        if ((hm[q] >> lane) & 1u) {
+          const int64_t pos = wpos + __popc(hm[q] & lt);
           if (pos < prm.o.cap) {
             const int k = q >> 2, hh = q & 3;
             prm.o.out_ids[pos] = prm.o.id_base + prm.head + 4 * (int64_t)(base + k * T + tid) + hh;
             if (MODE == kPairs) prm.o.out_poly[pos] = (int)c[q] - 1;
           }
-          ++pos;
         }
+        wpos += __popc(hm[q]);
       }
       __syncthreads();   // s_scan / s_base reuse next batch
     }
   }
   __syncwarp();
   if (s_qn[warp] > 0) drain<MODE>(prm.cvg, prm.xy, wq, s_qn[warp], lane, myhist, prm.o);
+  if (dreg != nullptr) {
+    __syncthreads();
+    if (tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
+  }
   if (MODE == kCountSmem) {
     __syncthreads();
     for (uint32_t i = tid; i < P; i += T) {
@@ -405,6 +476,97 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
       if (sum) atomicAdd(prm.o.counts + i, sum);
     }
   }
+}
+
+// Second kernel: the deferred boundary points of every CTA region, one per thread, exact test
+// over the pixel's edges (pip_eval).  COUNT: shared-memory histogram (or global atomics);
+// SELECT/PAIRS: per-block count pass, block scan, one global atomic, write pass.
+template <int MODE>
+__global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
+                                                  uint32_t cap, const unsigned int* __restrict__ fill, int nreg, Out o,
+                                                  int smem_hist) {
+  using BS = cub::BlockScan<int, 256>;
+  __shared__ typename BS::TempStorage tmp;
+  __shared__ unsigned long long s_gb;
+  __shared__ long long s_pre[1025];              // exclusive prefix of the region fills
+  extern __shared__ unsigned int dh[];
+  const int P = cvg->num_polys;
+  const bool sh = MODE == kCountSmem && smem_hist;
+  if (sh)
+    for (int i = threadIdx.x; i < P; i += 256) dh[i] = 0u;
+  if (threadIdx.x == 0) {                        // nreg <= 1024 regions (one per probe CTA)
+    long long a = 0;
+    for (int r = 0; r < nreg; ++r) { s_pre[r] = a; a += fill[r]; }
+    s_pre[nreg] = a;
+  }
+  __syncthreads();
+  const long long total = s_pre[nreg];
+  // flattened index space [0, total) in block-sized chunks, grid-stride (all threads loop together)
+  for (long long b0 = (long long)blockIdx.x * 256; b0 < total; b0 += (long long)gridDim.x * 256) {
+    const long long v = b0 + threadIdx.x;
+    DEntry e{0, 0, kHole, 0u};
+    if (v < total) {
+      int lo = 0, hi = nreg;                     // region r: s_pre[r] <= v < s_pre[r + 1]
+      while (hi - lo > 1) { const int mid = (lo + hi) >> 1; if (s_pre[mid] <= v) lo = mid; else hi = mid; }
+      e = defer[(size_t)lo * cap + (size_t)(v - s_pre[lo])];
+    }
+    const bool act = e.rec != kHole;
+    const int64_t pid = o.id_base + (int64_t)e.pidx;
+    if (MODE == kCountSmem || MODE == kCountGlobal) {
+      if (act) pip_eval(cvg, e.x, e.y, e.rec, [&](int q) {
+        if (sh) atomicAdd(&dh[q], 1u); else atomicAdd(o.counts + q, 1ull);
+      });
+    } else {
+      int nres = 0;
+      if (act) {
+        if (MODE == kSelect) { bool any = false; pip_eval(cvg, e.x, e.y, e.rec, [&](int) { any = true; }); nres = any; }
+        else pip_eval(cvg, e.x, e.y, e.rec, [&](int) { ++nres; });
+      }
+      int excl, tot;
+      BS(tmp).ExclusiveSum(nres, excl, tot);
+      if (threadIdx.x == 0) s_gb = tot ? atomicAdd(o.total, (unsigned long long)tot) : 0ull;
+      __syncthreads();
+      int64_t pos = (int64_t)s_gb + excl;
+      if (nres) {
+        if (MODE == kSelect) {
+          if (pos < o.cap) o.out_ids[pos] = pid;
+        } else {
+          pip_eval(cvg, e.x, e.y, e.rec, [&](int q) {
+            if (pos < o.cap) { o.out_ids[pos] = pid; o.out_poly[pos] = q; }
+            ++pos;
+          });
+        }
+      }
+      __syncthreads();
+    }
+  }
+  if (sh) {
+    __syncthreads();
+    for (int q = threadIdx.x; q < P; q += 256)
+      if (dh[q]) atomicAdd(o.counts + q, (unsigned long long)dh[q]);
+  }
+}
+
+// Stream-ordered scratch comes from the device's default memory pool; by default the pool hands
+// memory back to the driver at every synchronisation, which made each call re-map its scratch.
+void keep_pool_memory() {
+  static bool done = false;
+  if (done) return;
+  done = true;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = 16ull << 30;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  cudaGetLastError();
+}
+
+bool defer_enabled(int MODE) {
+  static const int env = [] { const char* e = getenv("SPADE_DEFER"); return e ? atoi(e) : -1; }();
+  if (env >= 0) return env != 0;
+  return MODE == kSelect || MODE == kPairs || true;
 }
 
 template <int MODE, int T, int U, int PF, int COMPACT>
@@ -427,10 +589,38 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.o.id_base = base.o.id_base + off;
     const int64_t chunks = (p.nvec + (int64_t)T * U - 1) / ((int64_t)T * U);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(sms, chunks));
+    // deferred boundary regions: n/grid/8 entries per CTA (overflow falls back to in-loop drains)
+    DEntry* dbuf = nullptr;
+    unsigned int* dfill = nullptr;
+    if (defer_enabled(MODE)) {
+      keep_pool_memory();
+      const int64_t per = std::min<int64_t>(std::max<int64_t>(m / grid / 16, 1024), 1 << 22);
+      p.defer_cap = (uint32_t)per;
+      if (cudaMallocAsync((void**)&dbuf, sizeof(DEntry) * per * grid, st) != cudaSuccess ||
+          cudaMallocAsync((void**)&dfill, sizeof(unsigned int) * grid, st) != cudaSuccess) {
+        cudaGetLastError();                       // no scratch: drain in-loop instead
+        if (dbuf) cudaFreeAsync(dbuf, st);
+        dbuf = nullptr; dfill = nullptr;
+      }
+      p.defer = dbuf;
+      p.defer_fill = dfill;
+    }
     kern<<<grid, T, smem, st>>>(p);
     count_launch();
     e = cudaGetLastError();
     if (e != cudaSuccess) return check_cuda(e, "probe launch");
+    if (dbuf) {
+      const int P = c->d.num_polys;
+      const int sh = (MODE == kCountSmem && (size_t)P * 4 <= 96 * 1024) ? 1 : 0;
+      const size_t dsm = sh ? (size_t)P * 4 : 0;
+      if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
+      k_deferred<MODE><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh);
+      count_launch();
+      e = cudaGetLastError();
+      cudaFreeAsync(dbuf, st);
+      cudaFreeAsync(dfill, st);
+      if (e != cudaSuccess) return check_cuda(e, "deferred boundary launch");
+    }
   }
   return SPADE_OK;
 }
