@@ -500,10 +500,13 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   Geo g;
   g.minx = h_ext[0]; g.miny = h_ext[1]; g.s = s; g.S = 1ll << s;
   const int64_t W0 = (ew >> s) + 1, H0 = (eh >> s) + 1;
-  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (160 KB),
+  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (<= 160 KB),
   // including one sentinel column and row of always-empty tiles (the probe clamps tile
-  // coordinates into them instead of testing the extent); tile side 2^b pixels, s + b <= 30
-  const int64_t kMaxTiles = 81920;
+  // coordinates into them instead of testing the extent); tile side 2^b pixels, s + b <= 30.
+  // The probe's COUNT histogram ((P+1) uint32) shares the ~196 KB budget with the tiles.
+  const int64_t hist1 = ((int64_t)P + 1) * 4, kSoft = 196 * 1024;
+  const int64_t kMaxTiles = hist1 <= kSoft - 8192 ? std::min<int64_t>(81920, std::max<int64_t>(4096, (kSoft - hist1) / 2))
+                                                  : 81920;
   int b = 0;
   while ((((W0 + (1 << b) - 1) >> b) + 1) * (((H0 + (1 << b) - 1) >> b) + 1) > kMaxTiles) ++b;
   if (s + b > 30) return fail(set_error(SPADE_ERR_INVALID_ARG, "canvas tiles too coarse (s=%d, b=%d)", s, b));

@@ -8,16 +8,17 @@
 // Map output via a unique slot per result + scan.
 //
 // B200 design:
-//   * one persistent CTA per SM, T threads; the coarse canvas (<= 80K uint16 tiles) is copied
-//     into shared memory once per CTA, so most points are classified by ONE LDS;
-//   * points stream with 256-bit loads (LDG.E.256, L1::no_allocate, L2::evict_first);
-//   * points in mixed tiles gather one int32 fine pixel from L2 (evict_last policy); all gathers of
-//     a thread's batch are issued before any is consumed (memory-level parallelism);
-//   * boundary points are compacted per warp (ballot) into a shared-memory queue and evaluated
-//     32 at a time (one per lane) against the few edges touching their pixel (exact int64 tests);
-//   * COUNT: shared-memory per-polygon histogram (smem atomics), flushed once per CTA with
-//     64-bit global atomics; SELECT/PAIRS: CTA-aggregated output reservation (one global atomic
-//     per CTA batch) and direct stores.
+//   * one persistent 1024-thread CTA per SM; the coarse canvas (<= 80K uint16 tiles + a sentinel
+//     column/row) is copied into shared memory once per CTA, so most points are classified by
+//     ONE shared-memory load;
+//   * points stream with 256-bit loads (LDG.E.256, L1::no_allocate, L2::evict_first), 4 points per
+//     thread per batch, and the next batch's loads are issued before the current batch is processed;
+//   * points in mixed tiles gather one int32 fine pixel (compact mixed-tile layout, L2 evict_last);
+//   * boundary points (a few %) are appended to a per-CTA region in global memory and tested by a
+//     second, load-balanced kernel (k_deferred) against the few edges touching their pixel;
+//   * COUNT: shared-memory per-polygon histogram (copies selected by lane), flushed once per CTA
+//     with 64-bit global atomics; SELECT/PAIRS: CTA-aggregated output reservation (one global
+//     atomic per 4096-point batch), slot-major coalesced stores.
 #include <cstdint>
 #include <algorithm>
 #include <cstdlib>
@@ -30,8 +31,22 @@ namespace {
 
 enum Mode { kCountSmem = 0, kCountGlobal = 1, kSelect = 2, kPairs = 3 };
 
+constexpr int kT = 1024;           // threads per CTA (one CTA per SM)
+constexpr int kNW = kT / 32;
+constexpr int kNPT = 4;            // points per thread per batch (one 256-bit vector)
+// Shared memory above ~196 KB per CTA shrinks the L1 carve-out below ~60 KB and costs ~35%
+// (measured on B200); the histogram copies are chosen to stay under it.
+constexpr size_t kSmemSoft = 196 * 1024;
+
 struct alignas(32) Vec4 { int4 a, b; };   // 4 points
-struct alignas(8) QEntry { uint32_t rec, pidx; };   // boundary point: record and point index
+
+// Deferred boundary point (the exact test runs in the second kernel).
+struct alignas(16) DEntry { int x, y; uint32_t rec, pidx; };
+constexpr uint32_t kHole = 0xffffffffu;   // DEntry.rec of a reserved-but-unused slot
+
+// Boundary point in a warp's shared-memory queue (COUNT with an in-loop exact test).
+struct alignas(8) QEntry { uint32_t rec, pidx; };
+constexpr int kQCap = 32 + 32 * kNPT;     // < 32 left over + one batch of the warp's points
 
 __device__ __forceinline__ Vec4 ld_stream(const Vec4* p) {
   Vec4 r;
@@ -63,16 +78,13 @@ struct Out {
   int64_t id_base;            // point id of xy[0]
 };
 
-// Deferred boundary point (the exact test runs in a second, load-balanced kernel).
-struct alignas(16) DEntry { int x, y; uint32_t rec, pidx; };
-constexpr uint32_t kHole = 0xffffffffu;   // DEntry.rec of a reserved-but-unused slot
-
 struct Params {
   CanvasDev cv;
-  DEntry* defer;              // per-CTA regions of defer_cap entries (nullptr: drain in-loop)
+  const CanvasDev* cvg;       // the same, in global memory (for the out-of-line exact test)
+  DEntry* defer;              // per-CTA regions of defer_cap entries
   uint32_t defer_cap;
   unsigned int* defer_fill;   // [grid] entries used per CTA region
-  const CanvasDev* cvg;       // the same, in global memory (for the out-of-line exact test)
+  uint32_t hcopies;           // COUNT histogram copies in shared memory (power of 2)
   const int2* xy;
   int64_t n;
   int64_t head;               // points before the first 32-byte aligned one (0..3)
@@ -80,7 +92,7 @@ struct Params {
   Out o;
 };
 
-// Point class c after the fine gather: c = fine pixel value + 1, i.e. 0 = no polygon,
+// Point class after the fine gather: c = fine pixel value + 1, i.e. 0 = no polygon,
 // 1 .. 2^31-1 = owner + 1, and >= 2^31 = record ~c (boundary / multi-owner pixel).  Uniform
 // coarse tiles give the same encoding directly (tile value = owner + 1, 0 = empty).
 __device__ __forceinline__ uint32_t classify_fine(int32_t v) { return (uint32_t)v + 1u; }
@@ -126,12 +138,17 @@ __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int p
   int cur = -1, par = 0;
   const int64_t e1 = r.edge_begin + r.edge_cnt;
   for (int64_t e = r.edge_begin; e < e1; ++e) {
+    const int4 g = __ldg(seg + e);
+    // an edge that straddles neither the horizontal line y = py nor the vertical line x = X
+    // contributes nothing (cr and cu are both 0): skip it without the cross product or its id
+    if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
+    if (!local_bit(g, X, px, py)) continue;
     const int p = __ldg(poly + e);
     if (p != cur) {
       if (cur >= 0) finalize(cur, par);
       cur = p; par = 0;
     }
-    par ^= local_bit(__ldg(seg + e), X, px, py);
+    par ^= 1;
   }
   if (cur >= 0) finalize(cur, par);
   while (ti < tn) emit(term_at(ti++));
@@ -143,10 +160,11 @@ __device__ __forceinline__ void count_hit(unsigned int* hist, unsigned long long
   else atomicAdd(counts + owner, 1ull);
 }
 
-// Emission from the rare paths (boundary queue drains, unaligned head/tail): per-lane atomics.
+// Emission from the rare in-kernel paths (deferral region full, unaligned head/tail): per-lane
+// atomics.
 template <int MODE>
-__device__ __forceinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, const Out& o,
-                                                int x, int y, uint32_t rec, int64_t pid) {
+__device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, Out o,
+                                             int x, int y, uint32_t rec, int64_t pid) {
   if (MODE == kCountSmem || MODE == kCountGlobal) {
     pip_eval(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, o.counts, p); });
   } else if (MODE == kSelect) {
@@ -191,97 +209,53 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
   else rare_emit_owner<MODE>(hist, o, (int)c - 1, pid);
 }
 
-// Evaluate up to 32 queued boundary points (one per lane).  Out of line: it is the rare path and
-// keeping it out of the streaming loop keeps that loop's register footprint small.  Queue entries
-// are 8 B (record, point index): a small queue leaves more of the SM's 256 KB for L1, which caches
-// the fine-pixel gathers of clustered points.
+// COUNT, in-loop variant: evaluate up to 32 queued boundary points (one per lane).  Out of line:
+// the streaming loop keeps a small register footprint.  The point is re-read here (L2).
 template <int MODE>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const int2* __restrict__ xy, const QEntry* wq,
-                                   int cnt, int lane, unsigned int* hist, Out o) {
-  const bool active = lane < cnt;
-  QEntry e{0u, 0u};
-  int2 p = make_int2(0, 0);
-  if (active) {
-    e = wq[lane];
-    p = __ldg(xy + e.pidx);                     // re-read here (rare) so the streaming loop never waits
-  }
-  const int64_t pid = o.id_base + (int64_t)e.pidx;
-  if (MODE == kCountSmem || MODE == kCountGlobal) {
-    if (active) pip_eval(cvg, p.x, p.y, e.rec, [&](int q) { count_hit<MODE>(hist, o.counts, q); });
-    return;
-  }
-  // SELECT / PAIRS: count this lane's results, reserve all of the warp's slots with ONE global
-  // atomic (a per-result atomic on the single counter serialises badly), then write them.
-  int nres = 0;
-  if (active) {
-    if (MODE == kSelect) { bool any = false; pip_eval(cvg, p.x, p.y, e.rec, [&](int) { any = true; }); nres = any; }
-    else pip_eval(cvg, p.x, p.y, e.rec, [&](int) { ++nres; });
-  }
-  int incl = nres;
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const int t = __shfl_up_sync(0xffffffffu, incl, d);
-    if (lane >= d) incl += t;
-  }
-  unsigned long long gb = 0;
-  if (lane == 31 && incl > 0) gb = atomicAdd(o.total, (unsigned long long)incl);
-  gb = __shfl_sync(0xffffffffu, gb, 31);
-  int64_t pos = (int64_t)gb + (incl - nres);
-  if (nres) {
-    if (MODE == kSelect) {
-      if (pos < o.cap) o.out_ids[pos] = pid;
-    } else {
-      pip_eval(cvg, p.x, p.y, e.rec, [&](int q) {
-        if (pos < o.cap) { o.out_ids[pos] = pid; o.out_poly[pos] = q; }
-        ++pos;
-      });
-    }
+                                   int cnt, int lane, unsigned int* hist, unsigned long long* counts) {
+  if (lane < cnt) {
+    const QEntry e = wq[lane];
+    const int2 p = __ldg(xy + e.pidx);
+    pip_eval(cvg, p.x, p.y, e.rec, [&](int q) { count_hit<MODE>(hist, counts, q); });
   }
 }
 
 // Per-CTA shared-memory layout (bytes, in order):
 //   tiles   (Wc+1) x (Hc+1) uint16 (pitch Wc+1), rounded up to 16 B; the last column and row are
 //           always-empty sentinels: tile coordinates are clamped into them (no extent test)
-//   queues  NW * (32 + 128 U) QEntry (8 B; boundary points per warp).  Keep the total <= ~196 KB:
-//           measured, the probe loses ~35% when the L1 carve-out left over drops below ~60 KB.
-//   COUNT   kHC copies of (P + 1) uint32 bins (bin P = "no polygon" trash bin)
+//   COUNT   hcopies x (P + 1) uint32 bins (bin P = "no polygon" trash bin), copy = lane & (hc-1)
+//   QUEUE   (COUNT, in-loop exact test) kNW x kQCap QEntry: boundary points per warp
 //   SELECT/PAIRS: 128 int warp sums + 32 int64 warp bases
-constexpr int kHC = 8;             // histogram copies (lane & 7): spreads same-polygon atomics
-
-__host__ __device__ constexpr int qcap_for(int U) { return 32 + 32 * 4 * U; }
-// tile array incl. the sentinel column and row, rounded up to 16 B
 __host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
+constexpr size_t kScanBytes = 128 * sizeof(int) + 32 * sizeof(long long);
 
-template <int MODE, int T, int U, int PF, int COMPACT>
-__global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params prm) {
+template <int MODE, int COMPACT, int QUEUE>
+__global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
   const CanvasDev& cv = prm.cv;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  constexpr int NW = T / 32;
-  constexpr int NPT = 4 * U;                      // points per thread per batch
+  constexpr int T = kT, NW = kNW, NPT = kNPT;
 
   const uint32_t tbytes = (uint32_t)tiles_bytes_for(cv.Wc, cv.Hc);
   uint16_t* tiles = (uint16_t*)smem;
-  QEntry* queues = (QEntry*)(smem + tbytes);
-  unsigned char* rest = smem + tbytes + NW * qcap_for(U) * sizeof(QEntry);
+  unsigned char* rest = smem + tbytes;
   const uint32_t P = (uint32_t)cv.num_polys;
   unsigned int* hist = (unsigned int*)rest;                       // COUNT
-  unsigned int* myhist = hist + (lane & (kHC - 1)) * (P + 1);
+  unsigned int* myhist = hist + (lane & (prm.hcopies - 1)) * (P + 1);
   int* s_scan = (int*)rest;                                       // SELECT/PAIRS
   long long* s_base = (long long*)(rest + 128 * sizeof(int));
+  __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
+  __shared__ int s_qn[kNW];                     // QUEUE: per-warp queue fill
+  QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : 0)) + warp * kQCap;
+  if (QUEUE && lane == 0) s_qn[warp] = 0;
 
   for (uint32_t i = tid; i < tbytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
   if (MODE == kCountSmem)
-    for (uint32_t i = tid; i < kHC * (P + 1); i += T) hist[i] = 0u;
-  __syncthreads();
-
-  QEntry* wq = queues + warp * qcap_for(U);
-  __shared__ int s_qn[NW];                      // per-warp queue fill
-  __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
-  if (lane == 0) s_qn[warp] = 0;
+    for (uint32_t i = tid; i < prm.hcopies * (P + 1); i += T) hist[i] = 0u;
   if (tid == 0) s_dfill = 0;
   __syncthreads();
-  DEntry* const dreg = prm.defer ? prm.defer + (size_t)blockIdx.x * prm.defer_cap : nullptr;
+  DEntry* const dreg = QUEUE ? nullptr : prm.defer + (size_t)blockIdx.x * prm.defer_cap;
   const uint64_t pol = policy_evict_last();
 
   // unaligned head and tail (< 8 points): CTA 0, warp 0
@@ -300,113 +274,98 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
 
   const Vec4* vp = (const Vec4*)(prm.xy + prm.head);
   const uint32_t nvec = (uint32_t)prm.nvec;      // launches hold < 2^31 points
-  const uint32_t chunk = (uint32_t)(T * U);
+  const uint32_t chunk = (uint32_t)T;
   const uint32_t minx = (uint32_t)cv.minx, miny = (uint32_t)cv.miny;
   const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
   const uint32_t Hc = (uint32_t)cv.Hc, Wc1 = Wc + 1u;
   const uint32_t b = (uint32_t)cv.b, bm = (1u << cv.b) - 1u, mixmin = cv.mix_min;
   const int32_t* __restrict__ finep = COMPACT ? cv.cfine : cv.fine;
-  auto load_batch = [&](Vec4 (&v)[U], uint32_t base) {
-    if (base + chunk <= nvec) {                  // CTA-uniform: full batch, no bounds checks
-#pragma unroll
-      for (int k = 0; k < U; ++k) v[k] = ld_stream(vp + base + k * T + tid);
-    } else {
-#pragma unroll
-      for (int k = 0; k < U; ++k) {
-        const uint32_t idx = base + k * T + tid;
-        if (idx < nvec) v[k] = ld_stream(vp + idx);
-        else { v[k].a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v[k].b = v[k].a; }
-      }
-    }
+  auto load_batch = [&](Vec4& v, uint32_t base) {
+    const uint32_t idx = base + tid;
+    if (base + chunk <= nvec) v = ld_stream(vp + idx);       // CTA-uniform: full batch
+    else if (idx < nvec) v = ld_stream(vp + idx);
+    else { v.a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v.b = v.a; }
   };
   const uint32_t stride = gridDim.x * chunk;
-  Vec4 nxt[U];
-  if (PF && blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
+  Vec4 nxt;
+  if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
   for (uint32_t base = blockIdx.x * chunk; base < nvec; base += stride) {
-    Vec4 v[U];
-    if (PF) {
-#pragma unroll
-      for (int k = 0; k < U; ++k) v[k] = nxt[k];
-      if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight while this one is processed
-    } else {
-      load_batch(v, base);
-    }
+    const Vec4 v = nxt;
+    if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight meanwhile
     // phase A: coarse (shared memory) lookup, branch-free.  Offsets from the extent origin are
     // unsigned; points left of / below the origin wrap to huge values and, like points right of /
     // above the canvas, clamp into the always-empty sentinel column / row (exact because
-    // 2^(s+b) <= 2^30, see canvas_build.cu).  c = 0 (none) | owner + 1 | tile value (mixed).
+    // 2^(s+b) <= 2^30, see canvas_build.cu).  Padding points (INT32_MIN) land there too.
     uint32_t c[NPT];
 #pragma unroll
     for (int q = 0; q < NPT; ++q) {
-      const int k = q >> 2, h = q & 3;
-      const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
-      const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
+      const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+      const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
       const uint32_t ux = (uint32_t)x - minx, uy = (uint32_t)y - miny;
-      const uint32_t ti = min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc);
-      c[q] = tiles[ti];
+      c[q] = tiles[min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc)];
     }
     // phase B: fine pixels of mixed tiles; all gathers of the batch in flight together
 #pragma unroll
     for (int q = 0; q < NPT; ++q) {
       if (c[q] >= mixmin) {
-        const int k = q >> 2, h = q & 3;
-        const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
-        const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
+        const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+        const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
         const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
         const uint32_t fidx = COMPACT ? ((((c[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
         c[q] = classify_fine((int32_t)ld_fine(finep + fidx, pol));
       }
     }
     // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
-    uint32_t orc = 0;
+    const uint32_t orc = c[0] | c[1] | c[2] | c[3];
+    if (QUEUE) {
+      // phase C1 (COUNT): boundary points -> warp queue (one smem atomic per lane that has any),
+      // drained 32 at a time from the top, in the loop: the ALU-heavy exact tests overlap the
+      // memory-bound stream of the other warps
+      if (__any_sync(0xffffffffu, (int)orc < 0)) {
+        uint32_t bnd = 0;
 #pragma unroll
-    for (int q = 0; q < NPT; ++q) orc |= c[q];
-    // phase C1: boundary points -> warp queue (one smem atomic per lane that has any), drained 32
-    // at a time from the top.  Capacity 160 = < 32 left over + 32 lanes x 4 points.
-    static_assert(NPT <= 4, "queue capacity assumes <= 4 points per thread per batch");
-    if (__any_sync(0xffffffffu, (int)orc < 0)) {
+        for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
+        if (bnd) {
+          int pos = atomicAdd(&s_qn[warp], __popc(bnd));
+#pragma unroll
+          for (int q = 0; q < NPT; ++q)
+            if ((bnd >> q) & 1u) wq[pos++] = QEntry{~c[q], (uint32_t)prm.head + 4 * (base + tid) + q};
+        }
+        __syncwarp();
+        int qn = s_qn[warp];
+        if (qn >= 32) {
+          do {
+            drain<MODE>(prm.cvg, prm.xy, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+            qn -= 32;
+          } while (qn >= 32);
+          __syncwarp();
+          if (lane == 0) s_qn[warp] = qn;
+        }
+        __syncwarp();
+      }
+    } else if ((int)orc < 0) {
+      // phase C1: boundary points -> this CTA's deferral region (one smem atomic per lane that has
+      // any, a 16-B store per point); if the region is full, test them right here (rare)
       uint32_t bnd = 0;
 #pragma unroll
       for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
-      if (dreg != nullptr && bnd) {
-        // defer to the second kernel: one smem atomic per lane, a 16-B store per point
-        const uint32_t nb = __popc(bnd);
-        const uint32_t dpos = atomicAdd(&s_dfill, nb);
-        const bool fits = dpos + nb <= prm.defer_cap;
-        uint32_t d = dpos;
+      const uint32_t nb = __popc(bnd);
+      uint32_t d = atomicAdd(&s_dfill, nb);
+      const bool fits = d + nb <= prm.defer_cap;
 #pragma unroll
-        for (int q = 0; q < NPT; ++q)
-          if ((bnd >> q) & 1u) {
-            const int k = q >> 2, h = q & 3;
-            const int x = h == 0 ? v[k].a.x : h == 1 ? v[k].a.z : h == 2 ? v[k].b.x : v[k].b.z;
-            const int y = h == 0 ? v[k].a.y : h == 1 ? v[k].a.w : h == 2 ? v[k].b.y : v[k].b.w;
-            if (fits) dreg[d] = DEntry{x, y, ~c[q], (uint32_t)prm.head + 4 * (base + k * T + tid) + h};
-            else if (d < prm.defer_cap) dreg[d] = DEntry{0, 0, kHole, 0u};   // region full: hole
-            ++d;
+      for (int q = 0; q < NPT; ++q) {
+        if ((bnd >> q) & 1u) {
+          const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+          const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+          const uint32_t pidx = (uint32_t)prm.head + 4 * (base + tid) + q;
+          if (fits) {
+            dreg[d] = DEntry{x, y, ~c[q], pidx};
+          } else {
+            if (d < prm.defer_cap) dreg[d] = DEntry{0, 0, kHole, 0u};
+            rare_emit_point<MODE>(prm.cvg, myhist, prm.o, x, y, ~c[q], prm.o.id_base + pidx);
           }
-        if (fits) bnd = 0;                                  // else: fall back to the warp queue
-      }
-      if (__any_sync(0xffffffffu, bnd != 0u)) {
-      if (bnd) {
-        int pos = atomicAdd(&s_qn[warp], __popc(bnd));
-#pragma unroll
-        for (int q = 0; q < NPT; ++q)
-          if ((bnd >> q) & 1u) {
-            const int k = q >> 2, h = q & 3;
-            wq[pos++] = QEntry{~c[q], (uint32_t)prm.head + 4 * (base + k * T + tid) + h};
-          }
-      }
-      __syncwarp();
-      int qn = s_qn[warp];
-      if (qn >= 32) {
-        do {
-          drain<MODE>(prm.cvg, prm.xy, wq + qn - 32, 32, lane, myhist, prm.o);
-          qn -= 32;
-        } while (qn >= 32);
-        __syncwarp();
-        if (lane == 0) s_qn[warp] = qn;
-      }
-      __syncwarp();
+          ++d;
+        }
       }
     }
     // phase C2: direct hits
@@ -451,8 +410,7 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
         if ((hm[q] >> lane) & 1u) {
           const int64_t pos = wpos + __popc(hm[q] & lt);
           if (pos < prm.o.cap) {
-            const int k = q >> 2, hh = q & 3;
-            prm.o.out_ids[pos] = prm.o.id_base + prm.head + 4 * (int64_t)(base + k * T + tid) + hh;
+            prm.o.out_ids[pos] = prm.o.id_base + prm.head + 4 * (int64_t)(base + tid) + q;
             if (MODE == kPairs) prm.o.out_poly[pos] = (int)c[q] - 1;
           }
         }
@@ -461,26 +419,25 @@ __global__ void __launch_bounds__(T, 1) k_probe(const __grid_constant__ Params p
       __syncthreads();   // s_scan / s_base reuse next batch
     }
   }
-  __syncwarp();
-  if (s_qn[warp] > 0) drain<MODE>(prm.cvg, prm.xy, wq, s_qn[warp], lane, myhist, prm.o);
-  if (dreg != nullptr) {
-    __syncthreads();
-    if (tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
+  if (QUEUE) {
+    __syncwarp();
+    if (s_qn[warp] > 0) drain<MODE>(prm.cvg, prm.xy, wq, s_qn[warp], lane, myhist, prm.o.counts);
   }
+  __syncthreads();
+  if (!QUEUE && tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
   if (MODE == kCountSmem) {
-    __syncthreads();
     for (uint32_t i = tid; i < P; i += T) {
       unsigned long long sum = 0;
-#pragma unroll
-      for (int k = 0; k < kHC; ++k) sum += hist[k * (P + 1) + i];
+      for (uint32_t k = 0; k < prm.hcopies; ++k) sum += hist[k * (P + 1) + i];
       if (sum) atomicAdd(prm.o.counts + i, sum);
     }
   }
 }
 
-// Second kernel: the deferred boundary points of every CTA region, one per thread, exact test
-// over the pixel's edges (pip_eval).  COUNT: shared-memory histogram (or global atomics);
-// SELECT/PAIRS: per-block count pass, block scan, one global atomic, write pass.
+// Second kernel: the deferred boundary points of every CTA region, flattened and spread over
+// many blocks (one point per thread), exact test over the pixel's edges (pip_eval).  COUNT:
+// shared-memory histogram (or global atomics); SELECT/PAIRS: per-block count pass, block scan,
+// one global atomic, write pass.
 template <int MODE>
 __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                   uint32_t cap, const unsigned int* __restrict__ fill, int nreg, Out o,
@@ -491,7 +448,7 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
   __shared__ long long s_pre[1025];              // exclusive prefix of the region fills
   extern __shared__ unsigned int dh[];
   const int P = cvg->num_polys;
-  const bool sh = MODE == kCountSmem && smem_hist;
+  const bool sh = (MODE == kCountSmem || MODE == kCountGlobal) && smem_hist;
   if (sh)
     for (int i = threadIdx.x; i < P; i += 256) dh[i] = 0u;
   if (threadIdx.x == 0) {                        // nreg <= 1024 regions (one per probe CTA)
@@ -501,7 +458,6 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
   }
   __syncthreads();
   const long long total = s_pre[nreg];
-  // flattened index space [0, total) in block-sized chunks, grid-stride (all threads loop together)
   for (long long b0 = (long long)blockIdx.x * 256; b0 < total; b0 += (long long)gridDim.x * 256) {
     const long long v = b0 + threadIdx.x;
     DEntry e{0, 0, kHole, 0u};
@@ -563,20 +519,15 @@ void keep_pool_memory() {
   cudaGetLastError();
 }
 
-bool defer_enabled(int MODE) {
-  static const int env = [] { const char* e = getenv("SPADE_DEFER"); return e ? atoi(e) : -1; }();
-  if (env >= 0) return env != 0;
-  return MODE == kSelect || MODE == kPairs || true;
-}
-
-template <int MODE, int T, int U, int PF, int COMPACT>
+template <int MODE, int COMPACT, int QUEUE>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
-  const size_t smem = tiles_bytes_for(c->d.Wc, c->d.Hc) + (T / 32) * qcap_for(U) * sizeof(QEntry) + extra_smem;
-  auto kern = k_probe<MODE, T, U, PF, COMPACT>;
+  const size_t smem = tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? kNW * kQCap * sizeof(QEntry) : 0);
+  auto kern = k_probe<MODE, COMPACT, QUEUE>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
   const int sms = device_sm_count();
-  // launches of fewer than 2^31 points (32-bit vector indices and queue point offsets)
+  keep_pool_memory();
+  // launches of fewer than 2^31 points (32-bit vector indices and point offsets)
   const int64_t kMax = (1ll << 31) - 64;
   for (int64_t off = 0; off < n; off += kMax) {
     const int64_t m = std::min(kMax, n - off);
@@ -587,85 +538,52 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.head = std::min<int64_t>(m, (int64_t)(((32 - (addr & 31)) & 31) / 8));
     p.nvec = (m - p.head) / 4;
     p.o.id_base = base.o.id_base + off;
-    const int64_t chunks = (p.nvec + (int64_t)T * U - 1) / ((int64_t)T * U);
+    const int64_t chunks = (p.nvec + kT - 1) / kT;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(sms, chunks));
-    // deferred boundary regions: n/grid/8 entries per CTA (overflow falls back to in-loop drains)
+    // deferral regions: n/grid/16 entries per CTA (6.25% boundary points; more are tested in place)
+    const int64_t per = QUEUE ? 0 : std::min<int64_t>(std::max<int64_t>(m / grid / 16, 1024), 1 << 22);
     DEntry* dbuf = nullptr;
     unsigned int* dfill = nullptr;
-    if (defer_enabled(MODE)) {
-      keep_pool_memory();
-      const int64_t per = std::min<int64_t>(std::max<int64_t>(m / grid / 16, 1024), 1 << 22);
-      p.defer_cap = (uint32_t)per;
-      if (cudaMallocAsync((void**)&dbuf, sizeof(DEntry) * per * grid, st) != cudaSuccess ||
-          cudaMallocAsync((void**)&dfill, sizeof(unsigned int) * grid, st) != cudaSuccess) {
-        cudaGetLastError();                       // no scratch: drain in-loop instead
+    if (!QUEUE) {
+      e = cudaMallocAsync((void**)&dbuf, sizeof(DEntry) * per * grid, st);
+      if (e == cudaSuccess) e = cudaMallocAsync((void**)&dfill, sizeof(unsigned int) * grid, st);
+      if (e != cudaSuccess) {
         if (dbuf) cudaFreeAsync(dbuf, st);
-        dbuf = nullptr; dfill = nullptr;
+        return check_cuda(e, "probe scratch");
       }
-      p.defer = dbuf;
-      p.defer_fill = dfill;
     }
-    kern<<<grid, T, smem, st>>>(p);
+    p.defer = dbuf;
+    p.defer_cap = (uint32_t)per;
+    p.defer_fill = dfill;
+    kern<<<grid, kT, smem, st>>>(p);
     count_launch();
     e = cudaGetLastError();
-    if (e != cudaSuccess) return check_cuda(e, "probe launch");
-    if (dbuf) {
+    if (e == cudaSuccess && !QUEUE) {
       const int P = c->d.num_polys;
-      const int sh = (MODE == kCountSmem && (size_t)P * 4 <= 96 * 1024) ? 1 : 0;
+      const int sh = ((MODE == kCountSmem || MODE == kCountGlobal) && (size_t)P * 4 <= 96 * 1024) ? 1 : 0;
       const size_t dsm = sh ? (size_t)P * 4 : 0;
       if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
       k_deferred<MODE><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh);
       count_launch();
       e = cudaGetLastError();
-      cudaFreeAsync(dbuf, st);
-      cudaFreeAsync(dfill, st);
-      if (e != cudaSuccess) return check_cuda(e, "deferred boundary launch");
     }
+    if (dbuf) cudaFreeAsync(dbuf, st);
+    if (dfill) cudaFreeAsync(dfill, st);
+    if (e != cudaSuccess) return check_cuda(e, "probe launch");
   }
   return SPADE_OK;
 }
 
-constexpr size_t kSmemBudget = 227 * 1024;
-
-// Launch-shape variants of the probe (threads per CTA, 4-point vectors per thread per batch,
-// register double-buffered prefetch of the next batch).  SPADE_PROBE_VARIANT=<i> overrides the
-// default for tuning runs; the default is the measured best.
-struct Variant { int T, U, PF; };
-constexpr Variant kVariants[] = {{1024, 1, 1}, {768, 1, 1}, {512, 1, 1}};
-constexpr int kDefaultVariant = 0;
-
-int variant_index() {
-  static int v = [] {
-    const char* e = getenv("SPADE_PROBE_VARIANT");
-    int i = e ? atoi(e) : kDefaultVariant;
-    return (i >= 0 && i < (int)(sizeof(kVariants) / sizeof(kVariants[0]))) ? i : kDefaultVariant;
-  }();
-  return v;
-}
-
-template <int MODE, int COMPACT>
-int launch_variant2(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
-  switch (variant_index()) {
-    case 1: return launch<MODE, 768, 1, 1, COMPACT>(c, xy, n, p, extra, st);
-    case 2: return launch<MODE, 512, 1, 1, COMPACT>(c, xy, n, p, extra, st);
-    default: return launch<MODE, 1024, 1, 1, COMPACT>(c, xy, n, p, extra, st);
-  }
-}
-
-template <int MODE>
-int launch_variant(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
-  return c->d.compact ? launch_variant2<MODE, 1>(c, xy, n, p, extra, st) : launch_variant2<MODE, 0>(c, xy, n, p, extra, st);
-}
-
-size_t fixed_smem(const spade_canvas* c) {
-  const Variant v = kVariants[variant_index()];
-  return tiles_bytes_for(c->d.Wc, c->d.Hc) + (v.T / 32) * qcap_for(v.U) * sizeof(QEntry);
+template <int MODE, int QUEUE = 0>
+int launch_layout(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
+  return c->d.compact ? launch<MODE, 1, QUEUE>(c, xy, n, p, extra, st) : launch<MODE, 0, QUEUE>(c, xy, n, p, extra, st);
 }
 
 Params base_params(const spade_canvas* c) {
   Params p{};
   p.cv = c->d;
   p.cvg = c->d_dev;
+  p.hcopies = 1;
   return p;
 }
 
@@ -675,9 +593,25 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.counts = (unsigned long long*)counts;
-  const size_t hist = (size_t)kHC * (c->d.num_polys + 1) * 4;
-  if (fixed_smem(c) + hist <= kSmemBudget) return launch_variant<kCountSmem>(c, (const int2*)xy, n, p, hist, st);
-  return launch_variant<kCountGlobal>(c, (const int2*)xy, n, p, 0, st);
+  // shared-memory histogram: as many copies (8, 4, 2, 1) as stay under the L1-preserving budget;
+  // boundary points tested in the loop (warp queues) when those fit too, else deferred
+  const size_t tiles = tiles_bytes_for(c->d.Wc, c->d.Hc);
+  const size_t one = (size_t)(c->d.num_polys + 1) * 4;
+  const size_t queue = (size_t)kNW * kQCap * sizeof(QEntry);
+  static const int force_defer = [] { const char* e = getenv("SPADE_DEFER"); return e ? atoi(e) : 0; }();
+  for (uint32_t hc = 8; hc >= 1; hc >>= 1) {
+    if (!force_defer && tiles + hc * one + queue <= kSmemSoft) {
+      p.hcopies = hc;
+      return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hc * one, st);
+    }
+  }
+  for (uint32_t hc = 8; hc >= 1; hc >>= 1) {
+    if (tiles + hc * one <= kSmemSoft || (hc == 1 && tiles + one <= 227 * 1024)) {
+      p.hcopies = hc;
+      return launch_layout<kCountSmem>(c, (const int2*)xy, n, p, hc * one, st);
+    }
+  }
+  return launch_layout<kCountGlobal>(c, (const int2*)xy, n, p, 0, st);
 }
 
 int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* out, int64_t cap,
@@ -685,7 +619,7 @@ int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t b
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = out; p.o.cap = cap; p.o.total = d_total;
-  return launch_variant<kSelect>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
+  return launch_layout<kSelect>(c, (const int2*)xy, n, p, kScanBytes, st);
 }
 
 int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* opt, int32_t* opl,
@@ -693,7 +627,7 @@ int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t ba
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = opt; p.o.out_poly = opl; p.o.cap = cap; p.o.total = d_total;
-  return launch_variant<kPairs>(c, (const int2*)xy, n, p, 128 * sizeof(int) + 32 * sizeof(long long), st);
+  return launch_layout<kPairs>(c, (const int2*)xy, n, p, kScanBytes, st);
 }
 
 }  // namespace spade
