@@ -85,7 +85,7 @@ def c4(n_points: int = 1_000_000_000) -> Workload:
 
 def c5(n_points_per_gpu: int = 1_000_000_000) -> Workload:
     return Workload("c5_taxi1Bpergpu_x40k_zip_count", "count", taxi_params(501), 501, n_points_per_gpu,
-                    pg.jittered_tiling(200, 200, 375, seed=502), max_dim=8192,
+                    pg.jittered_tiling(200, 200, 375, seed=502), max_dim=16384,
                     desc="scale-out join COUNT: 1B points per GPU x 40k zip-code-like polygons")
 
 

@@ -540,8 +540,12 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.o.id_base = base.o.id_base + off;
     const int64_t chunks = (p.nvec + kT - 1) / kT;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(sms, chunks));
-    // deferral regions: n/grid/16 entries per CTA (6.25% boundary points; more are tested in place)
-    const int64_t per = QUEUE ? 0 : std::min<int64_t>(std::max<int64_t>(m / grid / 16, 1024), 1 << 22);
+    // deferral regions sized from the canvas's boundary-pixel fraction fb (points are not uniform,
+    // so 2 fb + 4%, at most all points); overflowing points are tested in place (slow, rare)
+    const double fb = (double)c->num_runs / ((double)c->d.W * (double)c->d.H);
+    const double frac = std::min(1.0, 2.0 * fb + 0.04);
+    const int64_t per = QUEUE ? 0 : std::min<int64_t>(std::max<int64_t>((int64_t)(frac * (double)m / grid) + 64, 1024),
+                                                       (int64_t)1 << 26);
     DEntry* dbuf = nullptr;
     unsigned int* dfill = nullptr;
     if (!QUEUE) {
