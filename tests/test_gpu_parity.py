@@ -134,3 +134,57 @@ def test_tiling_with_islands_exactly_one_owner(spade):
     pt, pl = spade.join_pairs(cv, torch.as_tensor(xy).cuda())
     pt = pt.cpu().numpy()
     assert len(pt) == len(xy) and len(np.unique(pt)) == len(xy)   # every point in exactly one polygon
+
+
+def test_host_streaming_count_matches_oracle(spade):
+    """spade_join_count_host (host-resident points, chunked H2D overlapped with the probe)."""
+    import torch
+    w = configs.c1()
+    xy = np.concatenate([gen.points_host(w.points, w.point_seed, 0, 300_000), configs.c1_edge_points(w.polys)])
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    got = spade.join_count_host(cv, xy)                                  # pageable numpy buffer
+    np.testing.assert_array_equal(got, oracle.join_count(xy, w.polys))
+    pinned = torch.from_numpy(xy).pin_memory()
+    acc = np.full(cv.num_polys, 7, np.int64)                            # accumulates into counts
+    spade.join_count_host(cv, pinned, acc)
+    np.testing.assert_array_equal(acc - 7, got)
+
+
+def test_invalid_arguments_are_reported(spade):
+    import ctypes
+    import torch
+    lib = spade.load()
+    w = configs.c1()
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    xy = torch.zeros((8, 2), dtype=torch.int32, device="cuda")
+    counts = torch.zeros(cv.num_polys, dtype=torch.int64, device="cuda")
+    s = ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    P = ctypes.c_void_p
+    assert lib.spade_join_count(None, P(xy.data_ptr()), 8, P(counts.data_ptr()), s) == spade.SPADE_ERR_INVALID_ARG
+    assert lib.spade_join_count(cv.handle, P(xy.data_ptr()), -1, P(counts.data_ptr()), s) == spade.SPADE_ERR_INVALID_ARG
+    assert lib.spade_join_count(cv.handle, None, 8, P(counts.data_ptr()), s) == spade.SPADE_ERR_INVALID_ARG
+    assert lib.spade_join_count(cv.handle, P(xy.data_ptr() + 4), 7, P(counts.data_ptr()), s) == spade.SPADE_ERR_INVALID_ARG
+    assert lib.spade_join_count(cv.handle, None, 0, P(counts.data_ptr()), s) == spade.SPADE_OK   # n == 0: no-op
+    n_out = ctypes.c_int64()
+    assert lib.spade_select(cv.handle, P(xy.data_ptr()), 8, 0, None, 0, None, s) == spade.SPADE_ERR_INVALID_ARG
+    assert lib.spade_select(cv.handle, P(xy.data_ptr()), 8, 0, None, -5, ctypes.byref(n_out), s) == spade.SPADE_ERR_INVALID_ARG
+    assert b"negative" in lib.spade_last_error()
+    bad = {"ring_xy": np.zeros((3, 2), np.int32), "ring_off": np.array([0, 2, 1], np.int64),
+           "poly_ring_off": np.array([0, 2], np.int64)}
+    with pytest.raises(spade.SpadeError) as e:
+        spade.Canvas(bad)
+    assert e.value.code == spade.SPADE_ERR_INVALID_ARG
+
+
+def test_results_independent_of_point_id_base_and_chunking(spade):
+    import torch
+    w = configs.c1()
+    xy = torch.as_tensor(gen.points_host(w.points, w.point_seed, 0, 50_000)).cuda()
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    full = spade.join_count(cv, xy)
+    parts = torch.zeros_like(full)
+    for a in range(0, 50_000, 7_919):
+        spade.join_count(cv, xy[a:a + 7_919], parts)
+    assert torch.equal(full, parts)
+    pt, pl = spade.join_pairs(cv, xy, point_id_base=10**12)
+    assert int(pt.min()) >= 10**12 and int(pt.max()) < 10**12 + 50_000
