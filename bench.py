@@ -161,6 +161,28 @@ def cpu_oracle_rate(w, target_s, seed_offset=0):
                       f"({dt:.1f} s)", "seconds": dt, "sum_counts": int(counts.sum())}
 
 
+def cpu_rtree_rate(w, target_s):
+    """The simple R-tree CPU join (STR over polygon bboxes + exact predicate), as it stands, on an
+    index-strided sample of the workload's points, all host cores."""
+    import numpy as np
+    import gen
+    import oracle
+    nt = oracle.default_threads()
+    pilot = gen.points_at(w.points, w.point_seed, np.arange(0, 20000, dtype=np.int64) * 4999)
+    t0 = time.perf_counter()
+    oracle.rtree_join_count(pilot, w.polys, nthreads=nt)
+    dt = max(time.perf_counter() - t0, 1e-3)
+    m = int(max(20000, min(50_000_000, len(pilot) * target_s / dt)))
+    stride = max(1, w.n_points // m)
+    xy = gen.points_at(w.points, w.point_seed, np.arange(m, dtype=np.int64) * stride)
+    t0 = time.perf_counter()
+    oracle.rtree_join_count(xy, w.polys, nthreads=nt)
+    dt = time.perf_counter() - t0
+    return {"value": m / dt, "unit": "points/s", "cores": nt, "kind": "rtree",
+            "sample": f"{m} points = every {stride}-th global index, STR R-tree over "
+                      f"{len(w.polys['poly_ring_off']) - 1} polygon bboxes + exact predicate ({dt:.1f} s)"}
+
+
 def run_reference(a):
     ws, rank, _ = dist_env()
     if rank != 0:
@@ -361,6 +383,7 @@ def main():
         cb.pop("seconds", None)
         cb.pop("sum_counts", None)
         line["cpu_baseline"] = cb
+        line["cpu_rtree_baseline"] = cpu_rtree_rate(w, a.cpu_seconds / 2)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if ws > 1:

@@ -23,10 +23,12 @@ _lib = None
 
 
 def build(force: bool = False) -> str:
-    """Compile spade_oracle.c into liboracle.so (plain gcc, -O2, pthreads)."""
-    src = os.path.join(_HERE, "spade_oracle.c")
-    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(src):
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-pthread", "-o", _LIB_PATH, src])
+    """Compile spade_oracle.c (+ the R-tree CPU baseline, rtree_join.c) into liboracle.so
+    (plain gcc, -O2, pthreads)."""
+    srcs = [os.path.join(_HERE, "spade_oracle.c"), os.path.join(_HERE, "rtree_join.c")]
+    newest = max(os.path.getmtime(x) for x in srcs)
+    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < newest:
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-pthread", "-o", _LIB_PATH, *srcs])
     return _LIB_PATH
 
 
@@ -45,6 +47,8 @@ def _load():
         lib.oracle_join_pairs.restype = i64
         lib.oracle_select.argtypes = [P, i64, i64, P, P, P, i32, P, i64, ctypes.c_int]
         lib.oracle_select.restype = i64
+        lib.rtree_join_count.argtypes = [P, i64, P, P, P, i32, P, ctypes.c_int]
+        lib.rtree_join_count.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -114,6 +118,20 @@ def select(xy, polys, point_id_base: int = 0, nthreads: int | None = None) -> np
     if total < 0:
         raise MemoryError("oracle_select failed")
     return out[:total]
+
+
+def rtree_join_count(xy, polys, nthreads: int | None = None) -> np.ndarray:
+    """COUNT by the simple R-tree CPU join (STR over polygon bboxes + the same exact predicate);
+    the second CPU baseline of BASELINE.json's north_star.  Identical results to join_count."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    ring_xy, ring_off, poly_ring_off, P = _polys(polys)
+    counts = np.zeros(max(P, 1), dtype=np.int64)
+    rc = lib.rtree_join_count(_ptr(xy), len(xy), _ptr(ring_xy), _ptr(ring_off), _ptr(poly_ring_off), P,
+                              _ptr(counts), nthreads or default_threads())
+    if rc != 0:
+        raise MemoryError("rtree_join_count failed")
+    return counts[:P]
 
 
 def labels_at(xy, polys, nthreads: int | None = None):

@@ -239,3 +239,17 @@ def test_select_pairs_count_agree():
     assert np.bincount(pl, minlength=len(counts)).tolist() == counts.tolist()
     assert ids.tolist() == sorted(set(pt.tolist()))
     assert counts.sum() > len(ids) > 0          # config 1 overlaps: some points in >1 polygon
+
+
+# --------------------------------------------------------------------------------------------
+# 7. the R-tree CPU baseline agrees with the brute-force oracle
+
+@pytest.mark.parametrize("seed", range(3))
+def test_rtree_baseline_matches_oracle(seed):
+    rng = np.random.default_rng(500 + seed)
+    polys = random_polyset(rng, 0, 60, 12)
+    xy = lattice(-3, -3, 63, 63)
+    assert oracle.rtree_join_count(xy, polys).tolist() == oracle.join_count(xy, polys).tolist()
+    t = pg.jittered_tiling(7, 5, 20, domain=1 << 18, n_islands=3, seed=seed)
+    xy2 = gen.points_host(gen.taxi_params(seed, domain=1 << 18), seed, 0, 20000)
+    assert oracle.rtree_join_count(xy2, t).tolist() == oracle.join_count(xy2, t).tolist()
