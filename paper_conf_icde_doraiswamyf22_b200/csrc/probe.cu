@@ -44,8 +44,9 @@ struct alignas(32) Vec4 { int4 a, b; };   // 4 points
 struct alignas(16) DEntry { int x, y; uint32_t rec, pidx; };
 constexpr uint32_t kHole = 0xffffffffu;   // DEntry.rec of a reserved-but-unused slot
 
-// Boundary point in a warp's shared-memory queue (COUNT with an in-loop exact test).
-struct alignas(8) QEntry { uint32_t rec, pidx; };
+// Boundary point in a warp's shared-memory queue (COUNT with an in-loop exact test): just the
+// point; the drain re-derives its record from the canvas (shared memory + an L2-resident pixel).
+struct alignas(8) QEntry { int x, y; };
 constexpr int kQCap = 32 + 32 * kNPT;     // < 32 left over + one batch of the warp's points
 
 __device__ __forceinline__ Vec4 ld_stream(const Vec4* p) {
@@ -210,14 +211,17 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
 }
 
 // COUNT, in-loop variant: evaluate up to 32 queued boundary points (one per lane).  Out of line:
-// the streaming loop keeps a small register footprint.  The point is re-read here (L2).
+// the streaming loop keeps a small register footprint.
 template <int MODE>
-__device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const int2* __restrict__ xy, const QEntry* wq,
+__device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const QEntry* wq,
                                    int cnt, int lane, unsigned int* hist, unsigned long long* counts) {
   if (lane < cnt) {
     const QEntry e = wq[lane];
-    const int2 p = __ldg(xy + e.pidx);
-    pip_eval(cvg, p.x, p.y, e.rec, [&](int q) { count_hit<MODE>(hist, counts, q); });
+    const CanvasDev& cv = *cvg;
+    const uint32_t fx = ((uint32_t)e.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)e.y - (uint32_t)cv.miny) >> cv.s;
+    const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
+    const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
+    pip_eval(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, counts, q); });
   }
 }
 
@@ -329,13 +333,17 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
           int pos = atomicAdd(&s_qn[warp], __popc(bnd));
 #pragma unroll
           for (int q = 0; q < NPT; ++q)
-            if ((bnd >> q) & 1u) wq[pos++] = QEntry{~c[q], (uint32_t)prm.head + 4 * (base + tid) + q};
+            if ((bnd >> q) & 1u) {
+              const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+              const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+              wq[pos++] = QEntry{x, y};
+            }
         }
         __syncwarp();
         int qn = s_qn[warp];
         if (qn >= 32) {
           do {
-            drain<MODE>(prm.cvg, prm.xy, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+            drain<MODE>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
             qn -= 32;
           } while (qn >= 32);
           __syncwarp();
@@ -421,7 +429,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   }
   if (QUEUE) {
     __syncwarp();
-    if (s_qn[warp] > 0) drain<MODE>(prm.cvg, prm.xy, wq, s_qn[warp], lane, myhist, prm.o.counts);
+    if (s_qn[warp] > 0) drain<MODE>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.o.counts);
   }
   __syncthreads();
   if (!QUEUE && tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
