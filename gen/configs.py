@@ -73,7 +73,7 @@ def c2(n_points: int = 100_000_000) -> Workload:
 
 def c3(n_points: int = 1_000_000_000) -> Workload:
     return Workload("c3_taxi1B_x260_neighborhoods_count", "count", taxi_params(301), 301, n_points,
-                    pg.jittered_tiling(20, 13, 135, seed=302), max_dim=8192,
+                    pg.jittered_tiling(20, 13, 135, seed=302), max_dim=16384,
                     desc="point-polygon join COUNT: 1B taxi-like points x 260 neighborhood-like polygons")
 
 

@@ -481,10 +481,10 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
         if (sh) atomicAdd(&dh[q], 1u); else atomicAdd(o.counts + q, 1ull);
       });
     } else {
-      int nres = 0;
+      int nres = 0, first = -1;
       if (act) {
         if (MODE == kSelect) { bool any = false; pip_eval(cvg, e.x, e.y, e.rec, [&](int) { any = true; }); nres = any; }
-        else pip_eval(cvg, e.x, e.y, e.rec, [&](int) { ++nres; });
+        else pip_eval(cvg, e.x, e.y, e.rec, [&](int q) { if (nres++ == 0) first = q; });
       }
       int excl, tot;
       BS(tmp).ExclusiveSum(nres, excl, tot);
@@ -494,6 +494,8 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
       if (nres) {
         if (MODE == kSelect) {
           if (pos < o.cap) o.out_ids[pos] = pid;
+        } else if (nres == 1) {                    // the common case: no second evaluation
+          if (pos < o.cap) { o.out_ids[pos] = pid; o.out_poly[pos] = first; }
         } else {
           pip_eval(cvg, e.x, e.y, e.rec, [&](int q) {
             if (pos < o.cap) { o.out_ids[pos] = pid; o.out_poly[pos] = q; }
