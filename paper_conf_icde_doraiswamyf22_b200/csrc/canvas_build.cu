@@ -193,12 +193,96 @@ __global__ void k_local(const Frag* __restrict__ frags, int64_t F, int W, const 
   }
 }
 
-__global__ void k_gather_edges(const int32_t* __restrict__ sorted_e, int64_t L, const int4* __restrict__ seg,
-                               const int32_t* __restrict__ poly, int4* __restrict__ rseg, int32_t* __restrict__ rpoly) {
+// --- pixel-local edge de-duplication (an edge shared by two polygons, or used twice, is stored
+// once with a polygon toggle mask) ---------------------------------------------------------------
+// entries sorted by (bid, poly): head of each distinct (bid, poly)
+__global__ void k_iota(int32_t* __restrict__ a, int64_t n) {
+  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < n; t += (int64_t)gridDim.x * kBT) a[t] = (int32_t)t;
+}
+
+__global__ void k_polyhead(const uint64_t* __restrict__ key, int64_t L, int32_t* __restrict__ head) {
+  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < L; t += (int64_t)gridDim.x * kBT)
+    head[t] = (t == 0 || key[t] != key[t - 1]) ? 1 : 0;
+}
+
+// pg = inclusive scan of head: distinct (bid, poly) index pg - 1; per-record polygon range
+__global__ void k_recpolys(const uint64_t* __restrict__ key, int64_t L, const int32_t* __restrict__ head,
+                           const int32_t* __restrict__ pg, int32_t* __restrict__ rec_polys) {
+  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < L; t += (int64_t)gridDim.x * kBT)
+    if (head[t]) rec_polys[pg[t] - 1] = (int32_t)(key[t] & 0xffffffffu);
+}
+
+__global__ void k_polyrange(int64_t NB, const int64_t* __restrict__ le_beg, const int32_t* __restrict__ le_cnt,
+                            const int32_t* __restrict__ pg, int32_t* __restrict__ pbeg, int32_t* __restrict__ pcnt) {
+  for (int64_t b = blockIdx.x * (int64_t)kBT + threadIdx.x; b < NB; b += (int64_t)gridDim.x * kBT) {
+    const int32_t n = le_cnt[b];
+    if (n == 0) { pbeg[b] = 0; pcnt[b] = 0; continue; }
+    const int64_t e0 = le_beg[b];
+    pbeg[b] = pg[e0] - 1;
+    pcnt[b] = pg[e0 + n - 1] - pg[e0] + 1;
+  }
+}
+
+__device__ __forceinline__ uint32_t seg_hash(int4 e) {
+  // canonical orientation, then a 64-bit mix folded to 32 bits
+  int ax = e.x, ay = e.y, bx = e.z, by = e.w;
+  if (bx < ax || (bx == ax && by < ay)) { int t = ax; ax = bx; bx = t; t = ay; ay = by; by = t; }
+  uint64_t h = ((uint64_t)(uint32_t)ax << 32 | (uint32_t)ay) * 0x9E3779B97F4A7C15ull;
+  h ^= ((uint64_t)(uint32_t)bx << 32 | (uint32_t)by) + 0x632BE59BD9B4E019ull + (h << 6) + (h >> 2);
+  h ^= h >> 29; h *= 0xBF58476D1CE4E5B9ull; h ^= h >> 32;
+  return (uint32_t)h;
+}
+__device__ __forceinline__ bool same_seg(int4 a, int4 b) {
+  return (a.x == b.x && a.y == b.y && a.z == b.z && a.w == b.w) || (a.x == b.z && a.y == b.w && a.z == b.x && a.w == b.y);
+}
+
+// per entry (sorted by (bid, poly)): local polygon index and the (bid, segment hash) key
+__global__ void k_segkey(const uint64_t* __restrict__ key, const int32_t* __restrict__ ev, int64_t L,
+                         const int4* __restrict__ seg, const int32_t* __restrict__ pg, const int32_t* __restrict__ pbeg,
+                         uint64_t* __restrict__ key2, int32_t* __restrict__ li) {
   for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < L; t += (int64_t)gridDim.x * kBT) {
-    int32_t e = sorted_e[t];
-    rseg[t] = seg[e];
-    rpoly[t] = poly[e];
+    const uint32_t bid = (uint32_t)(key[t] >> 32);
+    li[t] = pg[t] - 1 - pbeg[bid];
+    key2[t] = ((uint64_t)bid << 32) | seg_hash(seg[ev[t]]);
+  }
+}
+
+// entries sorted by (bid, hash): the first occurrence of each exact segment within its equal-key
+// run carries the XOR of the polygon bits of all its occurrences; zero masks (a segment used
+// an even number of times by the same polygons) contribute nothing and are dropped.  Records with
+// more than kMaskPolys polygons keep every entry with its local index.
+template <int PASS>
+__global__ void k_merge(const uint64_t* __restrict__ key2, const int32_t* __restrict__ tix, int64_t L,
+                        const int32_t* __restrict__ ev, const int32_t* __restrict__ li, const int4* __restrict__ seg,
+                        const int32_t* __restrict__ pcnt, const int64_t* __restrict__ le_beg, int32_t* __restrict__ mcnt,
+                        const int64_t* __restrict__ mbeg, int32_t* __restrict__ mfill,
+                        int4* __restrict__ oseg, uint64_t* __restrict__ omask) {
+  for (int64_t u = blockIdx.x * (int64_t)kBT + threadIdx.x; u < L; u += (int64_t)gridDim.x * kBT) {
+    const uint64_t k = key2[u];
+    const uint32_t bid = (uint32_t)(k >> 32);
+    const int4 e = seg[ev[tix[u]]];
+    uint64_t m;
+    const bool slow = pcnt[bid] > kMaskPolys;
+    if (slow) {
+      m = (uint64_t)li[tix[u]];
+    } else {
+      bool first = true;
+      for (int64_t w = u - 1; w >= 0 && key2[w] == k; --w)
+        if (same_seg(seg[ev[tix[w]]], e)) { first = false; break; }
+      if (!first) continue;
+      m = 1ull << li[tix[u]];
+      for (int64_t w = u + 1; w < L && key2[w] == k; ++w)
+        if (same_seg(seg[ev[tix[w]]], e)) m ^= 1ull << li[tix[w]];
+      if (m == 0) continue;
+    }
+    if (PASS == 0) {
+      atomicAdd(&mcnt[bid], 1);
+    } else {
+      // slow records keep the (bid, poly) order of the entries: grouped by local index
+      const int64_t pos = mbeg[bid] + (slow ? (int64_t)tix[u] - le_beg[bid] : (int64_t)atomicAdd(&mfill[bid], 1));
+      oseg[pos] = e;
+      omask[pos] = m;
+    }
   }
 }
 
@@ -266,8 +350,10 @@ __device__ __forceinline__ int cu_test(int4 e, int64_t qx, int64_t qy) {
 template <int PASS>
 __global__ void k_kset(int64_t NB, const int64_t* __restrict__ pix_of, Geo g, const int32_t* __restrict__ corner,
                        const int32_t* __restrict__ csets, const int2* __restrict__ crng,
-                       const int64_t* __restrict__ le_beg, const int32_t* __restrict__ le_cnt,
-                       const int4* __restrict__ rseg, const int32_t* __restrict__ rpoly,
+                       const int64_t* __restrict__ mbeg, const int32_t* __restrict__ mcnt,
+                       const int4* __restrict__ rseg, const uint64_t* __restrict__ rmask,
+                       const int32_t* __restrict__ pbeg, const int32_t* __restrict__ pcnt,
+                       const int32_t* __restrict__ rec_polys,
                        int32_t* __restrict__ ksize, const int64_t* __restrict__ koff, int32_t* __restrict__ kout,
                        RunRec* __restrict__ recs) {
   for (int64_t b = blockIdx.x * (int64_t)kBT + threadIdx.x; b < NB; b += (int64_t)gridDim.x * kBT) {
@@ -281,28 +367,38 @@ __global__ void k_kset(int64_t NB, const int64_t* __restrict__ pix_of, Geo g, co
     int64_t out = big ? koff[b] : 0;
     int n = 0;
     int32_t first = kEmpty;
-    const int64_t e0 = le_beg[b], e1 = e0 + le_cnt[b];
-    int64_t e = e0;
+    const int64_t e0 = mbeg[b], e1 = e0 + mcnt[b];
+    const int32_t pb = pbeg[b], pc = pcnt[b];
+    auto put = [&](int32_t Q) {
+      if (big) kout[out++] = Q;
+      if (n == 0) first = Q;
+      ++n;
+    };
     int ci = 0;
-    while (e < e1 || ci < cn) {
-      const int32_t P = e < e1 ? rpoly[e] : INT32_MAX;
-      const int32_t Cp = ci < cn ? (cv >= 0 ? cv : csets[cb + ci]) : INT32_MAX;
-      int par = 0;
-      int32_t Q;
-      if (Cp < P) { Q = Cp; par = 1; ++ci; }
-      else {
-        Q = P;
-        for (; e < e1 && rpoly[e] == P; ++e) par ^= cu_test(rseg[e], X, Y0);
-        if (Cp == P) { par ^= 1; ++ci; }
+    auto cel = [&](int k) { return cv >= 0 ? cv : csets[cb + k]; };
+    auto merge_upto = [&](int32_t P, int par) {      // corner-set members < P pass through
+      while (ci < cn && cel(ci) < P) { put(cel(ci)); ++ci; }
+      if (ci < cn && cel(ci) == P) { par ^= 1; ++ci; }
+      if (par) put(P);
+    };
+    if (pc <= kMaskPolys) {
+      uint64_t m = 0;
+      for (int64_t e = e0; e < e1; ++e) if (cu_test(rseg[e], X, Y0)) m ^= rmask[e];
+      for (int k = 0; k < pc; ++k) {
+        const int par = (int)((m >> k) & 1u);
+        const int32_t P = rec_polys[pb + k];
+        merge_upto(P, par);
       }
-      if (par) {
-        if (big) kout[out++] = Q;
-        if (n == 0) first = Q;
-        ++n;
+    } else {
+      for (int k = 0; k < pc; ++k) {
+        int par = 0;
+        for (int64_t e = e0; e < e1; ++e) if ((int)rmask[e] == k) par ^= cu_test(rseg[e], X, Y0);
+        merge_upto(rec_polys[pb + k], par);
       }
     }
+    merge_upto(INT32_MAX, 0);
     if (PASS == 0) ksize[b] = n;
-    else recs[b] = RunRec{e0, (int32_t)(e1 - e0), first};   // |K| >= 2 fixed up by k_kset_rng
+    else recs[b] = RunRec{e0, (int32_t)(e1 - e0), first, pb, pc};   // |K| >= 2 fixed up by k_kset_rng
   }
 }
 
@@ -328,7 +424,7 @@ __global__ void k_finalize(int64_t WH, const int32_t* __restrict__ bflag, const 
 
 __global__ void k_multi_recs(int64_t NG, int64_t NB, RunRec* __restrict__ recs) {
   for (int64_t g = blockIdx.x * (int64_t)kBT + threadIdx.x; g < NG; g += (int64_t)gridDim.x * kBT)
-    recs[NB + g] = RunRec{0, 0, (int32_t)(-2 - g)};
+    recs[NB + g] = RunRec{0, 0, (int32_t)(-2 - g), 0, 0};
 }
 
 // K-B5: tile summary.  tval = owner + 1 / 0 for uniform tiles; mixed tiles flagged in tmix.
@@ -569,11 +665,47 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortPairs(t, sz, lk, lk2, lv, lv2, L, 0, 32 + bbits, st); }), "sort local edges");
   if (NB > 0)
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, le_cnt, le_beg, NB, st); }), "scan local edges");
-  if (cudaMalloc(&c->run_seg, sizeof(int4) * std::max<int64_t>(L, 1)) != cudaSuccess ||
-      cudaMalloc(&c->run_poly, sizeof(int32_t) * std::max<int64_t>(L, 1)) != cudaSuccess)
+  // distinct polygons per boundary pixel, local indices, de-duplicated edges with toggle masks
+  int32_t *ph, *pg, *pbeg, *pcnt, *li, *tix, *tix2, *mcnt, *mfill;
+  int64_t* mbeg;
+  uint64_t* key2s;
+  ALLOC(ph, L, "dedup"); ALLOC(pg, L, "dedup"); ALLOC(pbeg, NB, "dedup"); ALLOC(pcnt, NB, "dedup");
+  ALLOC(li, L, "dedup"); ALLOC(tix, L, "dedup"); ALLOC(tix2, L, "dedup"); ALLOC(key2s, L, "dedup");
+  ALLOC(mcnt, NB, "dedup"); ALLOC(mfill, NB, "dedup"); ALLOC(mbeg, NB + 1, "dedup");
+  int32_t D32 = 0;
+  if (L > 0) {
+    LAUNCH(k_polyhead, L, lk2, L, ph);
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, ph, pg, L, st); }), "scan polys");
+    TRYF(cudaMemcpyAsync(&D32, pg + L - 1, 4, cudaMemcpyDeviceToHost, st), "D");
+    TRYF(cudaStreamSynchronize(st), "sync polys");
+  }
+  if (cudaMalloc(&c->rec_polys, sizeof(int32_t) * std::max<int64_t>(D32, 1)) != cudaSuccess)
+    return fail(set_error(SPADE_ERR_OOM, "build: record polygon lists"));
+  if (L > 0) LAUNCH(k_recpolys, L, lk2, L, ph, pg, c->rec_polys);
+  if (NB > 0) LAUNCH(k_polyrange, NB, NB, le_beg, le_cnt, pg, pbeg, pcnt);
+  int64_t LM = 0;
+  TRYF(cudaMemsetAsync(mcnt, 0, sizeof(int32_t) * std::max<int64_t>(NB, 1), st), "memset");
+  TRYF(cudaMemsetAsync(mfill, 0, sizeof(int32_t) * std::max<int64_t>(NB, 1), st), "memset");
+  if (L > 0) {
+    LAUNCH(k_segkey, L, lk2, lv2, L, seg, pg, pbeg, lk, li);            // lk reused for (bid, hash) keys
+    LAUNCH(k_iota, L, tix, L);
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortPairs(t, sz, lk, key2s, tix, tix2, L, 0, 32 + bbits, st); }), "sort segments");
+    LAUNCH(k_merge<0>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, nullptr, nullptr, nullptr, nullptr);
+  }
+  if (NB > 0) {
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, mcnt, mbeg, NB, st); }), "scan merged");
+    int64_t lb = 0; int32_t lc = 0;
+    TRYF(cudaMemcpyAsync(&lb, mbeg + NB - 1, 8, cudaMemcpyDeviceToHost, st), "LM");
+    TRYF(cudaMemcpyAsync(&lc, mcnt + NB - 1, 4, cudaMemcpyDeviceToHost, st), "LM");
+    TRYF(cudaStreamSynchronize(st), "sync merged");
+    LM = lb + lc;
+  }
+  if (cudaMalloc(&c->run_seg, sizeof(int4) * std::max<int64_t>(LM, 1)) != cudaSuccess ||
+      cudaMalloc(&c->run_mask, sizeof(uint64_t) * std::max<int64_t>(LM, 1)) != cudaSuccess)
     return fail(set_error(SPADE_ERR_OOM, "build: local edge arrays"));
-  if (L > 0) LAUNCH(k_gather_edges, L, lv2, L, seg, epoly, c->run_seg, c->run_poly);
+  if (L > 0) LAUNCH(k_merge<1>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, mbeg, mfill, c->run_seg, c->run_mask);
   tmp.release(lk); tmp.release(lk2); tmp.release(lv); tmp.release(lv2); tmp.release(frags); tmp.release(lw_off);
+  tmp.release(ph); tmp.release(pg); tmp.release(li); tmp.release(tix); tmp.release(tix2); tmp.release(key2s);
 
   // --- K-B3 corner owner sets ---
   uint64_t* ev2;
@@ -625,8 +757,8 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   ALLOC(ksize, NB, "K sizes"); ALLOC(kidx, NB, "K sizes"); ALLOC(koff, NB + 1, "K offsets");
   int64_t KT = 0; int64_t NK = 0;
   if (NB > 0) {
-    LAUNCH(k_kset<0>, NB, NB, pix_of, g, corner, csets, crng, le_beg, le_cnt, c->run_seg, c->run_poly,
-           ksize, nullptr, nullptr, nullptr);
+    LAUNCH(k_kset<0>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, c->run_seg, c->run_mask,
+           pbeg, pcnt, c->rec_polys, ksize, nullptr, nullptr, nullptr);
     cub::TransformInputIterator<int64_t, BigSize, const int32_t*> it_sz(ksize, BigSize());
     cub::TransformInputIterator<int32_t, BigFlag, const int32_t*> it_b(ksize, BigFlag());
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, it_sz, koff, NB, st); }), "scan K");
@@ -650,8 +782,8 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
     TRYF(cudaMemcpyAsync(c->set_rng, crng, sizeof(int2) * NG, cudaMemcpyDeviceToDevice, st), "copy sets");
   }
   if (NB > 0) {
-    LAUNCH(k_kset<1>, NB, NB, pix_of, g, corner, csets, crng, le_beg, le_cnt, c->run_seg, c->run_poly,
-           ksize, koff, c->sets + M, c->runs);
+    LAUNCH(k_kset<1>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, c->run_seg, c->run_mask,
+           pbeg, pcnt, c->rec_polys, ksize, koff, c->sets + M, c->runs);
     LAUNCH(k_kset_rng, NB, NB, ksize, koff, kidx, NG, M, c->set_rng, c->runs);
   }
   if (NG > 0) LAUNCH(k_multi_recs, NG, NG, NB, c->runs);
@@ -688,7 +820,7 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   c->empty = false;
   c->num_runs = NB;
   c->num_records = NB + NG;
-  c->num_run_edges = L;
+  c->num_run_edges = LM;
   c->num_set_entries = M + KT;
   c->mixed_tile_frac = (double)h_mixed / ((double)Wc * Hc);
   CanvasDev& d = c->d;
@@ -698,7 +830,8 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   d.compact = compact ? 1 : 0;
   d.mix_min = compact ? kTileMixedCompact : kTileMixed;
   d.cfine = c->cfine;
-  d.fine = c->fine; d.coarse = c->coarse; d.runs = c->runs; d.run_seg = c->run_seg; d.run_poly = c->run_poly;
+  d.fine = c->fine; d.coarse = c->coarse; d.runs = c->runs; d.run_seg = c->run_seg; d.run_mask = c->run_mask;
+  d.rec_polys = c->rec_polys;
   d.sets = c->sets; d.set_rng = c->set_rng;
   if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
   if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));

@@ -115,7 +115,8 @@ __device__ __forceinline__ int local_bit(int4 e, int X, int px, int py) {
 }
 
 // Exact point-in-polygon for a point on boundary pixel (or multi-owner pixel) record `rec`:
-//   inside(p, P) = [P in K] XOR parity_P(local_bit over P's edges touching the pixel)
+//   inside(p, P) = [P in K] XOR parity_P(local_bit over P's edges touching the pixel),
+// the parities of all (<= 64) polygons of the pixel accumulated at once as a bit mask
 // emit(P) is called for every polygon containing the point, in increasing polygon order.
 template <class Emit>
 __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
@@ -135,23 +136,40 @@ __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int p
     if (par) emit(P);
   };
   const int4* seg = cv->run_seg;
-  const int32_t* poly = cv->run_poly;
-  int cur = -1, par = 0;
+  const uint64_t* msk = cv->run_mask;
+  const int32_t* rp = cv->rec_polys + r.poly_begin;
   const int64_t e1 = r.edge_begin + r.edge_cnt;
-  for (int64_t e = r.edge_begin; e < e1; ++e) {
-    const int4 g = __ldg(seg + e);
-    // an edge that straddles neither the horizontal line y = py nor the vertical line x = X
-    // contributes nothing (cr and cu are both 0): skip it without the cross product or its id
-    if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
-    if (!local_bit(g, X, px, py)) continue;
-    const int p = __ldg(poly + e);
-    if (p != cur) {
-      if (cur >= 0) finalize(cur, par);
-      cur = p; par = 0;
+  if (r.poly_cnt <= kMaskPolys) {
+    // each de-duplicated edge toggles the parity of every polygon that uses it
+    uint64_t m = 0;
+    for (int64_t e = r.edge_begin; e < e1; ++e) {
+      const int4 g = __ldg(seg + e);
+      // an edge that straddles neither the horizontal line y = py nor the vertical line x = X
+      // contributes nothing (cr and cu are both 0): skip it without the cross product or its mask
+      if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
+      if (local_bit(g, X, px, py)) m ^= __ldg(msk + e);
     }
-    par ^= 1;
+    while (m) {
+      const int k = __ffsll((long long)m) - 1;
+      m &= m - 1;
+      finalize(__ldg(rp + k), 1);
+    }
+  } else {
+    // > kMaskPolys polygons: edges grouped by local polygon index (run_mask = index)
+    int cur = -1, par = 0;
+    for (int64_t e = r.edge_begin; e < e1; ++e) {
+      const int4 g = __ldg(seg + e);
+      if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
+      if (!local_bit(g, X, px, py)) continue;
+      const int k = (int)__ldg(msk + e);
+      if (k != cur) {
+        if (cur >= 0 && par) finalize(__ldg(rp + cur), 1);
+        cur = k; par = 0;
+      }
+      par ^= 1;
+    }
+    if (cur >= 0 && par) finalize(__ldg(rp + cur), 1);
   }
-  if (cur >= 0) finalize(cur, par);
   while (ti < tn) emit(term_at(ti++));
 }
 

@@ -94,7 +94,7 @@ int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const in
 void spade_canvas_free(spade_canvas* c) {
   if (!c) return;
   cudaDeviceSynchronize();
-  cudaFree(c->fine); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->runs); cudaFree(c->run_seg); cudaFree(c->run_poly);
+  cudaFree(c->fine); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->runs); cudaFree(c->run_seg); cudaFree(c->run_mask); cudaFree(c->rec_polys);
   cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->d_dev);
   delete c;
 }

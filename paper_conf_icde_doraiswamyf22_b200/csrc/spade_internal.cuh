@@ -21,15 +21,21 @@ constexpr int32_t kMultiMark = INT32_MIN;     // transient during the fill only
 // the tile's pixels are the m-th block of 2^b x 2^b int32 in cfine (only mixed tiles stored).
 constexpr uint16_t kTileEmpty = 0, kTileMixed = 0xFFFF, kTileMixedCompact = 0x8000;
 
-// Boundary-index record.  For a boundary pixel: the edges touching the closed pixel,
-// [edge_begin, +edge_cnt) in run_seg/run_poly (sorted by polygon), and the corrected corner set K
-// (`term`).  For a multi-owner non-boundary pixel: edge_cnt = 0 and term =
-// its owner set.  term >= 0: {term};  term == -1: {};  term <= -2: set m = -2 - term (sets/set_rng).
+// Boundary-index record.  For a boundary pixel: the distinct polygons whose edges touch the
+// closed pixel, rec_polys[poly_begin, +poly_cnt) (ascending), the de-duplicated edges
+// [edge_begin, +edge_cnt) in run_seg with run_mask = XOR of (1 << local polygon index) over the
+// polygons using that segment (an edge shared by two polygons is stored once; poly_cnt > 64:
+// run_mask holds one local index per edge, no merging), and the corrected corner set K (`term`;
+// DESIGN.md "Canvas").  For a multi-owner non-boundary pixel: no edges, term = its owner set.
+// term >= 0: {term};  term == -1: {};  term <= -2: set m = -2 - term (sets/set_rng).
 struct RunRec {
   int64_t edge_begin;
   int32_t edge_cnt;
   int32_t term;
+  int32_t poly_begin;
+  int32_t poly_cnt;
 };
+constexpr int kMaskPolys = 64;     // records with more distinct polygons use the slow path
 
 struct CanvasDev {            // passed by value to kernels
   int32_t minx, miny;         // extent origin
@@ -47,7 +53,8 @@ struct CanvasDev {            // passed by value to kernels
   const uint16_t* coarse;
   const RunRec* runs;         // records: boundary pixels, then multi-owner pixels
   const int4* run_seg;        // (ax, ay, bx, by) of the edges touching each boundary pixel
-  const int32_t* run_poly;
+  const uint64_t* run_mask;   // polygon toggle mask (or local polygon index) per edge
+  const int32_t* rec_polys;   // distinct polygons of each record
   const int32_t* sets;        // concatenated sorted owner sets
   const int2* set_rng;        // (begin, count)
 };
@@ -66,7 +73,8 @@ struct spade_canvas {
   uint16_t* coarse = nullptr;
   spade::RunRec* runs = nullptr;
   int4* run_seg = nullptr;
-  int32_t* run_poly = nullptr;
+  uint64_t* run_mask = nullptr;
+  int32_t* rec_polys = nullptr;
   int32_t* sets = nullptr;
   int2* set_rng = nullptr;
   spade::CanvasDev* d_dev = nullptr;   // copy of d in device memory (out-of-line exact test)

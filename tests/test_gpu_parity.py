@@ -188,3 +188,36 @@ def test_results_independent_of_point_id_base_and_chunking(spade):
     assert torch.equal(full, parts)
     pt, pl = spade.join_pairs(cv, xy, point_id_base=10**12)
     assert int(pt.min()) >= 10**12 and int(pt.max()) < 10**12 + 50_000
+
+
+def _fan(n, R=1_000_000, overlap=False, spikes=False):
+    """n triangles around the origin (adjacent ones share an edge); overlap=True adds a second
+    copy of every triangle (shared edges across all polygons); spikes=True gives every triangle a
+    degenerate out-and-back spur (an edge traversed twice by the same ring)."""
+    th = np.linspace(0, 2 * np.pi, n + 1)
+    v = np.stack([np.round(R * np.cos(th)), np.round(R * np.sin(th))], 1).astype(np.int64)
+    v[-1] = v[0]
+    polys = []
+    for i in range(n):
+        ring = [(0, 0), tuple(v[i]), tuple(v[i + 1])]
+        if spikes:
+            m = (v[i] + v[i + 1]) // 2
+            ring = [(0, 0), tuple(v[i]), tuple(m), tuple(m * 2 - m // 3), tuple(m), tuple(v[i + 1])]
+        polys.append([np.array(ring)])
+    if overlap:
+        polys = polys + [list(p) for p in polys]
+    return pg.assemble(polys)
+
+
+@pytest.mark.parametrize("n,overlap,spikes", [(40, False, False), (40, True, False), (20, True, True),
+                                              (63, False, True), (100, False, False), (90, True, False)])
+@pytest.mark.parametrize("s", [9, 12])
+def test_many_polygons_one_pixel(spade, n, overlap, spikes, s):
+    """Boundary pixels with up to 180 polygons: edges shared by 2-4 polygons are stored once
+    with a polygon toggle mask (<= 64 polygons) or per polygon (> 64)."""
+    polys = _fan(n, overlap=overlap, spikes=spikes)
+    rng = np.random.default_rng(n + s)
+    near = rng.integers(-3000, 3000, (20000, 2))
+    far = rng.integers(-1_100_000, 1_100_000, (20000, 2))
+    xy = np.concatenate([near, far, lattice(-40, -40, 40, 40)]).astype(np.int32)
+    check_all(spade, polys, xy, s=s, max_dim=4096)
