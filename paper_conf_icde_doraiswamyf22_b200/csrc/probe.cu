@@ -22,7 +22,10 @@
 #include <cstdint>
 #include <algorithm>
 #include <cstdlib>
+#include <vector>
+#include <cstdio>
 #include <cub/block/block_scan.cuh>
+#include <cub/block/block_radix_sort.cuh>
 #include "spade_internal.cuh"
 
 namespace spade {
@@ -69,15 +72,48 @@ __device__ __forceinline__ uint32_t ld_fine(const int32_t* p, uint64_t pol) {
   return r;
 }
 
+__device__ __forceinline__ uint32_t nctaid_x() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%nctaid.x;" : "=r"(r));
+  return r;
+}
+
+struct U4 {
+  uint32_t c[4];
+  __device__ __forceinline__ uint32_t& operator[](int i) { return c[i]; }
+  __device__ __forceinline__ uint32_t operator[](int i) const { return c[i]; }
+};
+
 // Output side of a launch (what the sinks write).
+// SELECT/PAIRS output slots are handed out in chunks of `chunk` slots per warp (one global atomic
+// per chunk, no CTA barrier in the probe loop).  Every warp's last chunk is partly unused: its
+// hole is recorded and k_fixup/k_move fill the holes with the results stored past them, so the
+// output ends up dense.  Slots at or past the caller's capacity go to an overflow buffer of
+// `ovf_cap` >= (number of warps) x chunk slots, enough to hold all results whenever they fit.
 struct Out {
   unsigned long long* counts; // COUNT
-  unsigned long long* total;  // SELECT/PAIRS: number of results (may exceed capacity)
+  unsigned long long* total;  // SELECT/PAIRS: slots handed out (results + holes; may exceed capacity)
   int64_t* out_ids;           // SELECT ids / PAIRS point ids
   int32_t* out_poly;          // PAIRS polygon ids
   int64_t cap;
   int64_t id_base;            // point id of xy[0]
+  int64_t* ovf_ids;           // overflow slots [cap, cap + ovf_cap)
+  int32_t* ovf_poly;
+  int64_t ovf_cap;
+  longlong2* holes;           // [grid * kNW] (start, length) of each warp's unused chunk tail
+  uint32_t chunk;             // slots per warp chunk
 };
+
+template <int MODE>
+__device__ __forceinline__ void put_result(const Out& o, int64_t pos, int64_t id, int poly) {
+  if (pos < o.cap) {
+    o.out_ids[pos] = id;
+    if (MODE == kPairs) o.out_poly[pos] = poly;
+  } else if (pos - o.cap < o.ovf_cap) {
+    o.ovf_ids[pos - o.cap] = id;
+    if (MODE == kPairs) o.ovf_poly[pos - o.cap] = poly;
+  }
+}
 
 struct Params {
   CanvasDev cv;
@@ -182,41 +218,29 @@ __device__ __forceinline__ void count_hit(unsigned int* hist, unsigned long long
 // Emission from the rare in-kernel paths (deferral region full, unaligned head/tail): per-lane
 // atomics.
 template <int MODE>
-__device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, Out o,
+__device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, const Out& o,
                                              int x, int y, uint32_t rec, int64_t pid) {
   if (MODE == kCountSmem || MODE == kCountGlobal) {
     pip_eval(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, o.counts, p); });
   } else if (MODE == kSelect) {
     bool any = false;
     pip_eval(cvg, x, y, rec, [&](int) { any = true; });
-    if (any) {
-      unsigned long long q = atomicAdd(o.total, 1ull);
-      if ((int64_t)q < o.cap) o.out_ids[q] = pid;
-    }
+    if (any) put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, 0);
   } else {
-    pip_eval(cvg, x, y, rec, [&](int p) {
-      unsigned long long q = atomicAdd(o.total, 1ull);
-      if ((int64_t)q < o.cap) { o.out_ids[q] = pid; o.out_poly[q] = p; }
-    });
+    pip_eval(cvg, x, y, rec, [&](int p) { put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, p); });
   }
 }
 
 template <int MODE>
 __device__ __forceinline__ void rare_emit_owner(unsigned int* hist, const Out& o, int owner, int64_t pid) {
   if (MODE == kCountSmem || MODE == kCountGlobal) count_hit<MODE>(hist, o.counts, owner);
-  else {
-    unsigned long long q = atomicAdd(o.total, 1ull);
-    if ((int64_t)q < o.cap) {
-      o.out_ids[q] = pid;
-      if (MODE == kPairs) o.out_poly[q] = owner;
-    }
-  }
+  else put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, owner);
 }
 
 // One scalar point (unaligned head / tail): classify synchronously.
 template <int MODE>
 __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, unsigned int* hist,
-                                          Out o, int x, int y, int64_t pid) {
+                                          const Out& o, int x, int y, int64_t pid) {
   const CanvasDev cv = *cvg;
   const uint32_t ux = (uint32_t)x - (uint32_t)cv.minx, uy = (uint32_t)y - (uint32_t)cv.miny;
   if (ux > cv.extw || uy > cv.exth) return;
@@ -248,9 +272,7 @@ __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint
 //           always-empty sentinels: tile coordinates are clamped into them (no extent test)
 //   COUNT   hcopies x (P + 1) uint32 bins (bin P = "no polygon" trash bin), copy = lane & (hc-1)
 //   QUEUE   (COUNT, in-loop exact test) kNW x kQCap QEntry: boundary points per warp
-//   SELECT/PAIRS: 128 int warp sums + 32 int64 warp bases
 __host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
-constexpr size_t kScanBytes = 128 * sizeof(int) + 32 * sizeof(long long);
 
 template <int MODE, int COMPACT, int QUEUE>
 __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params prm) {
@@ -265,8 +287,6 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   const uint32_t P = (uint32_t)cv.num_polys;
   unsigned int* hist = (unsigned int*)rest;                       // COUNT
   unsigned int* myhist = hist + (lane & (prm.hcopies - 1)) * (P + 1);
-  int* s_scan = (int*)rest;                                       // SELECT/PAIRS
-  long long* s_base = (long long*)(rest + 128 * sizeof(int));
   __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
   __shared__ int s_qn[kNW];                     // QUEUE: per-warp queue fill
   QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : 0)) + warp * kQCap;
@@ -309,35 +329,39 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     else { v.a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v.b = v.a; }
   };
   const uint32_t stride = gridDim.x * chunk;
-  Vec4 nxt;
-  if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
-  for (uint32_t base = blockIdx.x * chunk; base < nvec; base += stride) {
-    const Vec4 v = nxt;
-    if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight meanwhile
+  // SELECT/PAIRS: this warp's output chunk [wbase, wbase + K), wused slots used (lane-uniform)
+  const uint32_t K = prm.o.chunk;
+  long long wbase = 0;
+  uint32_t wused = K;
+  // phases A + B of one batch: c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
+  auto classify = [&](const Vec4 v) {
+    U4 f;
     // phase A: coarse (shared memory) lookup, branch-free.  Offsets from the extent origin are
     // unsigned; points left of / below the origin wrap to huge values and, like points right of /
     // above the canvas, clamp into the always-empty sentinel column / row (exact because
     // 2^(s+b) <= 2^30, see canvas_build.cu).  Padding points (INT32_MIN) land there too.
-    uint32_t c[NPT];
 #pragma unroll
     for (int q = 0; q < NPT; ++q) {
       const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
       const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
       const uint32_t ux = (uint32_t)x - minx, uy = (uint32_t)y - miny;
-      c[q] = tiles[min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc)];
+      f[q] = tiles[min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc)];
     }
     // phase B: fine pixels of mixed tiles; all gathers of the batch in flight together
 #pragma unroll
     for (int q = 0; q < NPT; ++q) {
-      if (c[q] >= mixmin) {
+      if (f[q] >= mixmin) {
         const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
         const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
         const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
-        const uint32_t fidx = COMPACT ? ((((c[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
-        c[q] = classify_fine((int32_t)ld_fine(finep + fidx, pol));
+        const uint32_t fidx = COMPACT ? ((((f[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
+        f[q] = classify_fine((int32_t)ld_fine(finep + fidx, pol));
       }
     }
-    // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
+    return f;
+  };
+  // phase C of one batch: the sinks.  getxy(q): coordinates of point q of this thread.
+  auto process = [&](uint32_t base, const U4 c, auto getxy) {
     const uint32_t orc = c[0] | c[1] | c[2] | c[3];
     if (QUEUE) {
       // phase C1 (COUNT): boundary points -> warp queue (one smem atomic per lane that has any),
@@ -352,9 +376,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #pragma unroll
           for (int q = 0; q < NPT; ++q)
             if ((bnd >> q) & 1u) {
-              const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
-              const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
-              wq[pos++] = QEntry{x, y};
+              const int2 p = getxy(q);
+              wq[pos++] = QEntry{p.x, p.y};
             }
         }
         __syncwarp();
@@ -381,14 +404,13 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #pragma unroll
       for (int q = 0; q < NPT; ++q) {
         if ((bnd >> q) & 1u) {
-          const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
-          const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+          const int2 p = getxy(q);
           const uint32_t pidx = (uint32_t)prm.head + 4 * (base + tid) + q;
           if (fits) {
-            dreg[d] = DEntry{x, y, ~c[q], pidx};
+            dreg[d] = DEntry{p.x, p.y, ~c[q], pidx};
           } else {
             if (d < prm.defer_cap) dreg[d] = DEntry{0, 0, kHole, 0u};
-            rare_emit_point<MODE>(prm.cvg, myhist, prm.o, x, y, ~c[q], prm.o.id_base + pidx);
+            rare_emit_point<MODE>(prm.cvg, myhist, prm.o, p.x, p.y, ~c[q], prm.o.id_base + pidx);
           }
           ++d;
         }
@@ -404,47 +426,129 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
       for (int q = 0; q < NPT; ++q)
         if (c[q] != 0u && !(c[q] >> 31)) atomicAdd(prm.o.counts + (c[q] - 1u), 1ull);
     } else {
-      // CTA-aggregated reservation of output slots for this batch (Map with a scan).
+      // Output slots for this batch (Map with a scan) from the warp's current chunk: a warp
+      // scan (ballots), a new chunk (one global atomic, lane 0) when the batch does not fit.
       // Within the warp the results are laid out slot-major (all lanes' slot 0 hits, then slot 1,
-      // ...), so every store instruction writes one contiguous run: coalesced 8-B / 4-B stores.
+      // ...), so every store instruction writes one or two contiguous runs.
       unsigned hm[NPT];
-      int wtot = 0;
+      uint32_t wtot = 0;
 #pragma unroll
       for (int q = 0; q < NPT; ++q) {
         hm[q] = __ballot_sync(0xffffffffu, c[q] != 0u && !(c[q] >> 31));
         wtot += __popc(hm[q]);
       }
-      if (lane == 0) s_scan[warp] = wtot;
-      __syncthreads();
-      if (warp == 0) {
-        int wsum = lane < NW ? s_scan[lane] : 0, wincl = wsum;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          int t = __shfl_up_sync(0xffffffffu, wincl, o);
-          if (lane >= o) wincl += t;
+      if (wtot) {
+        const uint32_t room = K - wused;
+        const long long b0 = wbase + wused;
+        long long b1 = 0;
+        if (wtot > room) {
+          if (lane == 0) b1 = (long long)atomicAdd(prm.o.total, (unsigned long long)K);
+          b1 = __shfl_sync(0xffffffffu, b1, 0);
         }
-        unsigned long long gb = 0;
-        if (lane == 31 && wincl > 0) gb = atomicAdd(prm.o.total, (unsigned long long)wincl);
-        gb = __shfl_sync(0xffffffffu, gb, 31);
-        if (lane < NW) s_base[lane] = (long long)gb + (wincl - wsum);
+        const unsigned lt = (1u << lane) - 1u;
+        uint32_t k0 = 0;
+#pragma unroll
+        for (int q = 0; q < NPT; ++q) {
+          if ((hm[q] >> lane) & 1u) {
+            const uint32_t k = k0 + __popc(hm[q] & lt);
+            const int64_t pos = k < room ? b0 + k : b1 + (k - room);
+            put_result<MODE>(prm.o, pos, prm.o.id_base + prm.head + 4 * (int64_t)(base + tid) + q, (int)c[q] - 1);
+          }
+          k0 += __popc(hm[q]);
+        }
+        if (wtot > room) { wbase = b1; wused = wtot - room; }
+        else wused += wtot;
       }
-      __syncthreads();
-      int64_t wpos = s_base[warp];
-      const unsigned lt = (1u << lane) - 1u;
+    }
+  };
+  const uint32_t first = blockIdx.x * chunk;
+  if (QUEUE) {
+    // COUNT with in-loop exact tests (the C3 configuration): written out without the lambdas,
+    // which cost this register-bound variant a spill
+    Vec4 nxt;
+    if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
+    // (the stride is re-read from the special register each batch: kept live, it spilled)
+    for (uint32_t base = blockIdx.x * chunk; base < nvec; base += nctaid_x() * chunk) {
+      const Vec4 v = nxt;
+      const uint32_t stride = nctaid_x() * chunk;
+      if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight meanwhile
+      // phase A: coarse (shared memory) lookup, branch-free.  Offsets from the extent origin are
+      // unsigned; points left of / below the origin wrap to huge values and, like points right of /
+      // above the canvas, clamp into the always-empty sentinel column / row (exact because
+      // 2^(s+b) <= 2^30, see canvas_build.cu).  Padding points (INT32_MIN) land there too.
+      uint32_t c[NPT];
 #pragma unroll
       for (int q = 0; q < NPT; ++q) {
-        if ((hm[q] >> lane) & 1u) {
-          const int64_t pos = wpos + __popc(hm[q] & lt);
-          if (pos < prm.o.cap) {
-            prm.o.out_ids[pos] = prm.o.id_base + prm.head + 4 * (int64_t)(base + tid) + q;
-            if (MODE == kPairs) prm.o.out_poly[pos] = (int)c[q] - 1;
-          }
-        }
-        wpos += __popc(hm[q]);
+        const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+        const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+        const uint32_t ux = (uint32_t)x - minx, uy = (uint32_t)y - miny;
+        c[q] = tiles[min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc)];
       }
-      __syncthreads();   // s_scan / s_base reuse next batch
+      // phase B: fine pixels of mixed tiles; all gathers of the batch in flight together
+#pragma unroll
+      for (int q = 0; q < NPT; ++q) {
+        if (c[q] >= mixmin) {
+          const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+          const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+          const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
+          const uint32_t fidx = COMPACT ? ((((c[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
+          c[q] = classify_fine((int32_t)ld_fine(finep + fidx, pol));
+        }
+      }
+      // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
+      const uint32_t orc = c[0] | c[1] | c[2] | c[3];
+      {
+        // phase C1 (COUNT): boundary points -> warp queue (one smem atomic per lane that has any),
+        // drained 32 at a time from the top, in the loop: the ALU-heavy exact tests overlap the
+        // memory-bound stream of the other warps
+        if (__any_sync(0xffffffffu, (int)orc < 0)) {
+          uint32_t bnd = 0;
+#pragma unroll
+          for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
+          if (bnd) {
+            int pos = atomicAdd(&s_qn[warp], __popc(bnd));
+#pragma unroll
+            for (int q = 0; q < NPT; ++q)
+              if ((bnd >> q) & 1u) {
+                const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+                const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+                wq[pos++] = QEntry{x, y};
+              }
+          }
+          __syncwarp();
+          int qn = s_qn[warp];
+          if (qn >= 32) {
+            do {
+              drain<MODE>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+              qn -= 32;
+            } while (qn >= 32);
+            __syncwarp();
+            if (lane == 0) s_qn[warp] = qn;
+          }
+          __syncwarp();
+        }
+      }
+      // phase C2: direct hits (branch-free: non-hits and boundary points go to the trash bin P)
+#pragma unroll
+      for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P)], 1u);
+    }
+  } else {
+    // only the next batch of points is prefetched; there are no CTA barriers in the loop, the 32
+    // warps hide each other's gather latency
+    Vec4 nxt;
+    if (first < nvec) load_batch(nxt, first);
+    for (uint32_t base = first; base < nvec; base += nctaid_x() * chunk) {
+      const Vec4 v = nxt;
+      const uint32_t stride = nctaid_x() * chunk;
+      if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight meanwhile
+      process(base, classify(v), [v](int q) {
+        return make_int2(q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z,
+                         q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w);
+      });
     }
   }
+  if ((MODE == kSelect || MODE == kPairs) && lane == 0)
+    prm.o.holes[(size_t)blockIdx.x * kNW + warp] = make_longlong2(wbase + wused, (long long)(K - wused));
   if (QUEUE) {
     __syncwarp();
     if (s_qn[warp] > 0) drain<MODE>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.o.counts);
@@ -511,14 +615,11 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
       int64_t pos = (int64_t)s_gb + excl;
       if (nres) {
         if (MODE == kSelect) {
-          if (pos < o.cap) o.out_ids[pos] = pid;
+          put_result<MODE>(o, pos, pid, 0);
         } else if (nres == 1) {                    // the common case: no second evaluation
-          if (pos < o.cap) { o.out_ids[pos] = pid; o.out_poly[pos] = first; }
+          put_result<MODE>(o, pos, pid, first);
         } else {
-          pip_eval(cvg, e.x, e.y, e.rec, [&](int q) {
-            if (pos < o.cap) { o.out_ids[pos] = pid; o.out_poly[pos] = q; }
-            ++pos;
-          });
+          pip_eval(cvg, e.x, e.y, e.rec, [&](int q) { put_result<MODE>(o, pos++, pid, q); });
         }
       }
       __syncthreads();
@@ -528,6 +629,121 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
     __syncthreads();
     for (int q = threadIdx.x; q < P; q += 256)
       if (dh[q]) atomicAdd(o.counts + q, (unsigned long long)dh[q]);
+  }
+}
+
+// Output compaction after a SELECT/PAIRS launch (probe + deferred kernel).  The slots handed out
+// are [T0, T); the holes (each warp's unused chunk tail) total H, so the results are M = T - H
+// and must end up in [T0, M).  k_fixup (one block) sorts the holes, sets *total = M and lists
+// (a) the hole slots below M (destinations, in order) and (b) the runs of result slots at or past
+// M (sources, in order); k_move copies the k-th source into the k-th destination.
+constexpr int kFixT = 1024, kFixItems = 5;
+constexpr int kMaxHoles = kFixT * kFixItems;    // warps per launch (grid <= 160 CTAs)
+struct FixMeta {
+  long long M, nmove;
+};
+
+template <int MODE>
+__global__ void __launch_bounds__(kFixT) k_fixup(const longlong2* __restrict__ holes, int nh, unsigned long long* total,
+                                                 int64_t cap, long long* __restrict__ dst_start,
+                                                 long long* __restrict__ dst_pre, long long* __restrict__ src_start,
+                                                 long long* __restrict__ src_pre, FixMeta* meta) {
+  using Sort = cub::BlockRadixSort<unsigned long long, kFixT, kFixItems, long long>;
+  using Scan = cub::BlockScan<long long, kFixT>;
+  __shared__ union {
+    typename Sort::TempStorage sort;
+    typename Scan::TempStorage scan;
+    long long next[kMaxHoles + 1];
+  } sm;
+  __shared__ unsigned long long s_H;
+  unsigned long long key[kFixItems];
+  long long len[kFixItems];
+  long long hl = 0;
+#pragma unroll
+  for (int i = 0; i < kFixItems; ++i) {
+    const int h = threadIdx.x * kFixItems + i;
+    const longlong2 v = h < nh ? holes[h] : make_longlong2(0, 0);
+    len[i] = v.y;
+    key[i] = v.y > 0 ? (unsigned long long)v.x : ~0ull;      // empty holes sort last
+    hl += v.y;
+  }
+  if (threadIdx.x == 0) s_H = 0;
+  __syncthreads();
+  atomicAdd(&s_H, (unsigned long long)hl);
+  Sort(sm.sort).Sort(key, len);                   // blocked arrangement, ascending starts
+  __syncthreads();
+  const long long T = (long long)*total, M = T - (long long)s_H;
+  // Hole i = [a, e).  Destinations: its part below M.  Sources: the run of result slots after
+  // its part at or past M, [max(e, M), max(a', M)) with a' the next hole's start (T after the
+  // last), plus the leading run [M, max(a_0, M)).
+#pragma unroll
+  for (int i = 0; i < kFixItems; ++i)
+    sm.next[threadIdx.x * kFixItems + i] = key[i] != ~0ull ? max((long long)key[i], M) : T;
+  if (threadIdx.x == 0) sm.next[kMaxHoles] = T;
+  __syncthreads();
+  long long dl[kFixItems], gs[kFixItems], gl[kFixItems];
+  long long dsum = 0, gsum = 0;
+#pragma unroll
+  for (int i = 0; i < kFixItems; ++i) {
+    const bool valid = key[i] != ~0ull;
+    const long long a = (long long)key[i], e = a + len[i];
+    dl[i] = valid && a < M ? min(e, M) - a : 0;
+    gs[i] = valid ? max(e, M) : T;
+    gl[i] = valid ? max(sm.next[threadIdx.x * kFixItems + i + 1] - gs[i], 0ll) : 0;
+    dsum += dl[i];
+    gsum += gl[i];
+  }
+  const long long lead = sm.next[0] - M;
+  __syncthreads();                                // sm.next is reused by the scans
+  long long dex, gex;
+  Scan(sm.scan).ExclusiveSum(dsum, dex);
+  __syncthreads();
+  Scan(sm.scan).ExclusiveSum(gsum, gex);
+#pragma unroll
+  for (int i = 0; i < kFixItems; ++i) {
+    const int h = threadIdx.x * kFixItems + i;
+    dst_start[h] = key[i] != ~0ull ? (long long)key[i] : T;
+    dst_pre[h] = dex;                             // exclusive prefix of destination slots
+    dex += dl[i];
+    src_start[h + 1] = gs[i];
+    src_pre[h + 1] = lead + gex;                  // exclusive prefix of source slots
+    gex += gl[i];
+  }
+  if (threadIdx.x == 0) {
+    src_start[0] = M;
+    src_pre[0] = 0;
+  }
+  if (threadIdx.x == kFixT - 1) {
+    FixMeta m;
+    m.M = M;
+    m.nmove = M <= cap ? dex : 0;                 // results lost to capacity: nothing to repair
+    *meta = m;
+    *total = (unsigned long long)M;
+  }
+}
+
+// k-th destination slot / source slot: upper-bound searches in the prefix arrays
+__device__ __forceinline__ int find_run(const long long* __restrict__ pre, int n, long long k) {
+  int lo = 0, hi = n;                            // last i with pre[i] <= k
+  while (hi - lo > 1) { const int mid = (lo + hi) >> 1; if (pre[mid] <= k) lo = mid; else hi = mid; }
+  return lo;
+}
+
+template <int MODE>
+__global__ void k_move(Out o, const long long* __restrict__ dst_start, const long long* __restrict__ dst_pre,
+                       const long long* __restrict__ src_start, const long long* __restrict__ src_pre,
+                       const FixMeta* __restrict__ meta) {
+  const FixMeta m = *meta;
+  for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < m.nmove;
+       k += (long long)gridDim.x * blockDim.x) {
+    const int di = find_run(dst_pre, kMaxHoles, k);
+    const long long d = dst_start[di] + (k - dst_pre[di]);
+    const int si = find_run(src_pre, kMaxHoles + 1, k);
+    const long long q = src_start[si] + (k - src_pre[si]);
+    const bool ov = q >= o.cap;
+    const int64_t id = ov ? o.ovf_ids[q - o.cap] : o.out_ids[q];
+    o.out_ids[d] = id;                           // d < M <= cap
+    if (MODE == kPairs) o.out_poly[d] = ov ? o.ovf_poly[q - o.cap] : o.out_poly[q];
   }
 }
 
@@ -567,22 +783,48 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.nvec = (m - p.head) / 4;
     p.o.id_base = base.o.id_base + off;
     const int64_t chunks = (p.nvec + kT - 1) / kT;
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(sms, chunks));
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(std::min(sms, kMaxHoles / kNW), chunks));
     // deferral regions sized from the canvas's boundary-pixel fraction fb (points are not uniform,
     // so 2 fb + 4%, at most all points); overflowing points are tested in place (slow, rare)
     const double fb = (double)c->num_runs / ((double)c->d.W * (double)c->d.H);
     const double frac = std::min(1.0, 2.0 * fb + 0.04);
     const int64_t per = QUEUE ? 0 : std::min<int64_t>(std::max<int64_t>((int64_t)(frac * (double)m / grid) + 64, 1024),
                                                        (int64_t)1 << 26);
-    DEntry* dbuf = nullptr;
-    unsigned int* dfill = nullptr;
-    if (!QUEUE) {
-      e = cudaMallocAsync((void**)&dbuf, sizeof(DEntry) * per * grid, st);
-      if (e == cudaSuccess) e = cudaMallocAsync((void**)&dfill, sizeof(unsigned int) * grid, st);
-      if (e != cudaSuccess) {
-        if (dbuf) cudaFreeAsync(dbuf, st);
-        return check_cuda(e, "probe scratch");
-      }
+    // SELECT/PAIRS: warp output chunks of K slots (about 1/16 of a warp's points, 256..2048),
+    // overflow slots for every warp's possible hole, hole list and compaction tables
+    constexpr bool kOut = MODE == kSelect || MODE == kPairs;
+    uint32_t K = 0;
+    if (kOut) {
+      const int64_t per_warp = m / ((int64_t)grid * kNW) / 16;
+      K = 256;
+      while (K < 2048 && (int64_t)K * 2 <= per_warp) K *= 2;
+    }
+    const int64_t ovf = kOut ? (int64_t)grid * kNW * K : 0;
+    size_t sz[9] = {sizeof(DEntry) * (QUEUE ? 0 : per * grid), QUEUE ? 0 : sizeof(unsigned int) * grid,
+                    sizeof(int64_t) * ovf, MODE == kPairs ? sizeof(int32_t) * ovf : 0,
+                    kOut ? sizeof(longlong2) * kMaxHoles : 0, kOut ? 8 * (size_t)kMaxHoles : 0,
+                    kOut ? 8 * (size_t)kMaxHoles : 0, kOut ? 8 * (size_t)(kMaxHoles + 1) : 0,
+                    kOut ? 8 * (size_t)(kMaxHoles + 1) + sizeof(FixMeta) : 0};
+    size_t total_sz = 0, offs[9];
+    for (int i = 0; i < 9; ++i) { offs[i] = total_sz; total_sz += (sz[i] + 255) & ~(size_t)255; }
+    unsigned char* scratch = nullptr;
+    if (total_sz > 0) {
+      e = cudaMallocAsync((void**)&scratch, total_sz, st);
+      if (e != cudaSuccess) return check_cuda(e, "probe scratch");
+    }
+    DEntry* dbuf = QUEUE ? nullptr : (DEntry*)(scratch + offs[0]);
+    unsigned int* dfill = QUEUE ? nullptr : (unsigned int*)(scratch + offs[1]);
+    long long* fix_ds = (long long*)(scratch + offs[5]);
+    long long* fix_dp = (long long*)(scratch + offs[6]);
+    long long* fix_ss = (long long*)(scratch + offs[7]);
+    long long* fix_sp = (long long*)(scratch + offs[8]);
+    FixMeta* fix_meta = (FixMeta*)(scratch + offs[8] + 8 * (size_t)(kMaxHoles + 1));
+    if (kOut) {
+      p.o.chunk = K;
+      p.o.ovf_ids = (int64_t*)(scratch + offs[2]);
+      p.o.ovf_poly = MODE == kPairs ? (int32_t*)(scratch + offs[3]) : nullptr;
+      p.o.ovf_cap = ovf;
+      p.o.holes = (longlong2*)(scratch + offs[4]);
     }
     p.defer = dbuf;
     p.defer_cap = (uint32_t)per;
@@ -598,9 +840,25 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       k_deferred<MODE><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh);
       count_launch();
       e = cudaGetLastError();
+      static const bool dbg = getenv("SPADE_DEBUG_DEFER") != nullptr;
+      if (dbg && e == cudaSuccess) {           // diagnostics only: synchronises
+        std::vector<unsigned int> f(grid);
+        cudaMemcpyAsync(f.data(), dfill, sizeof(unsigned int) * grid, cudaMemcpyDeviceToHost, st);
+        cudaStreamSynchronize(st);
+        long long tot = 0; unsigned int mx = 0;
+        for (unsigned int x : f) { tot += x; mx = std::max(mx, x); }
+        fprintf(stderr, "[spade] deferred %lld of %lld points (%.2f%%), max region %u of cap %lld, runs %lld, run edges %lld\n",
+                tot, (long long)m, 100.0 * tot / m, mx, (long long)per, (long long)c->num_runs, (long long)c->num_run_edges);
+      }
     }
-    if (dbuf) cudaFreeAsync(dbuf, st);
-    if (dfill) cudaFreeAsync(dfill, st);
+    if (kOut && e == cudaSuccess) {
+      k_fixup<MODE><<<1, kFixT, 0, st>>>(p.o.holes, grid * kNW, p.o.total, p.o.cap, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
+      count_launch();
+      k_move<MODE><<<sms * 4, 256, 0, st>>>(p.o, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
+      count_launch();
+      e = cudaGetLastError();
+    }
+    if (scratch) cudaFreeAsync(scratch, st);
     if (e != cudaSuccess) return check_cuda(e, "probe launch");
   }
   return SPADE_OK;
@@ -651,7 +909,7 @@ int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t b
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = out; p.o.cap = cap; p.o.total = d_total;
-  return launch_layout<kSelect>(c, (const int2*)xy, n, p, kScanBytes, st);
+  return launch_layout<kSelect>(c, (const int2*)xy, n, p, 0, st);
 }
 
 int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* opt, int32_t* opl,
@@ -659,7 +917,7 @@ int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t ba
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = opt; p.o.out_poly = opl; p.o.cap = cap; p.o.total = d_total;
-  return launch_layout<kPairs>(c, (const int2*)xy, n, p, kScanBytes, st);
+  return launch_layout<kPairs>(c, (const int2*)xy, n, p, 0, st);
 }
 
 }  // namespace spade
