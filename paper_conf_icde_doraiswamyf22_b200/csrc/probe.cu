@@ -267,11 +267,53 @@ __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint
   }
 }
 
+// SELECT/PAIRS, in-loop variant: the exact test of one queued boundary point (lane < cnt), by
+// its index into the launch's points: (number of results, first polygon).  Out of line.
+template <int MODE>
+__device__ __noinline__ uint2 drain_eval(const CanvasDev* __restrict__ cvg, const uint16_t* tiles,
+                                         const int2* __restrict__ xy, uint32_t pidx) {
+  const CanvasDev& cv = *cvg;
+  const int2 p = __ldg(xy + pidx);
+  const uint32_t fx = ((uint32_t)p.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)p.y - (uint32_t)cv.miny) >> cv.s;
+  const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
+  const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
+  uint32_t n = 0, first = 0;
+  if (MODE == kSelect) {
+    pip_eval(cvg, p.x, p.y, ~c, [&](int) { n = 1; });
+  } else {
+    pip_eval(cvg, p.x, p.y, ~c, [&](int q) { if (n++ == 0) first = (uint32_t)q; });
+  }
+  return make_uint2(n, first);
+}
+
+// Output slots of one warp-wide emission: result k goes to k < room ? b0 + k : b1 + (k - room).
+struct Slots {
+  long long b0, b1;
+  uint32_t room;
+  __device__ __forceinline__ long long at(uint32_t k) const { return k < room ? b0 + k : b1 + (long long)(k - room); }
+};
+
+// A queued point with more than one result (overlapping polygons): evaluated again, results
+// written to slots k, k+1, ...  Out of line (rare).
+__device__ __noinline__ void emit_multi(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const int2* __restrict__ xy,
+                                        uint32_t pidx, const Out& o, Slots sl, uint32_t k) {
+  const CanvasDev& cv = *cvg;
+  const int2 p = __ldg(xy + pidx);
+  const uint32_t fx = ((uint32_t)p.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)p.y - (uint32_t)cv.miny) >> cv.s;
+  const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
+  const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
+  pip_eval(cvg, p.x, p.y, ~c, [&](int q) { put_result<kPairs>(o, sl.at(k++), o.id_base + pidx, q); });
+}
+
 // Per-CTA shared-memory layout (bytes, in order):
 //   tiles   (Wc+1) x (Hc+1) uint16 (pitch Wc+1), rounded up to 16 B; the last column and row are
 //           always-empty sentinels: tile coordinates are clamped into them (no extent test)
 //   COUNT   hcopies x (P + 1) uint32 bins (bin P = "no polygon" trash bin), copy = lane & (hc-1)
-//   QUEUE   (COUNT, in-loop exact test) kNW x kQCap QEntry: boundary points per warp
+//   QUEUE   (in-loop exact test) kNW x kQCap QEntry (COUNT: coordinates) or uint32 (SELECT/
+//           PAIRS: point index) per warp: boundary points
+__host__ __device__ __forceinline__ size_t queue_bytes(int mode) {
+  return (size_t)kNW * kQCap * (mode == kSelect || mode == kPairs ? sizeof(uint32_t) : sizeof(QEntry));
+}
 __host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
 
 template <int MODE, int COMPACT, int QUEUE>
@@ -290,6 +332,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
   __shared__ int s_qn[kNW];                     // QUEUE: per-warp queue fill
   QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : 0)) + warp * kQCap;
+  uint32_t* wqi = (uint32_t*)rest + warp * kQCap;                 // SELECT/PAIRS queue
   if (QUEUE && lane == 0) s_qn[warp] = 0;
 
   for (uint32_t i = tid; i < tbytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
@@ -328,11 +371,49 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     else if (idx < nvec) v = ld_stream(vp + idx);
     else { v.a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v.b = v.a; }
   };
-  const uint32_t stride = gridDim.x * chunk;
   // SELECT/PAIRS: this warp's output chunk [wbase, wbase + K), wused slots used (lane-uniform)
   const uint32_t K = prm.o.chunk;
   long long wbase = 0;
-  uint32_t wused = K;
+  uint32_t wcap = 0, wused = 0;
+  // Slots for `wtot` results of this warp (lane-uniform).  A new chunk covers at most what the
+  // warp can still produce from its direct hits (<= 128 per remaining batch), so the last chunk's
+  // hole stays small; results beyond that (multi-polygon points) get a chunk of their own size.
+  auto reserve = [&](uint32_t wtot, uint32_t later_batches) {
+    Slots sl;
+    sl.room = wcap - wused;
+    sl.b0 = wbase + wused;
+    sl.b1 = 0;
+    if (wtot > sl.room) {
+      const uint32_t need = wtot - sl.room;
+      const uint32_t want = max(need, min(K, need + 128u * min(later_batches, 64u)));
+      if (lane == 0) sl.b1 = (long long)atomicAdd(prm.o.total, (unsigned long long)want);
+      sl.b1 = __shfl_sync(0xffffffffu, sl.b1, 0);
+      wbase = sl.b1;
+      wcap = want;
+      wused = need;
+    } else {
+      wused += wtot;
+    }
+    return sl;
+  };
+  // SELECT/PAIRS drain of 32 queued points (one per lane, lane < cnt)
+  auto drain_out = [&](const uint32_t* q, int cnt, uint32_t later_batches) {
+    uint2 r = make_uint2(0u, 0u);
+    const uint32_t pidx = lane < cnt ? q[lane] : 0u;
+    if (lane < cnt) r = drain_eval<MODE>(prm.cvg, tiles, prm.xy, pidx);
+    uint32_t incl = r.x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
+    }
+    const uint32_t wtot = __shfl_sync(0xffffffffu, incl, 31);
+    if (wtot == 0) return;
+    const Slots sl = reserve(wtot, later_batches);
+    const uint32_t k = incl - r.x;
+    if (r.x == 1) put_result<MODE>(prm.o, sl.at(k), prm.o.id_base + pidx, (int)r.y);
+    else if (MODE == kPairs && r.x > 1) emit_multi(prm.cvg, tiles, prm.xy, pidx, prm.o, sl, k);
+  };
   // phases A + B of one batch: c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
   auto classify = [&](const Vec4 v) {
     U4 f;
@@ -376,15 +457,20 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #pragma unroll
           for (int q = 0; q < NPT; ++q)
             if ((bnd >> q) & 1u) {
-              const int2 p = getxy(q);
-              wq[pos++] = QEntry{p.x, p.y};
+              if (MODE == kSelect || MODE == kPairs) {
+                wqi[pos++] = (uint32_t)prm.head + 4 * (base + tid) + q;
+              } else {
+                const int2 p = getxy(q);
+                wq[pos++] = QEntry{p.x, p.y};
+              }
             }
         }
         __syncwarp();
         int qn = s_qn[warp];
         if (qn >= 32) {
           do {
-            drain<MODE>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+            if (MODE == kSelect || MODE == kPairs) drain_out(wqi + qn - 32, 32, (nvec - 1 - base) / (nctaid_x() * chunk));
+            else drain<MODE>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
             qn -= 32;
           } while (qn >= 32);
           __syncwarp();
@@ -438,31 +524,21 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         wtot += __popc(hm[q]);
       }
       if (wtot) {
-        const uint32_t room = K - wused;
-        const long long b0 = wbase + wused;
-        long long b1 = 0;
-        if (wtot > room) {
-          if (lane == 0) b1 = (long long)atomicAdd(prm.o.total, (unsigned long long)K);
-          b1 = __shfl_sync(0xffffffffu, b1, 0);
-        }
+        const Slots sl = reserve(wtot, (nvec - 1 - base) / (nctaid_x() * chunk));
         const unsigned lt = (1u << lane) - 1u;
         uint32_t k0 = 0;
 #pragma unroll
         for (int q = 0; q < NPT; ++q) {
-          if ((hm[q] >> lane) & 1u) {
-            const uint32_t k = k0 + __popc(hm[q] & lt);
-            const int64_t pos = k < room ? b0 + k : b1 + (k - room);
-            put_result<MODE>(prm.o, pos, prm.o.id_base + prm.head + 4 * (int64_t)(base + tid) + q, (int)c[q] - 1);
-          }
+          if ((hm[q] >> lane) & 1u)
+            put_result<MODE>(prm.o, sl.at(k0 + __popc(hm[q] & lt)),
+                             prm.o.id_base + prm.head + 4 * (int64_t)(base + tid) + q, (int)c[q] - 1);
           k0 += __popc(hm[q]);
         }
-        if (wtot > room) { wbase = b1; wused = wtot - room; }
-        else wused += wtot;
       }
     }
   };
   const uint32_t first = blockIdx.x * chunk;
-  if (QUEUE) {
+  if (QUEUE && MODE == kCountSmem) {
     // COUNT with in-loop exact tests (the C3 configuration): written out without the lambdas,
     // which cost this register-bound variant a spill
     Vec4 nxt;
@@ -547,9 +623,14 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
       });
     }
   }
-  if ((MODE == kSelect || MODE == kPairs) && lane == 0)
-    prm.o.holes[(size_t)blockIdx.x * kNW + warp] = make_longlong2(wbase + wused, (long long)(K - wused));
-  if (QUEUE) {
+  if (MODE == kSelect || MODE == kPairs) {
+    if (QUEUE) {
+      __syncwarp();
+      if (s_qn[warp] > 0) drain_out(wqi, s_qn[warp], 0u);
+    }
+    if (lane == 0) prm.o.holes[(size_t)blockIdx.x * kNW + warp] = make_longlong2(wbase + wused, (long long)(wcap - wused));
+  }
+  if (QUEUE && (MODE == kCountSmem || MODE == kCountGlobal)) {
     __syncwarp();
     if (s_qn[warp] > 0) drain<MODE>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.o.counts);
   }
@@ -765,7 +846,7 @@ void keep_pool_memory() {
 
 template <int MODE, int COMPACT, int QUEUE>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
-  const size_t smem = tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? kNW * kQCap * sizeof(QEntry) : 0);
+  const size_t smem = tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? queue_bytes(MODE) : 0);
   auto kern = k_probe<MODE, COMPACT, QUEUE>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
@@ -877,6 +958,13 @@ Params base_params(const spade_canvas* c) {
   return p;
 }
 
+// SELECT/PAIRS: boundary points tested in the loop (warp queues) when the queues fit beside the
+// tiles; SPADE_DEFER=1 forces the deferral kernel (A/B switch)
+bool use_queue(const spade_canvas* c, int mode) {
+  static const int force_defer = [] { const char* e = getenv("SPADE_DEFER"); return e ? atoi(e) : 0; }();
+  return !force_defer && tiles_bytes_for(c->d.Wc, c->d.Hc) + queue_bytes(mode) <= kSmemSoft;
+}
+
 }  // namespace
 
 int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts, cudaStream_t st) {
@@ -887,7 +975,7 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   // boundary points tested in the loop (warp queues) when those fit too, else deferred
   const size_t tiles = tiles_bytes_for(c->d.Wc, c->d.Hc);
   const size_t one = (size_t)(c->d.num_polys + 1) * 4;
-  const size_t queue = (size_t)kNW * kQCap * sizeof(QEntry);
+  const size_t queue = queue_bytes(kCountSmem);
   static const int force_defer = [] { const char* e = getenv("SPADE_DEFER"); return e ? atoi(e) : 0; }();
   for (uint32_t hc = 8; hc >= 1; hc >>= 1) {
     if (!force_defer && tiles + hc * one + queue <= kSmemSoft) {
@@ -909,6 +997,7 @@ int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t b
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = out; p.o.cap = cap; p.o.total = d_total;
+  if (use_queue(c, kSelect)) return launch_layout<kSelect, 1>(c, (const int2*)xy, n, p, 0, st);
   return launch_layout<kSelect>(c, (const int2*)xy, n, p, 0, st);
 }
 
@@ -917,6 +1006,7 @@ int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t ba
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = opt; p.o.out_poly = opl; p.o.cap = cap; p.o.total = d_total;
+  if (use_queue(c, kPairs)) return launch_layout<kPairs, 1>(c, (const int2*)xy, n, p, 0, st);
   return launch_layout<kPairs>(c, (const int2*)xy, n, p, 0, st);
 }
 

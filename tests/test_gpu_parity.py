@@ -221,3 +221,48 @@ def test_many_polygons_one_pixel(spade, n, overlap, spikes, s):
     far = rng.integers(-1_100_000, 1_100_000, (20000, 2))
     xy = np.concatenate([near, far, lattice(-40, -40, 40, 40)]).astype(np.int32)
     check_all(spade, polys, xy, s=s, max_dim=4096)
+
+
+@pytest.mark.parametrize("op", ["pairs", "select"])
+def test_exact_capacity_and_compaction(spade, op):
+    """3M points on C1's overlapping polygons: the per-warp output chunks leave holes that are
+    compacted away; with capacity exactly M the tail slots go through the overflow buffer; with
+    M - 1 the call reports M; slots past the capacity are never written."""
+    import ctypes
+    import torch
+    w = configs.c1()
+    xy_h = gen.points_host(gen.uniform_params(-20, -20, 1064, 1064), 77, 0, 3_000_000)
+    xy = torch.as_tensor(xy_h).cuda()
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    lib = spade.load()
+    if op == "pairs":
+        opt, opl = oracle.join_pairs(xy_h, w.polys, point_id_base=9)
+        M = len(opt)
+    else:
+        oids = oracle.select(xy_h, w.polys, point_id_base=9)
+        M = len(oids)
+    pad = 4096
+    pt = torch.full((M + pad,), -7, dtype=torch.int64, device="cuda")
+    pl = torch.full((M + pad,), -7, dtype=torch.int32, device="cuda")
+    n_out = ctypes.c_int64()
+
+    def call(cap):
+        if op == "pairs":
+            return lib.spade_join_pairs(cv.handle, ctypes.c_void_p(xy.data_ptr()), len(xy_h), 9,
+                                        ctypes.c_void_p(pt.data_ptr()), ctypes.c_void_p(pl.data_ptr()), cap,
+                                        ctypes.byref(n_out), None)
+        return lib.spade_select(cv.handle, ctypes.c_void_p(xy.data_ptr()), len(xy_h), 9,
+                                ctypes.c_void_p(pt.data_ptr()), cap, ctypes.byref(n_out), None)
+
+    assert call(M - 1) == spade.SPADE_ERR_CAPACITY and n_out.value == M
+    pt.fill_(-7)
+    pl.fill_(-7)
+    assert call(M) == 0 and n_out.value == M
+    torch.cuda.synchronize()
+    assert bool((pt[M:] == -7).all()) and bool((pl[M:] == -7).all())
+    if op == "pairs":
+        a, b = sorted_pairs(pt[:M].cpu().numpy(), pl[:M].cpu().numpy())
+        np.testing.assert_array_equal(a, opt)
+        np.testing.assert_array_equal(b, opl)
+    else:
+        np.testing.assert_array_equal(np.sort(pt[:M].cpu().numpy()), oids)
