@@ -26,6 +26,7 @@
 #include <cstdio>
 #include <cub/block/block_scan.cuh>
 #include <cub/block/block_radix_sort.cuh>
+#include <cub/block/block_reduce.cuh>
 #include "spade_internal.cuh"
 
 namespace spade {
@@ -724,50 +725,80 @@ struct FixMeta {
   long long M, nmove;
 };
 
-template <int MODE>
+// Sorting the holes by start: relative 32-bit keys with only the bits the range needs (the
+// common case), else full 64-bit keys.
+template <typename Key>
+__device__ __forceinline__ void sort_holes(unsigned long long (&start)[kFixItems], int (&len)[kFixItems],
+                                           unsigned long long lo, int bits, void* tmp) {
+  using Sort = cub::BlockRadixSort<Key, kFixT, kFixItems, int>;
+  Key key[kFixItems];
+#pragma unroll
+  for (int i = 0; i < kFixItems; ++i) key[i] = (Key)(start[i] - lo);
+  Sort(*(typename Sort::TempStorage*)tmp).Sort(key, len, 0, bits);
+#pragma unroll
+  for (int i = 0; i < kFixItems; ++i) start[i] = lo + (unsigned long long)key[i];
+}
+
 __global__ void __launch_bounds__(kFixT) k_fixup(const longlong2* __restrict__ holes, int nh, unsigned long long* total,
                                                  int64_t cap, long long* __restrict__ dst_start,
                                                  long long* __restrict__ dst_pre, long long* __restrict__ src_start,
                                                  long long* __restrict__ src_pre, FixMeta* meta) {
-  using Sort = cub::BlockRadixSort<unsigned long long, kFixT, kFixItems, long long>;
+  using Sort32 = cub::BlockRadixSort<unsigned int, kFixT, kFixItems, int>;
+  using Sort64 = cub::BlockRadixSort<unsigned long long, kFixT, kFixItems, int>;
   using Scan = cub::BlockScan<long long, kFixT>;
+  using Red = cub::BlockReduce<unsigned long long, kFixT>;
   __shared__ union {
-    typename Sort::TempStorage sort;
+    typename Sort32::TempStorage s32;
+    typename Sort64::TempStorage s64;
     typename Scan::TempStorage scan;
+    typename Red::TempStorage red;
     long long next[kMaxHoles + 1];
   } sm;
-  __shared__ unsigned long long s_H;
-  unsigned long long key[kFixItems];
-  long long len[kFixItems];
-  long long hl = 0;
+  __shared__ unsigned long long s_H, s_lo, s_hi;
+  const long long T = (long long)*total;
+  unsigned long long st[kFixItems];
+  int len[kFixItems];
+  unsigned long long hl = 0, lo = ~0ull, hi = 0;
 #pragma unroll
   for (int i = 0; i < kFixItems; ++i) {
     const int h = threadIdx.x * kFixItems + i;
     const longlong2 v = h < nh ? holes[h] : make_longlong2(0, 0);
-    len[i] = v.y;
-    key[i] = v.y > 0 ? (unsigned long long)v.x : ~0ull;      // empty holes sort last
-    hl += v.y;
+    len[i] = (int)v.y;
+    st[i] = v.y > 0 ? (unsigned long long)v.x : ~0ull;       // empty holes: sorted last
+    hl += (unsigned long long)v.y;
+    if (v.y > 0) { lo = min(lo, (unsigned long long)v.x); hi = max(hi, (unsigned long long)v.x); }
   }
-  if (threadIdx.x == 0) s_H = 0;
+  unsigned long long r = Red(sm.red).Sum(hl);
+  if (threadIdx.x == 0) s_H = r;
   __syncthreads();
-  atomicAdd(&s_H, (unsigned long long)hl);
-  Sort(sm.sort).Sort(key, len);                   // blocked arrangement, ascending starts
+  r = Red(sm.red).Reduce(lo, cub::Min());
+  if (threadIdx.x == 0) s_lo = r;
   __syncthreads();
-  const long long T = (long long)*total, M = T - (long long)s_H;
+  r = Red(sm.red).Reduce(hi, cub::Max());
+  if (threadIdx.x == 0) s_hi = r;
+  __syncthreads();
+  const unsigned long long L = s_lo == ~0ull ? 0ull : s_lo, span = s_lo == ~0ull ? 0ull : s_hi - s_lo + 1;
+#pragma unroll
+  for (int i = 0; i < kFixItems; ++i) if (st[i] == ~0ull) st[i] = L + span;   // empty: past every start
+  const int bits = span == 0 ? 1 : 64 - __clzll(span);
+  if (bits <= 32) sort_holes<unsigned int>(st, len, L, bits, &sm);
+  else sort_holes<unsigned long long>(st, len, L, bits, &sm);
+  __syncthreads();
+  const long long M = T - (long long)s_H;
   // Hole i = [a, e).  Destinations: its part below M.  Sources: the run of result slots after
   // its part at or past M, [max(e, M), max(a', M)) with a' the next hole's start (T after the
   // last), plus the leading run [M, max(a_0, M)).
 #pragma unroll
   for (int i = 0; i < kFixItems; ++i)
-    sm.next[threadIdx.x * kFixItems + i] = key[i] != ~0ull ? max((long long)key[i], M) : T;
+    sm.next[threadIdx.x * kFixItems + i] = len[i] > 0 ? max((long long)st[i], M) : T;
   if (threadIdx.x == 0) sm.next[kMaxHoles] = T;
   __syncthreads();
   long long dl[kFixItems], gs[kFixItems], gl[kFixItems];
   long long dsum = 0, gsum = 0;
 #pragma unroll
   for (int i = 0; i < kFixItems; ++i) {
-    const bool valid = key[i] != ~0ull;
-    const long long a = (long long)key[i], e = a + len[i];
+    const bool valid = len[i] > 0;
+    const long long a = (long long)st[i], e = a + len[i];
     dl[i] = valid && a < M ? min(e, M) - a : 0;
     gs[i] = valid ? max(e, M) : T;
     gl[i] = valid ? max(sm.next[threadIdx.x * kFixItems + i + 1] - gs[i], 0ll) : 0;
@@ -783,7 +814,7 @@ __global__ void __launch_bounds__(kFixT) k_fixup(const longlong2* __restrict__ h
 #pragma unroll
   for (int i = 0; i < kFixItems; ++i) {
     const int h = threadIdx.x * kFixItems + i;
-    dst_start[h] = key[i] != ~0ull ? (long long)key[i] : T;
+    dst_start[h] = len[i] > 0 ? (long long)st[i] : T;
     dst_pre[h] = dex;                             // exclusive prefix of destination slots
     dex += dl[i];
     src_start[h + 1] = gs[i];
@@ -933,7 +964,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       }
     }
     if (kOut && e == cudaSuccess) {
-      k_fixup<MODE><<<1, kFixT, 0, st>>>(p.o.holes, grid * kNW, p.o.total, p.o.cap, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
+      k_fixup<<<1, kFixT, 0, st>>>(p.o.holes, grid * kNW, p.o.total, p.o.cap, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
       count_launch();
       k_move<MODE><<<sms * 4, 256, 0, st>>>(p.o, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
       count_launch();
