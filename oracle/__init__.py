@@ -25,7 +25,8 @@ _lib = None
 def build(force: bool = False) -> str:
     """Compile spade_oracle.c (+ the R-tree CPU baseline, rtree_join.c) into liboracle.so
     (plain gcc, -O2, pthreads)."""
-    srcs = [os.path.join(_HERE, "spade_oracle.c"), os.path.join(_HERE, "rtree_join.c")]
+    srcs = [os.path.join(_HERE, "spade_oracle.c"), os.path.join(_HERE, "rtree_join.c"),
+            os.path.join(_HERE, "distance_oracle.c")]
     newest = max(os.path.getmtime(x) for x in srcs)
     if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < newest:
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-pthread", "-o", _LIB_PATH, *srcs])
@@ -49,6 +50,16 @@ def _load():
         lib.oracle_select.restype = i64
         lib.rtree_join_count.argtypes = [P, i64, P, P, P, i32, P, ctypes.c_int]
         lib.rtree_join_count.restype = ctypes.c_int
+        lib.oracle_in_disk.argtypes = [i64, i64, i64, i64, i64]
+        lib.oracle_in_disk.restype = ctypes.c_int
+        lib.oracle_disk_join_count.argtypes = [P, i64, P, P, i32, P, ctypes.c_int]
+        lib.oracle_disk_join_count.restype = ctypes.c_int
+        lib.oracle_disk_join_pairs.argtypes = [P, i64, i64, P, P, i32, P, P, i64, ctypes.c_int]
+        lib.oracle_disk_join_pairs.restype = i64
+        lib.oracle_disk_select.argtypes = [P, i64, i64, P, P, i32, P, i64, ctypes.c_int]
+        lib.oracle_disk_select.restype = i64
+        lib.oracle_knn.argtypes = [P, i64, i64, i64, i64, i64, P, P]
+        lib.oracle_knn.restype = i64
         _lib = lib
     return _lib
 
@@ -142,3 +153,71 @@ def labels_at(xy, polys, nthreads: int | None = None):
     for a, b in zip(pt.tolist(), pl.tolist()):
         out[a].append(b)
     return out
+
+
+# ---- distance-based queries over points and kNN (distance_oracle.c) ----
+
+def _disks(disks):
+    cxy = np.ascontiguousarray(disks["center_xy"], dtype=np.int32).reshape(-1, 2)
+    r2 = np.ascontiguousarray(disks["r2"], dtype=np.int64).reshape(-1)
+    assert len(r2) == len(cxy)
+    return cxy, r2, len(cxy)
+
+
+def in_disk(px: int, py: int, cx: int, cy: int, r2: int) -> bool:
+    """(px-cx)^2 + (py-cy)^2 <= r2 (closed disk, squared integer radius)."""
+    return bool(_load().oracle_in_disk(int(px), int(py), int(cx), int(cy), int(r2)))
+
+
+def disk_join_count(xy, disks, nthreads: int | None = None) -> np.ndarray:
+    """int64[D] number of points within each disk (aggregation over a distance canvas)."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    cxy, r2, D = _disks(disks)
+    counts = np.zeros(max(D, 1), dtype=np.int64)
+    if lib.oracle_disk_join_count(_ptr(xy), len(xy), _ptr(cxy), _ptr(r2), D, _ptr(counts),
+                                  nthreads or default_threads()) != 0:
+        raise MemoryError("oracle_disk_join_count failed")
+    return counts[:D]
+
+
+def disk_join_pairs(xy, disks, point_id_base: int = 0, nthreads: int | None = None):
+    """(point_ids int64, disk_ids int32) sorted by (point, disk): the type 1 / type 2 distance
+    join with the disks as the constraint side."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    cxy, r2, D = _disks(disks)
+    nt = nthreads or default_threads()
+    total = lib.oracle_disk_join_pairs(_ptr(xy), len(xy), point_id_base, _ptr(cxy), _ptr(r2), D, None, None, 0, nt)
+    if total < 0:
+        raise MemoryError("oracle_disk_join_pairs failed")
+    pt = np.empty(max(total, 1), dtype=np.int64)
+    pl = np.empty(max(total, 1), dtype=np.int32)
+    lib.oracle_disk_join_pairs(_ptr(xy), len(xy), point_id_base, _ptr(cxy), _ptr(r2), D, _ptr(pt), _ptr(pl), total, nt)
+    return pt[:total], pl[:total]
+
+
+def disk_select(xy, disks, point_id_base: int = 0, nthreads: int | None = None) -> np.ndarray:
+    """int64 ids of points within at least one disk, ascending (distance selection)."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    cxy, r2, D = _disks(disks)
+    out = np.empty(max(len(xy), 1), dtype=np.int64)
+    total = lib.oracle_disk_select(_ptr(xy), len(xy), point_id_base, _ptr(cxy), _ptr(r2), D, _ptr(out), len(out),
+                                   nthreads or default_threads())
+    if total < 0:
+        raise MemoryError("oracle_disk_select failed")
+    return out[:total]
+
+
+def knn(xy, q, k: int, point_id_base: int = 0):
+    """(ids int64[min(k,n)], dist2 int64) of the k points nearest to q, ties by id."""
+    lib = _load()
+    xy = np.ascontiguousarray(xy, dtype=np.int32).reshape(-1, 2)
+    m = max(min(k, len(xy)), 1)
+    ids = np.empty(m, dtype=np.int64)
+    d2 = np.empty(m, dtype=np.int64)
+    got = lib.oracle_knn(_ptr(xy), len(xy), point_id_base, int(q[0]), int(q[1]), int(k), _ptr(ids), _ptr(d2))
+    if got < 0:
+        raise MemoryError("oracle_knn failed")
+    return ids[:got], d2[:got]

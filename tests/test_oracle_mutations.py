@@ -22,18 +22,39 @@ MUTANTS = {
                         "for (int64_t r = ring_begin; r < ring_begin + 1 && r < ring_end; ++r) {"),
     "flipped_sign": ("return by > ay ? (o > 0) : (o < 0);", "return by > ay ? (o < 0) : (o > 0);"),
 }
+# distance / kNN oracle (oracle/distance_oracle.c) against tests/test_distance_oracle_pins.py
+DIST_MUTANTS = {
+    "open_disk": ("return dx * dx + dy * dy <= (__int128)r2;", "return dx * dx + dy * dy < (__int128)r2;"),
+    "dropped_dy": ("return dx * dx + dy * dy <= (__int128)r2;", "return dx * dx <= (__int128)r2;"),
+    "mixed_term": ("return dx * dx + dy * dy <= (__int128)r2;", "return dx * dx + dx * dy <= (__int128)r2;"),
+    "int64_overflow": ("__int128 dx = (__int128)px - cx, dy = (__int128)py - cy;\n    return",
+                       "int64_t dx = px - cx, dy = py - cy;\n    return"),
+    "swapped_axis": ("__int128 dx = (__int128)px - cx, dy = (__int128)py - cy;\n    return",
+                     "__int128 dx = (__int128)px - cy, dy = (__int128)py - cx;\n    return"),
+    "knn_reversed_ties": ("return (x->id > y->id) - (x->id < y->id);", "return (x->id < y->id) - (x->id > y->id);"),
+    "knn_off_by_one": ("for (int64_t i = 0; i < k; ++i) {\n        out_ids[i] = a[i].id;",
+                       "for (int64_t i = 0; i < k; ++i) {\n        out_ids[i] = a[i + (i + 1 < n)].id;"),
+}
+
+
+def _run_mutant(tmp_path, name, src_name, old, new, pins):
+    for d in ("oracle", "gen", "tests"):
+        shutil.copytree(os.path.join(ROOT, d), tmp_path / d,
+                        ignore=shutil.ignore_patterns("liboracle.so", "__pycache__", "*.o"))
+    src = tmp_path / "oracle" / src_name
+    text = src.read_text()
+    assert text.count(old) == 1, f"mutation site for {name} not found"
+    src.write_text(text.replace(old, new))
+    r = subprocess.run([sys.executable, "-m", "pytest", pins, "-q", "-x",
+                        "-p", "no:cacheprovider"], cwd=tmp_path, capture_output=True, text=True, timeout=600)
+    assert r.returncode != 0, f"mutant {name} survived the pins:\n{r.stdout[-2000:]}"
 
 
 @pytest.mark.parametrize("name", sorted(MUTANTS))
 def test_pins_kill_mutant(name, tmp_path):
-    old, new = MUTANTS[name]
-    for d in ("oracle", "gen", "tests"):
-        shutil.copytree(os.path.join(ROOT, d), tmp_path / d,
-                        ignore=shutil.ignore_patterns("liboracle.so", "__pycache__", "*.o"))
-    src = tmp_path / "oracle" / "spade_oracle.c"
-    text = src.read_text()
-    assert text.count(old) == 1, f"mutation site for {name} not found"
-    src.write_text(text.replace(old, new))
-    r = subprocess.run([sys.executable, "-m", "pytest", "tests/test_oracle_pins.py", "-q", "-x",
-                        "-p", "no:cacheprovider"], cwd=tmp_path, capture_output=True, text=True, timeout=600)
-    assert r.returncode != 0, f"mutant {name} survived the pins:\n{r.stdout[-2000:]}"
+    _run_mutant(tmp_path, name, "spade_oracle.c", *MUTANTS[name], "tests/test_oracle_pins.py")
+
+
+@pytest.mark.parametrize("name", sorted(DIST_MUTANTS))
+def test_distance_pins_kill_mutant(name, tmp_path):
+    _run_mutant(tmp_path, name, "distance_oracle.c", *DIST_MUTANTS[name], "tests/test_distance_oracle_pins.py")
