@@ -35,8 +35,9 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5"],
-                    help="c3 (default) = the metric's join+COUNT config; c2 select, c4 pairs, c5 40k polygons")
+    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5", "dj", "dj2", "knn"],
+                    help="c3 (default) = the metric's join+COUNT config; c2 select, c4 pairs, c5 40k polygons; "
+                         "dj / dj2 distance joins (type 1 pairs / type 2 count), knn kNN selection")
     ap.add_argument("--points-per-gpu", type=int, default=None, help="default: the config's size (1B; C2 100M)")
     ap.add_argument("--impl", default="spade", choices=["spade", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -60,11 +61,16 @@ METRICS = {
     "count": METRIC,
     "select": "points/sec for spatial selection (ids of points inside the query polygon)",
     "pairs": "points/sec for point-polygon join emitting (point_id, polygon_id) pairs",
+    "dist_pairs": "points/sec for the type 1 distance join emitting (point_id, disk_id) pairs",
+    "dist_count": "points/sec for the type 2 distance join COUNT (per-disk counts)",
+    "knn": "points/sec scanned by kNN selection (circle aggregation + distance select + sort)",
 }
 
 
 def workload(name, n_per_gpu):
     from gen import configs
+    if name in configs.DISTANCE:
+        return configs.DISTANCE[name](n_per_gpu or 1_000_000_000)
     if name in ("c1", "c2"):
         return getattr(configs, name)() if n_per_gpu is None else getattr(configs, name)(n_per_gpu)
     return getattr(configs, name)(n_per_gpu or 1_000_000_000)
@@ -137,12 +143,41 @@ class ClockSampler:
                 "samples": len(self.samples)}
 
 
+def _oracle_run(w, xy, nt):
+    """The oracle call matching the workload's operation (as it stands)."""
+    import numpy as np
+    import oracle
+    if getattr(w, "op", "") == "knn":
+        oracle.knn(xy, w.query, w.k)
+        return np.zeros(1, np.int64)
+    if hasattr(w, "disks"):
+        return oracle.disk_join_count(xy, w.disks, nthreads=nt)
+    return oracle.join_count(xy, w.polys, nthreads=nt)
+
+
 def cpu_oracle_rate(w, target_s, seed_offset=0):
     """Time the oracle (as it stands) on a bounded sample of the workload's points."""
     import numpy as np
     import gen
     import oracle
     nt = oracle.default_threads()
+    if hasattr(w, "disks"):
+        idx = np.arange(0, 2000, dtype=np.int64) * 499 + seed_offset
+        pilot = gen.points_at(w.points, w.point_seed, idx)
+        t0 = time.perf_counter()
+        _oracle_run(w, pilot, nt)
+        dt = max(time.perf_counter() - t0, 1e-3)
+        m = int(max(2000, min(50_000_000, len(pilot) * target_s / dt)))
+        stride = max(1, w.n_points // m)
+        xy = gen.points_at(w.points, w.point_seed, np.arange(m, dtype=np.int64) * stride + seed_offset)
+        t0 = time.perf_counter()
+        _oracle_run(w, xy, nt)
+        dt = time.perf_counter() - t0
+        what = (f"kNN (k={w.k}) by sorting all sampled points" if w.op == "knn" else
+                f"x {len(w.disks['r2'])} disks, brute force over all pairs")
+        return {"value": m / dt, "unit": "points/s", "cores": 1 if w.op == "knn" else nt, "kind": "oracle",
+                "sample": f"{m} points = every {stride}-th global index of the workload's point stream, {what} "
+                          f"({dt:.1f} s)", "seconds": dt, "sum_counts": 0}
     idx = np.arange(0, 2000, dtype=np.int64) * 499 + seed_offset
     pilot = gen.points_at(w.points, w.point_seed, idx)
     t0 = time.perf_counter()
@@ -198,8 +233,10 @@ def run_reference(a):
         rates.append(res["value"])
         secs += res["seconds"]
     value = statistics.median(rates)
+    op = w.op
+    is_dist = hasattr(w, "disks")
     line = {
-        "impl": "reference", "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": a.gpus,
+        "impl": "reference", "metric": METRICS[("dist_" + op) if is_dist and op != "knn" else op], "value": value, "unit": "points/s", "n_gpus": a.gpus,
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * secs / max(1, a.steps),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
         "data": "synthetic", "config": {"workload": w.name, "desc": w.desc, "points_per_gpu": w.n_points},
@@ -232,17 +269,23 @@ def main():
     sp.load()
     w = workload(a.workload, a.points_per_gpu)
     n = w.n_points
-    P = len(w.polys["poly_ring_off"]) - 1
+    is_dist = hasattr(w, "disks")
+    P = len(w.disks["r2"]) if is_dist else len(w.polys["poly_ring_off"]) - 1
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
 
-    # canvas build (timed separately; not part of a step)
+    # canvas build (timed separately; not part of a step); kNN builds no canvas (knn.cu)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    cv = sp.Canvas(w.polys, max_dim=a.max_dim or w.max_dim, dense=a.dense)
+    if w.op == "knn":
+        cv = None
+    elif is_dist:
+        cv = sp.Canvas.disks(w.disks["center_xy"], w.disks["r2"], max_dim=a.max_dim or w.max_dim, dense=a.dense)
+    else:
+        cv = sp.Canvas(w.polys, max_dim=a.max_dim or w.max_dim, dense=a.dense)
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
-    info = cv.info()
+    info = cv.info() if cv is not None else {}
 
     # this rank's shard: global indices [rank*n, (rank+1)*n), generated in place on the device
     xy = torch.empty((n, 2), dtype=torch.int32, device=dev)
@@ -262,6 +305,8 @@ def main():
             ev_k0.record(stream)
         if op == "count":
             sp.join_count(cv, xy, counts)
+        elif op == "knn":
+            n_results[0] = sp.knn(xy, w.query, w.k, point_id_base=rank * n)[0].numel()
         elif op == "select":
             n_results[0] = sp.select(cv, xy, point_id_base=rank * n, out=out_sel).numel()
         else:
@@ -302,10 +347,16 @@ def main():
     total_pts = n * ws
     value = total_pts * a.steps / (t_max / 1e3)
     # correctness guard: tilings cover the whole domain, every point is counted exactly once
-    if op == "count":
+    if op == "count" and is_dist:
+        check = {"pairs_counted": int(counts.sum().item())}
+    elif op == "count":
         check = {"sum_counts_equals_points": int(counts.sum().item()) == total_pts}
+    elif op == "pairs" and is_dist:
+        check = {"pairs": n_results[0], "pairs_per_point": n_results[0] / n}
     elif op == "pairs":
         check = {"one_pair_per_point": n_results[0] == n}
+    elif op == "knn":
+        check = {"k_returned": n_results[0], "k": w.k, "note": "single-GPU kNN per rank (N>1: per-shard)"}
     else:
         check = {"selected": n_results[0], "selectivity": n_results[0] / n}
 
@@ -313,7 +364,8 @@ def main():
     peak, peak_src = measured_peak()
     # algorithmic bytes per launch: the int2 stream, plus the results written (select: 8 B id per
     # selected point; pairs: 8 B id + 4 B polygon id per pair); counts are 8*P bytes, negligible
-    out_bytes = {"count": 0, "select": 8 * n_results[0], "pairs": 12 * n_results[0]}[op]
+    # kNN: two passes over the points (circle aggregation, distance selection)
+    out_bytes = {"count": 0, "select": 8 * n_results[0], "pairs": 12 * n_results[0], "knn": n * 8}[op]
     alg_bytes = n * 8 + out_bytes
     achieved = alg_bytes / (kavg / 1e3) / 1e9
     traffic, traffic_src = ncu_traffic(w.name)
@@ -321,18 +373,21 @@ def main():
     line = None
     if rank == 0:
         line = {
-            "metric": METRICS[op], "value": value, "unit": "points/s", "n_gpus": ws, "steps": a.steps,
+            "metric": METRICS[("dist_" + op) if is_dist and op != "knn" else op], "value": value, "unit": "points/s", "n_gpus": ws, "steps": a.steps,
             "warmup": max(3, a.warmup), "ms_per_step": t_max / a.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {
-                "workload": w.name, "desc": w.desc, "points_per_gpu": n, "polygons": P,
-                "vertices": int(len(w.polys["ring_xy"])), "parallelism": f"dp{ws} (points sharded, canvas replicated)",
+                "workload": w.name, "desc": w.desc, "points_per_gpu": n,
+                **({"disks": P} if is_dist and op != "knn" else {"k": w.k, "query": list(w.query)} if op == "knn"
+                   else {"polygons": P, "vertices": int(len(w.polys["ring_xy"]))}),
+                "parallelism": f"dp{ws} (points sharded, canvas replicated)",
                 "l2": "inputs (8 B/point, >= 8 GB per GPU) exceed the 126 MB L2; no flush needed",
                 "canvas": info, "canvas_build_s": build_s,
             },
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": {"count": "k_probe<COUNT> (spade_join_count)",
+                         "kernel": {"knn": "k_knn_hist + k_knn_select + top-k sort (spade_knn; includes its host syncs)",
+                                    "count": "k_probe<COUNT> (spade_join_count)",
                                     "select": "k_probe<SELECT> (spade_select; includes its n_out readback)",
                                     "pairs": "k_probe<PAIRS> (spade_join_pairs; includes its n_out readback)"}[op],
                          "kernel_ms": kavg, "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,

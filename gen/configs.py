@@ -89,4 +89,67 @@ def c5(n_points_per_gpu: int = 1_000_000_000) -> Workload:
                     desc="scale-out join COUNT: 1B points per GPU x 40k zip-code-like polygons")
 
 
+# ---- distance-based queries (Sec. 6.4-6.5) ----
+# The paper joins the Taxi data with 100..100K random points generated within its extent, at a
+# query distance of 5..100 m (20 m by default, Fig. 7).  The synthetic domain [0, 2^24)^2 stands
+# for the ~45 km Taxi extent: 1 m = 2^24 / 45,000 grid units.
+UNITS_PER_METER = (1 << 24) / 45_000.0
+
+
+def meters_to_r2(m: float) -> int:
+    """Squared radius in grid units for a distance in metres (floor of r^2, reading D2)."""
+    r = m * UNITS_PER_METER
+    return int(np.floor(r * r))
+
+
+@dataclass
+class DiskWorkload:
+    name: str
+    op: str                    # "pairs" | "count" | "select" | "knn"
+    points: SgParams
+    point_seed: int
+    n_points: int
+    disks: dict = field(repr=False)   # {"center_xy": (D,2) int32, "r2": (D,) int64}
+    max_dim: int = 4096
+    desc: str = ""
+    k: int = 0                 # kNN only
+    query: tuple = (0, 0)      # kNN only
+
+
+def random_centers(n: int, seed: int) -> np.ndarray:
+    """n uniform random points within the extent of the taxi-like data (the paper's generated
+    point set), kept 1,000 m from the domain edge so every disk stays inside it."""
+    rng = np.random.default_rng(seed)
+    m = int(1000 * UNITS_PER_METER)
+    return rng.integers(m, (1 << 24) - m, size=(n, 2)).astype(np.int32)
+
+
+def dj(n_points: int = 1_000_000_000, n_disks: int = 100_000, meters: float = 20.0) -> DiskWorkload:
+    c = random_centers(n_disks, 602)
+    return DiskWorkload(f"dj_taxi1B_x{n_disks // 1000}k_r{int(meters)}m_pairs", "pairs", taxi_params(601), 601,
+                        n_points, {"center_xy": c, "r2": np.full(n_disks, meters_to_r2(meters), np.int64)},
+                        max_dim=16384,
+                        desc=f"type 1 distance join: 1B taxi-like points x {n_disks} random points, distance <= {meters} m")
+
+
+def dj2(n_points: int = 1_000_000_000, n_disks: int = 100_000) -> DiskWorkload:
+    """Type 2 distance join: one radius per generated point, log-uniform in [5, 100] m."""
+    c = random_centers(n_disks, 612)
+    rng = np.random.default_rng(613)
+    m = np.exp(rng.uniform(np.log(5.0), np.log(100.0), n_disks))
+    r2 = np.array([meters_to_r2(x) for x in m], np.int64)
+    return DiskWorkload(f"dj2_taxi1B_x{n_disks // 1000}k_r5to100m_count", "count", taxi_params(611), 611, n_points,
+                        {"center_xy": c, "r2": r2}, max_dim=16384,
+                        desc=f"type 2 distance join COUNT: 1B taxi-like points x {n_disks} points with radii 5..100 m")
+
+
+def knn(n_points: int = 1_000_000_000, k: int = 50) -> DiskWorkload:
+    """kNN selection (Fig. 8): the k taxi points nearest to one generated query point."""
+    q = random_centers(100, 622)[0]
+    return DiskWorkload(f"knn_taxi1B_k{k}", "knn", taxi_params(621), 621, n_points,
+                        {"center_xy": np.zeros((0, 2), np.int32), "r2": np.zeros(0, np.int64)}, k=k,
+                        query=(int(q[0]), int(q[1])), desc=f"kNN selection: {k} nearest of 1B taxi-like points")
+
+
 ALL = {"c1": c1, "c2": c2, "c3": c3, "c4": c4, "c5": c5}
+DISTANCE = {"dj": dj, "dj2": dj2, "knn": knn}

@@ -85,6 +85,24 @@ SPADE_API int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off
                        int32_t num_polys, const spade_canvas_params* prm, spade_stream_t stream,
                        spade_canvas** out);
 
+/* Build a DISTANCE canvas ("Canvases for Distance-Based Queries", Sec. 4.2; used by the
+ * distance-based selections and joins of P:204-210, Sec. 5.2): one closed disk per constraint,
+ *   disk d = { (x, y) : (x - cx_d)^2 + (y - cy_d)^2 <= r2_d }      (readings D1-D4)
+ * The squared radius is an integer: for integer points "distance <= r" is exactly
+ * "dist2 <= floor(r^2)", so any real radius r is represented by r2 = floor(r^2).
+ *   center_xy [D*2] int32 disk centres (x, y) interleaved
+ *   r2        [D]   int64 squared radii, 0 <= r2 < 2^62
+ *   num_disks D >= 0; the disk id of center_xy[d] is d
+ * Type 1 distance join (one r): all r2 equal.  Type 2 (per-object r_i): per-disk r2.
+ * Every disk's integer points must lie in [-2^30, 2^30)^2: cx - isqrt(r2) >= -2^30 and
+ * cx + isqrt(r2) < 2^30 (same for y), else SPADE_ERR_COORD_RANGE; r2 out of range or NULL
+ * arrays: SPADE_ERR_INVALID_ARG.  The canvas is used with the same calls as a polygon canvas
+ * (spade_join_count, spade_select, spade_join_pairs, spade_join_count_host), with "polygon id"
+ * meaning disk id and "inside" meaning within the closed disk; disks may overlap (a point joins
+ * every disk containing it).  Ownership and synchronisation as spade_build_canvas. */
+SPADE_API int spade_build_disk_canvas(const int32_t* center_xy, const int64_t* r2, int32_t num_disks,
+                            const spade_canvas_params* prm, spade_stream_t stream, spade_canvas** out);
+
 /* Release a canvas (NULL is a no-op).  Synchronises the device. */
 SPADE_API void spade_canvas_free(spade_canvas* c);
 
@@ -128,6 +146,48 @@ SPADE_API int spade_join_pairs(const spade_canvas* c, const int32_t* xy, int64_t
  * paper's times are dominated by exactly this host->GPU transfer). */
 SPADE_API int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t n,
                           int64_t* counts_host, spade_stream_t stream);
+
+/* ---- kNN selection over points (Sec. 5.2), in the paper's three steps ------------
+ * The circles of step 1 are concentric around the query q with squared radii
+ *   r2_b = the largest squared distance of bucket b,  b = 0 .. SPADE_KNN_BINS-1, where
+ *   bucket(d2) = d2 (d2 < 4),  4 + 4(e-2) + ((d2 >> (e-2)) & 3) (d2 >= 4, e = floor(log2 d2))
+ * (consecutive radii differ by a factor <= sqrt(1.25): the paper's r_i = r_max / alpha^i with
+ * the circles aligned to quarter-octaves of the squared distance).
+ * Coordinates of the query and of every point must lie in [-2^30, 2^30) (squared distances are
+ * then exact in int64); points outside are counted in hist[SPADE_KNN_BINS] and make spade_knn
+ * fail with SPADE_ERR_COORD_RANGE.  The result is unique: the k points smallest in
+ * (squared distance, point id) (reading D3). */
+#define SPADE_KNN_BINS 248
+
+/* Step 1: aggregation over the circles.  ACCUMULATES into hist[SPADE_KNN_BINS + 1]
+ * (int64, device): hist[b] = points in bucket b, hist[SPADE_KNN_BINS] = out-of-range points;
+ * COUNT(circle b) = hist[0] + ... + hist[b].  Asynchronous.  Sum the histograms of several point
+ * shards (e.g. all_reduce) before step 2. */
+SPADE_API int spade_knn_histogram(const int32_t* xy, int64_t n, int32_t qx, int32_t qy, int64_t* hist,
+                        spade_stream_t stream);
+
+/* Between steps 1 and 2 (host): the smallest circle b with COUNT(circle b) >= k (the last
+ * circle if fewer than k points exist).  hist_host[SPADE_KNN_BINS + 1] as above.  Outputs its
+ * squared radius and its count (the number of candidates step 2 returns). */
+SPADE_API int spade_knn_radius(const int64_t* hist_host, int64_t k, int64_t* r2_out, int64_t* count_out);
+
+/* Step 2: distance selection — ids (point_id_base + index) and squared distances of the
+ * points with dist2 <= r2, order unspecified, capacity protocol of spade_select.  Syncs. */
+SPADE_API int spade_knn_select(const int32_t* xy, int64_t n, int64_t point_id_base, int32_t qx, int32_t qy,
+                     int64_t r2, int64_t* out_ids, int64_t* out_d2, int64_t capacity, int64_t* n_out,
+                     spade_stream_t stream);
+
+/* Step 3: sort m candidates (ids >= 0, d2 as from step 2) by (d2, id) and write the
+ * first min(k, m) to out_ids / out_d2 (out_d2 may be NULL).  Asynchronous. */
+SPADE_API int spade_knn_topk(const int64_t* ids, const int64_t* d2, int64_t m, int64_t k, int64_t* out_ids,
+                   int64_t* out_d2, spade_stream_t stream);
+
+/* All three steps on one device: the min(k, n) nearest points to (qx, qy).
+ *   out_ids [k] int64 device, out_d2 [k] int64 device (may be NULL), n_out HOST = min(k, n).
+ * Errors: INVALID_ARG (k < 0, NULL pointers), COORD_RANGE (query or a point out of range),
+ * OOM, CUDA.  Synchronises `stream`. */
+SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int32_t qx, int32_t qy, int64_t k,
+              int64_t* out_ids, int64_t* out_d2, int64_t* n_out, spade_stream_t stream);
 
 /* Number of kernels this library has launched in this process (for the bench's gpu_launches). */
 SPADE_API int64_t spade_launch_count(void);

@@ -9,6 +9,8 @@ CPU fallback: if the extension cannot be loaded, or no CUDA device is present, c
     ids    = select(canvas, xy)                  # spade_select         (selection)
     pt, pl = join_pairs(canvas, xy)              # spade_join_pairs     (join)
     counts = join_count_host(canvas, xy_numpy)   # spade_join_count_host (host-resident points)
+    dcv    = Canvas.disks(centers, r2)           # spade_build_disk_canvas (distance canvas)
+    ids, d2 = knn(xy, (qx, qy), k)               # spade_knn              (kNN selection)
 
 `polys` is a dict with ``ring_xy`` (V,2) int32, ``ring_off`` (R+1) int64, ``poly_ring_off``
 (P+1) int64 (numpy arrays or torch tensors), the layout spade_build_canvas takes.
@@ -59,6 +61,8 @@ def load(path: str | None = None):
     P, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
     lib.spade_build_canvas.argtypes = [P, P, P, i32, ctypes.POINTER(CanvasParams), P, ctypes.POINTER(P)]
     lib.spade_build_canvas.restype = ctypes.c_int
+    lib.spade_build_disk_canvas.argtypes = [P, P, i32, ctypes.POINTER(CanvasParams), P, ctypes.POINTER(P)]
+    lib.spade_build_disk_canvas.restype = ctypes.c_int
     lib.spade_canvas_free.argtypes = [P]
     lib.spade_canvas_free.restype = None
     lib.spade_canvas_info.argtypes = [P] + [ctypes.POINTER(i32)] * 6 + [ctypes.POINTER(i64)] * 2 + [ctypes.POINTER(ctypes.c_double)]
@@ -71,6 +75,16 @@ def load(path: str | None = None):
     lib.spade_join_pairs.restype = ctypes.c_int
     lib.spade_join_count_host.argtypes = [P, P, i64, P, P]
     lib.spade_join_count_host.restype = ctypes.c_int
+    lib.spade_knn_histogram.argtypes = [P, i64, i32, i32, P, P]
+    lib.spade_knn_histogram.restype = ctypes.c_int
+    lib.spade_knn_radius.argtypes = [P, i64, ctypes.POINTER(i64), ctypes.POINTER(i64)]
+    lib.spade_knn_radius.restype = ctypes.c_int
+    lib.spade_knn_select.argtypes = [P, i64, i64, i32, i32, i64, P, P, i64, ctypes.POINTER(i64), P]
+    lib.spade_knn_select.restype = ctypes.c_int
+    lib.spade_knn_topk.argtypes = [P, P, i64, i64, P, P, P]
+    lib.spade_knn_topk.restype = ctypes.c_int
+    lib.spade_knn.argtypes = [P, i64, i64, i32, i32, i64, P, P, ctypes.POINTER(i64), P]
+    lib.spade_knn.restype = ctypes.c_int
     lib.spade_launch_count.argtypes = []
     lib.spade_launch_count.restype = i64
     lib.spade_status_string.argtypes = [ctypes.c_int]
@@ -81,8 +95,9 @@ def load(path: str | None = None):
     return lib
 
 
-EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_canvas_free", "spade_canvas_info", "spade_join_count",
-                    "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_launch_count",
+EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canvas_free", "spade_canvas_info", "spade_join_count",
+                    "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_knn_histogram",
+                    "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_launch_count",
                     "spade_status_string", "spade_last_error"]
 
 
@@ -120,11 +135,15 @@ def launch_count() -> int:
 
 
 class Canvas:
-    """Discrete canvas + boundary index of a polygon set (owns device memory)."""
+    """Discrete canvas + boundary index of a polygon set (owns device memory).
+    ``Canvas.disks(...)`` builds a distance canvas (one closed disk per constraint) instead."""
 
     def __init__(self, polys, log2_pixel: int = -1, max_dim: int = 4096, dense: bool = False, stream=None):
         torch = _torch()
         lib = load()
+        if polys is None:                    # filled in by Canvas.disks
+            self._h, self._lib, self.num_polys = None, lib, 0
+            return
         ring_xy = _dev(polys["ring_xy"], torch.int32, 2)
         ring_off = _dev(polys["ring_off"], torch.int64)
         poly_ring_off = _dev(polys["poly_ring_off"], torch.int64)
@@ -137,6 +156,29 @@ class Canvas:
         _check(rc, "spade_build_canvas")
         self._h = h
         self._lib = lib
+
+    @classmethod
+    def disks(cls, center_xy, r2, log2_pixel: int = -1, max_dim: int = 4096, dense: bool = False, stream=None):
+        """Distance canvas (spade_build_disk_canvas): disk d = {p : |p - center_d|^2 <= r2[d]}.
+        ``r2`` may be a scalar (type 1 distance join, one radius) or one int64 per disk (type 2)."""
+        torch = _torch()
+        cxy = _dev(center_xy, torch.int32, 2)
+        D = int(cxy.shape[0])
+        r2t = torch.as_tensor(r2, dtype=torch.int64)
+        if r2t.numel() == 1 and D != 1:
+            r2t = r2t.reshape(1).expand(D)
+        r2t = r2t.to("cuda").contiguous()
+        if r2t.numel() != D:
+            raise ValueError("r2 must be a scalar or have one entry per disk")
+        self = cls(None)
+        prm = CanvasParams(log2_pixel, max_dim, SPADE_CANVAS_DENSE if dense else 0)
+        h = ctypes.c_void_p()
+        rc = self._lib.spade_build_disk_canvas(ctypes.c_void_p(cxy.data_ptr()), ctypes.c_void_p(r2t.data_ptr()), D,
+                                               ctypes.byref(prm), _stream(stream), ctypes.byref(h))
+        _check(rc, "spade_build_disk_canvas")
+        self._h = h
+        self.num_polys = D
+        return self
 
     @property
     def handle(self):
@@ -243,3 +285,76 @@ def join_count_host(canvas: Canvas, xy_host, counts_host=None, stream=None) -> n
                                    counts_host.ctypes.data_as(ctypes.c_void_p), _stream(stream))
     _check(rc, "spade_join_count_host")
     return counts_host
+
+
+# ---- kNN selection (spade_knn*): circles -> aggregation -> distance select -> sort ----
+KNN_BINS = 248
+
+
+def knn_histogram(xy, q, hist=None, stream=None):
+    """Step 1: int64[KNN_BINS + 1] CUDA tensor of squared-distance bucket counts (accumulated
+    into `hist` if given); the last entry counts points outside [-2^30, 2^30)."""
+    torch = _torch()
+    xy, n = _points(xy)
+    if hist is None:
+        hist = torch.zeros(KNN_BINS + 1, dtype=torch.int64, device="cuda")
+    _check(load().spade_knn_histogram(ctypes.c_void_p(xy.data_ptr()), n, int(q[0]), int(q[1]),
+                                      ctypes.c_void_p(hist.data_ptr()), _stream(stream)), "spade_knn_histogram")
+    return hist
+
+
+def knn_radius(hist_host, k: int):
+    """(r2, count): the smallest circle holding >= k points, from a host histogram."""
+    h = np.ascontiguousarray(np.asarray(hist_host, dtype=np.int64))
+    r2, cnt = ctypes.c_int64(), ctypes.c_int64()
+    _check(load().spade_knn_radius(h.ctypes.data_as(ctypes.c_void_p), int(k), ctypes.byref(r2), ctypes.byref(cnt)),
+           "spade_knn_radius")
+    return r2.value, cnt.value
+
+
+def knn_select(xy, q, r2: int, point_id_base: int = 0, capacity: int | None = None, stream=None):
+    """Step 2: (ids, d2) int64 CUDA tensors of the points with dist2 <= r2 (order unspecified)."""
+    torch = _torch()
+    xy, n = _points(xy)
+    cap = n if capacity is None else capacity
+    for _ in range(2):
+        ids = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+        d2 = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+        n_out = ctypes.c_int64()
+        rc = load().spade_knn_select(ctypes.c_void_p(xy.data_ptr()), n, point_id_base, int(q[0]), int(q[1]), int(r2),
+                                     ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(d2.data_ptr()), cap,
+                                     ctypes.byref(n_out), _stream(stream))
+        if rc == SPADE_ERR_CAPACITY:
+            cap = n_out.value
+            continue
+        _check(rc, "spade_knn_select")
+        return ids[: n_out.value], d2[: n_out.value]
+    raise SpadeError(SPADE_ERR_CAPACITY, "knn_select: capacity retry failed")
+
+
+def knn_topk(ids, d2, k: int, stream=None):
+    """Step 3: the first min(k, m) candidates in (d2, id) order, as (ids, d2) CUDA tensors."""
+    torch = _torch()
+    ids = ids.contiguous(); d2 = d2.contiguous()
+    m = ids.numel()
+    kk = min(int(k), m)
+    oi = torch.empty(max(kk, 1), dtype=torch.int64, device="cuda")
+    od = torch.empty(max(kk, 1), dtype=torch.int64, device="cuda")
+    _check(load().spade_knn_topk(ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(d2.data_ptr()), m, int(k),
+                                 ctypes.c_void_p(oi.data_ptr()), ctypes.c_void_p(od.data_ptr()), _stream(stream)),
+           "spade_knn_topk")
+    return oi[:kk], od[:kk]
+
+
+def knn(xy, q, k: int, point_id_base: int = 0, stream=None):
+    """The min(k, n) points nearest to q = (qx, qy), ties by id: (ids, d2) int64 CUDA tensors in
+    (d2, id) order (spade_knn: all three steps on this device)."""
+    torch = _torch()
+    xy, n = _points(xy)
+    ids = torch.empty(max(int(k), 1), dtype=torch.int64, device="cuda")
+    d2 = torch.empty(max(int(k), 1), dtype=torch.int64, device="cuda")
+    n_out = ctypes.c_int64()
+    _check(load().spade_knn(ctypes.c_void_p(xy.data_ptr()), n, point_id_base, int(q[0]), int(q[1]), int(k),
+                            ctypes.c_void_p(ids.data_ptr()), ctypes.c_void_p(d2.data_ptr()), ctypes.byref(n_out),
+                            _stream(stream)), "spade_knn")
+    return ids[: n_out.value], d2[: n_out.value]

@@ -8,7 +8,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libspade.so")
-SOURCES = ["spade_api.cu", "canvas_build.cu", "probe.cu"]
+SOURCES = ["spade_api.cu", "canvas_build.cu", "probe.cu", "knn.cu"]
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
               "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-Xptxas", "-v"]
 
@@ -22,7 +22,7 @@ def _stale(target, deps):
 
 def build(force: bool = False, verbose: bool = False) -> str:
     srcs = [os.path.join(CSRC, s) for s in SOURCES]
-    deps = srcs + [os.path.join(CSRC, "spade_internal.cuh"), os.path.join(ROOT, "include", "spade.h")]
+    deps = srcs + [os.path.abspath(__file__), os.path.join(CSRC, "spade_internal.cuh"), os.path.join(ROOT, "include", "spade.h")]
     if not force and not _stale(LIB, deps):
         return LIB
     objs = []

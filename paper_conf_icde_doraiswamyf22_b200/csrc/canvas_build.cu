@@ -161,6 +161,114 @@ __global__ void k_emit(const int4* __restrict__ seg, const int32_t* __restrict__
   }
 }
 
+// ---- distance canvases: disks (cx, cy, r2) -----------------------------------------
+// A pixel holds the integer points [X, X+S-1] x [Y0, Y0+S-1].  For the closed disk
+// (x-cx)^2 + (y-cy)^2 <= r2 the pixel is INSIDE when all its integer points are in the disk,
+// TOUCHED when at least one is, and a boundary pixel when touched but not inside.  Per row both
+// sets are column intervals (the disk's slice at height y is [cx - hw(y), cx + hw(y)],
+// hw(y) = isqrt(r2 - (y-cy)^2), widest at the y closest to cy and narrowest at the farthest), so a
+// disk contributes per row: boundary fragments left and right of the inside interval, and one
+// pair of fill events bounding it.  Exact integer arithmetic throughout (r2 < 2^62).
+
+__host__ __device__ __forceinline__ int64_t isqrt64(int64_t v) {   // floor(sqrt(v)), 0 <= v < 2^62
+  int64_t r = (int64_t)sqrt((double)v);
+  while (r > 0 && r * r > v) --r;
+  while ((r + 1) * (r + 1) <= v) ++r;
+  return r;
+}
+
+// K-D0: disks -> (cx, cy, r2 lo, r2 hi) "edges", range check, extent of their integer points.
+// bad: 1 = r2 outside [0, 2^62), 2 = a disk reaches outside [-2^30, 2^30)
+__global__ void k_disks(const int2* __restrict__ cxy, const int64_t* __restrict__ r2v, int32_t D,
+                        int4* __restrict__ seg, int32_t* __restrict__ poly, int* __restrict__ ext,
+                        int* __restrict__ bad) {
+  using BR = cub::BlockReduce<int, kBT>;
+  __shared__ typename BR::TempStorage tmp;
+  int mnx = INT_MAX, mny = INT_MAX, mxx = INT_MIN, mxy = INT_MIN, b = 0;
+  for (int64_t k = blockIdx.x * (int64_t)kBT + threadIdx.x; k < D; k += (int64_t)gridDim.x * kBT) {
+    const int2 c = cxy[k];
+    const int64_t r2 = r2v[k];
+    const int64_t lim = 1ll << 30;
+    if (r2 < 0 || r2 >= (1ll << 62)) { b = max(b, 1); continue; }
+    const int64_t R = isqrt64(r2);
+    if (c.x - R < -lim || c.x + R >= lim || c.y - R < -lim || c.y + R >= lim) { b = 2; continue; }
+    seg[k] = make_int4(c.x, c.y, (int)(uint32_t)(uint64_t)r2, (int)(uint32_t)((uint64_t)r2 >> 32));
+    poly[k] = (int32_t)k;
+    mnx = min(mnx, (int)(c.x - R)); mny = min(mny, (int)(c.y - R));
+    mxx = max(mxx, (int)(c.x + R)); mxy = max(mxy, (int)(c.y + R));
+  }
+  int r0 = BR(tmp).Reduce(mnx, cub::Min()); __syncthreads();
+  int r1 = BR(tmp).Reduce(mny, cub::Min()); __syncthreads();
+  int r2 = BR(tmp).Reduce(mxx, cub::Max()); __syncthreads();
+  int r3 = BR(tmp).Reduce(mxy, cub::Max()); __syncthreads();
+  int r4 = BR(tmp).Reduce(b, cub::Max());
+  if (threadIdx.x == 0) {
+    atomicMin(&ext[0], r0); atomicMin(&ext[1], r1); atomicMax(&ext[2], r2); atomicMax(&ext[3], r3);
+    if (r4) atomicMax(bad, r4);
+  }
+}
+
+__device__ __forceinline__ void disk_rows(int4 e, const Geo& g, int64_t R, int64_t& jlo, int64_t& jhi) {
+  jlo = imax64(floor_div((int64_t)e.y - R - g.miny, g.S), 0);
+  jhi = imin64(floor_div((int64_t)e.y + R - g.miny, g.S), g.H - 1);
+}
+
+// row j of disk e: touched columns [t0, t1], inside columns [i0, i1] (empty: i0 > i1)
+__device__ __forceinline__ void disk_row(int4 e, const Geo& g, int64_t R, int64_t j, int64_t& t0, int64_t& t1,
+                                         int64_t& i0, int64_t& i1) {
+  const int64_t cx = e.x, cy = e.y, r2 = disk_r2(e);
+  const int64_t Y0 = g.miny + j * g.S, Y1 = Y0 + g.S - 1;
+  const int64_t ya = imax64(Y0, cy - R), yb = imin64(Y1, cy + R);
+  const int64_t dymin = (ya <= cy && cy <= yb) ? 0 : imin64(ya > cy ? ya - cy : cy - ya, yb > cy ? yb - cy : cy - yb);
+  const int64_t hw = isqrt64(r2 - dymin * dymin);
+  t0 = imax64(floor_div(cx - hw - g.minx, g.S), 0);
+  t1 = imin64(floor_div(cx + hw - g.minx, g.S), g.W - 1);
+  const int64_t dymax = imax64(Y0 > cy ? Y0 - cy : cy - Y0, Y1 > cy ? Y1 - cy : cy - Y1);
+  i0 = 1; i1 = 0;
+  if (dymax <= R) {
+    const int64_t hm = isqrt64(r2 - dymax * dymax);
+    i0 = imax64(ceil_div(cx - hm - g.minx, g.S), t0);
+    i1 = imin64(floor_div(cx + hm - g.minx - g.S + 1, g.S), t1);
+  }
+}
+
+// two fragments and two fill events per (disk, row)
+__global__ void k_dcount(const int4* __restrict__ seg, int64_t E, Geo g, int64_t* __restrict__ nfrag,
+                         int64_t* __restrict__ nev) {
+  for (int64_t k = blockIdx.x * (int64_t)kBT + threadIdx.x; k < E; k += (int64_t)gridDim.x * kBT) {
+    const int4 e = seg[k];
+    int64_t a, b;
+    disk_rows(e, g, isqrt64(disk_r2(e)), a, b);
+    nfrag[k] = b >= a ? 2 * (b - a + 1) : 0;
+    nev[k] = nfrag[k];
+  }
+}
+
+__global__ void k_demit(const int4* __restrict__ seg, int64_t E, Geo g, const int64_t* __restrict__ frag_off,
+                        const int64_t* __restrict__ ev_off, Frag* __restrict__ frags, int64_t* __restrict__ frag_w,
+                        uint64_t* __restrict__ ev_keys, int pbits, int kbits) {
+  for (int64_t k = blockIdx.x * (int64_t)kBT + threadIdx.x; k < E; k += (int64_t)gridDim.x * kBT) {
+    const int4 e = seg[k];
+    const int64_t R = isqrt64(disk_r2(e));
+    int64_t a, b;
+    disk_rows(e, g, R, a, b);
+    int64_t o = frag_off[k], q = ev_off[k];
+    for (int64_t j = a; j <= b; ++j, o += 2, q += 2) {
+      int64_t t0, t1, i0, i1;
+      disk_row(e, g, R, j, t0, t1, i0, i1);
+      int64_t l0 = t0, l1 = t1, r0 = 0, r1 = -1, k0 = 0, k1 = 0;   // boundary [l0,l1] u [r0,r1]
+      if (i0 <= i1) { l1 = i0 - 1; r0 = i1 + 1; r1 = t1; k0 = 2 * i0; k1 = 2 * (i1 + 1); }
+      frags[o] = Frag{(int32_t)j, (int32_t)l0, (int32_t)l1, (int32_t)k};
+      frag_w[o] = l1 >= l0 ? l1 - l0 + 1 : 0;
+      frags[o + 1] = Frag{(int32_t)j, (int32_t)r0, (int32_t)r1, (int32_t)k};
+      frag_w[o + 1] = r1 >= r0 ? r1 - r0 + 1 : 0;
+      const uint64_t hk = ((uint64_t)j << (pbits + kbits)) | ((uint64_t)k << kbits);
+      ev_keys[q] = hk | (uint64_t)k0;                   // empty interior: [0, 0) fills nothing
+      ev_keys[q + 1] = hk | (uint64_t)k1;
+    }
+  }
+}
+
 __global__ void k_mark(const Frag* __restrict__ frags, int64_t F, int W, int32_t* __restrict__ bflag) {
   for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < F; t += (int64_t)gridDim.x * kBT) {
     Frag f = frags[t];
@@ -232,8 +340,10 @@ __device__ __forceinline__ uint32_t seg_hash(int4 e) {
   h ^= h >> 29; h *= 0xBF58476D1CE4E5B9ull; h ^= h >> 32;
   return (uint32_t)h;
 }
-__device__ __forceinline__ bool same_seg(int4 a, int4 b) {
-  return (a.x == b.x && a.y == b.y && a.z == b.z && a.w == b.w) || (a.x == b.z && a.y == b.w && a.z == b.x && a.w == b.y);
+// equal primitives: a polygon edge in either orientation; a disk exactly
+__device__ __forceinline__ bool same_seg(int4 a, int4 b, int kind) {
+  return (a.x == b.x && a.y == b.y && a.z == b.z && a.w == b.w) ||
+         (kind == kPolygons && a.x == b.z && a.y == b.w && a.z == b.x && a.w == b.y);
 }
 
 // per entry (sorted by (bid, poly)): local polygon index and the (bid, segment hash) key
@@ -256,7 +366,7 @@ __global__ void k_merge(const uint64_t* __restrict__ key2, const int32_t* __rest
                         const int32_t* __restrict__ ev, const int32_t* __restrict__ li, const int4* __restrict__ seg,
                         const int32_t* __restrict__ pcnt, const int64_t* __restrict__ le_beg, int32_t* __restrict__ mcnt,
                         const int64_t* __restrict__ mbeg, int32_t* __restrict__ mfill,
-                        int4* __restrict__ oseg, uint64_t* __restrict__ omask) {
+                        int4* __restrict__ oseg, uint64_t* __restrict__ omask, int kind) {
   for (int64_t u = blockIdx.x * (int64_t)kBT + threadIdx.x; u < L; u += (int64_t)gridDim.x * kBT) {
     const uint64_t k = key2[u];
     const uint32_t bid = (uint32_t)(k >> 32);
@@ -268,11 +378,11 @@ __global__ void k_merge(const uint64_t* __restrict__ key2, const int32_t* __rest
     } else {
       bool first = true;
       for (int64_t w = u - 1; w >= 0 && key2[w] == k; --w)
-        if (same_seg(seg[ev[tix[w]]], e)) { first = false; break; }
+        if (same_seg(seg[ev[tix[w]]], e, kind)) { first = false; break; }
       if (!first) continue;
       m = 1ull << li[tix[u]];
       for (int64_t w = u + 1; w < L && key2[w] == k; ++w)
-        if (same_seg(seg[ev[tix[w]]], e)) m ^= 1ull << li[tix[w]];
+        if (same_seg(seg[ev[tix[w]]], e, kind)) m ^= 1ull << li[tix[w]];
       if (m == 0) continue;
     }
     if (PASS == 0) {
@@ -355,7 +465,7 @@ __global__ void k_kset(int64_t NB, const int64_t* __restrict__ pix_of, Geo g, co
                        const int32_t* __restrict__ pbeg, const int32_t* __restrict__ pcnt,
                        const int32_t* __restrict__ rec_polys,
                        int32_t* __restrict__ ksize, const int64_t* __restrict__ koff, int32_t* __restrict__ kout,
-                       RunRec* __restrict__ recs) {
+                       RunRec* __restrict__ recs, int kind) {
   for (int64_t b = blockIdx.x * (int64_t)kBT + threadIdx.x; b < NB; b += (int64_t)gridDim.x * kBT) {
     const int64_t p = pix_of[b];
     const int64_t i = p % g.W, j = p / g.W;
@@ -383,7 +493,8 @@ __global__ void k_kset(int64_t NB, const int64_t* __restrict__ pix_of, Geo g, co
     };
     if (pc <= kMaskPolys) {
       uint64_t m = 0;
-      for (int64_t e = e0; e < e1; ++e) if (cu_test(rseg[e], X, Y0)) m ^= rmask[e];
+      if (kind == kPolygons)
+        for (int64_t e = e0; e < e1; ++e) if (cu_test(rseg[e], X, Y0)) m ^= rmask[e];
       for (int k = 0; k < pc; ++k) {
         const int par = (int)((m >> k) & 1u);
         const int32_t P = rec_polys[pb + k];
@@ -392,7 +503,8 @@ __global__ void k_kset(int64_t NB, const int64_t* __restrict__ pix_of, Geo g, co
     } else {
       for (int k = 0; k < pc; ++k) {
         int par = 0;
-        for (int64_t e = e0; e < e1; ++e) if ((int)rmask[e] == k) par ^= cu_test(rseg[e], X, Y0);
+        if (kind == kPolygons)
+          for (int64_t e = e0; e < e1; ++e) if ((int)rmask[e] == k) par ^= cu_test(rseg[e], X, Y0);
         merge_upto(rec_polys[pb + k], par);
       }
     }
@@ -521,49 +633,59 @@ cudaError_t cub_call(DevBufs& bufs, F f) {
 
 }  // namespace
 
-int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off, int32_t P,
-                 const spade_canvas_params* prm, cudaStream_t st, spade_canvas** out) {
+// One builder for both canvas kinds: the front end (K-B0/K-B1 for polygon edges, K-D0/K-D1 for
+// disks) produces primitives, boundary fragments and fill events; everything after is shared.
+static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off,
+                     const int32_t* center_xy, const int64_t* r2, int32_t P, const spade_canvas_params* prm,
+                     cudaStream_t st, spade_canvas** out) {
   *out = nullptr;
-  if (P < 0 || (P > 0 && (!ring_off || !poly_ring_off)))
-    return set_error(SPADE_ERR_INVALID_ARG, "spade_build_canvas: bad polygon arguments");
-  if (P > (1 << 30)) return set_error(SPADE_ERR_INVALID_ARG, "spade_build_canvas: too many polygons");
+  const char* fn = kind == kDisks ? "spade_build_disk_canvas" : "spade_build_canvas";
+  if (P < 0 || (kind == kPolygons && P > 0 && (!ring_off || !poly_ring_off)) || (kind == kDisks && P > 0 && (!center_xy || !r2)))
+    return set_error(SPADE_ERR_INVALID_ARG, "%s: bad arguments", fn);
+  if (P > (1 << 30)) return set_error(SPADE_ERR_INVALID_ARG, "%s: too many primitives", fn);
   int max_dim = 4096, forced_s = -1;
   if (prm) {
     if (prm->max_dim < 0 || prm->log2_pixel < -1 || prm->log2_pixel > 30)
-      return set_error(SPADE_ERR_INVALID_ARG, "spade_build_canvas: bad canvas params");
+      return set_error(SPADE_ERR_INVALID_ARG, "%s: bad canvas params", fn);
     if (prm->max_dim > 0) max_dim = prm->max_dim;
     forced_s = prm->log2_pixel;
   }
   if (max_dim < 1 || max_dim > 65536) return set_error(SPADE_ERR_INVALID_ARG, "max_dim out of [1, 65536]");
 
-  // --- offsets to the host for validation (R+1 and P+1 int64s) ---
-  std::vector<int64_t> h_pro(P + 1, 0);
   cudaError_t ce;
-  if (P > 0 && (ce = cudaMemcpyAsync(h_pro.data(), poly_ring_off, sizeof(int64_t) * (P + 1), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
-    return check_cuda(ce, "copy poly_ring_off");
-  if ((ce = cudaStreamSynchronize(st)) != cudaSuccess) return check_cuda(ce, "sync");
-  int64_t R = h_pro[P];
-  if (h_pro[0] != 0 || R < 0) return set_error(SPADE_ERR_INVALID_ARG, "poly_ring_off must start at 0");
-  for (int32_t p = 0; p < P; ++p)
-    if (h_pro[p + 1] < h_pro[p]) return set_error(SPADE_ERR_INVALID_ARG, "poly_ring_off not non-decreasing at %d", p);
-  std::vector<int64_t> h_ro(R + 1, 0);
-  if (R > 0) {
-    if ((ce = cudaMemcpyAsync(h_ro.data(), ring_off, sizeof(int64_t) * (R + 1), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
-      return check_cuda(ce, "copy ring_off");
+  int64_t V = 0, R = 0;        // V = number of primitives (polygon edges / disks)
+  if (kind == kPolygons) {
+    // --- offsets to the host for validation (R+1 and P+1 int64s) ---
+    std::vector<int64_t> h_pro(P + 1, 0);
+    if (P > 0 && (ce = cudaMemcpyAsync(h_pro.data(), poly_ring_off, sizeof(int64_t) * (P + 1), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+      return check_cuda(ce, "copy poly_ring_off");
     if ((ce = cudaStreamSynchronize(st)) != cudaSuccess) return check_cuda(ce, "sync");
+    R = h_pro[P];
+    if (h_pro[0] != 0 || R < 0) return set_error(SPADE_ERR_INVALID_ARG, "poly_ring_off must start at 0");
+    for (int32_t p = 0; p < P; ++p)
+      if (h_pro[p + 1] < h_pro[p]) return set_error(SPADE_ERR_INVALID_ARG, "poly_ring_off not non-decreasing at %d", p);
+    std::vector<int64_t> h_ro(R + 1, 0);
+    if (R > 0) {
+      if ((ce = cudaMemcpyAsync(h_ro.data(), ring_off, sizeof(int64_t) * (R + 1), cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+        return check_cuda(ce, "copy ring_off");
+      if ((ce = cudaStreamSynchronize(st)) != cudaSuccess) return check_cuda(ce, "sync");
+    }
+    V = h_ro[R];
+    if (h_ro[0] != 0 || V < 0) return set_error(SPADE_ERR_INVALID_ARG, "ring_off must start at 0");
+    for (int64_t r = 0; r < R; ++r)
+      if (h_ro[r + 1] < h_ro[r]) return set_error(SPADE_ERR_INVALID_ARG, "ring_off not non-decreasing at %lld", (long long)r);
+    if (V > 0 && !ring_xy) return set_error(SPADE_ERR_INVALID_ARG, "ring_xy is NULL");
+    if (V >= (1ll << 31)) return set_error(SPADE_ERR_INVALID_ARG, "too many vertices");
+  } else {
+    V = P;
   }
-  int64_t V = h_ro[R];
-  if (h_ro[0] != 0 || V < 0) return set_error(SPADE_ERR_INVALID_ARG, "ring_off must start at 0");
-  for (int64_t r = 0; r < R; ++r)
-    if (h_ro[r + 1] < h_ro[r]) return set_error(SPADE_ERR_INVALID_ARG, "ring_off not non-decreasing at %lld", (long long)r);
-  if (V > 0 && !ring_xy) return set_error(SPADE_ERR_INVALID_ARG, "ring_xy is NULL");
-  if (V >= (1ll << 31)) return set_error(SPADE_ERR_INVALID_ARG, "too many vertices");
 
   spade_canvas* c = new spade_canvas();
   cudaGetDevice(&c->device);
   c->d.num_polys = P;
+  c->d.kind = kind;
   auto fail = [&](int code) { spade_canvas_free(c); return code; };
-  if (V == 0) {  // no vertices: every point is outside every polygon
+  if (V == 0) {  // no primitives: every point is outside everything
     c->empty = true;
     *out = c;
     return SPADE_OK;
@@ -578,12 +700,15 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   int h_ext0[4] = {INT_MAX, INT_MAX, INT_MIN, INT_MIN};
   TRYF(cudaMemcpyAsync(ext, h_ext0, sizeof(h_ext0), cudaMemcpyHostToDevice, st), "ext init");
   TRYF(cudaMemsetAsync(bad, 0, sizeof(int), st), "memset");
-  LAUNCH(k_edges, V, (const int2*)ring_xy, ring_off, R, poly_ring_off, P, V, seg, epoly, ext, bad);
+  if (kind == kPolygons) LAUNCH(k_edges, V, (const int2*)ring_xy, ring_off, R, poly_ring_off, P, V, seg, epoly, ext, bad);
+  else LAUNCH(k_disks, V, (const int2*)center_xy, r2, P, seg, epoly, ext, bad);
   int h_ext[4], h_bad = 0;
   TRYF(cudaMemcpyAsync(h_ext, ext, sizeof(h_ext), cudaMemcpyDeviceToHost, st), "ext");
   TRYF(cudaMemcpyAsync(&h_bad, bad, sizeof(int), cudaMemcpyDeviceToHost, st), "bad");
   TRYF(cudaStreamSynchronize(st), "sync edges");
-  if (h_bad) return fail(set_error(SPADE_ERR_COORD_RANGE, "a polygon vertex lies outside [-2^30, 2^30)"));
+  if (kind == kPolygons && h_bad) return fail(set_error(SPADE_ERR_COORD_RANGE, "a polygon vertex lies outside [-2^30, 2^30)"));
+  if (kind == kDisks && h_bad == 1) return fail(set_error(SPADE_ERR_INVALID_ARG, "a squared radius lies outside [0, 2^62)"));
+  if (kind == kDisks && h_bad) return fail(set_error(SPADE_ERR_COORD_RANGE, "a disk reaches outside [-2^30, 2^30)"));
 
   // --- canvas geometry (reading C5) ---
   int64_t ew = (int64_t)h_ext[2] - h_ext[0], eh = (int64_t)h_ext[3] - h_ext[1];
@@ -617,7 +742,8 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   // --- K-B1 counts, scans, emit ---
   int64_t *nfrag, *nev, *frag_off, *ev_off;
   ALLOC(nfrag, V, "counts"); ALLOC(nev, V, "counts"); ALLOC(frag_off, V + 1, "counts"); ALLOC(ev_off, V + 1, "counts");
-  LAUNCH(k_count, V, seg, V, g, nfrag, nev);
+  if (kind == kPolygons) LAUNCH(k_count, V, seg, V, g, nfrag, nev);
+  else LAUNCH(k_dcount, V, seg, V, g, nfrag, nev);
   for (auto pr : {std::make_pair(nfrag, frag_off), std::make_pair(nev, ev_off)}) {
     int64_t* in = pr.first; int64_t* o = pr.second;
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, in, o + 1, V, st); }), "scan counts");
@@ -634,7 +760,8 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
 
   Frag* frags; int64_t* frag_w; uint64_t* ev;
   ALLOC(frags, F, "fragments"); ALLOC(frag_w, F + 1, "fragments"); ALLOC(ev, NE, "events");
-  LAUNCH(k_emit, V, seg, epoly, V, g, frag_off, ev_off, frags, frag_w, ev, pbits, kbits);
+  if (kind == kPolygons) LAUNCH(k_emit, V, seg, epoly, V, g, frag_off, ev_off, frags, frag_w, ev, pbits, kbits);
+  else LAUNCH(k_demit, V, seg, V, g, frag_off, ev_off, frags, frag_w, ev, pbits, kbits);
 
   // --- K-B2 boundary pixels, ids, pixel-local edge lists ---
   int32_t *bflag, *bscan;
@@ -690,7 +817,7 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
     LAUNCH(k_segkey, L, lk2, lv2, L, seg, pg, pbeg, lk, li);            // lk reused for (bid, hash) keys
     LAUNCH(k_iota, L, tix, L);
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortPairs(t, sz, lk, key2s, tix, tix2, L, 0, 32 + bbits, st); }), "sort segments");
-    LAUNCH(k_merge<0>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, nullptr, nullptr, nullptr, nullptr);
+    LAUNCH(k_merge<0>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, nullptr, nullptr, nullptr, nullptr, kind);
   }
   if (NB > 0) {
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, mcnt, mbeg, NB, st); }), "scan merged");
@@ -703,7 +830,7 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   if (cudaMalloc(&c->run_seg, sizeof(int4) * std::max<int64_t>(LM, 1)) != cudaSuccess ||
       cudaMalloc(&c->run_mask, sizeof(uint64_t) * std::max<int64_t>(LM, 1)) != cudaSuccess)
     return fail(set_error(SPADE_ERR_OOM, "build: local edge arrays"));
-  if (L > 0) LAUNCH(k_merge<1>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, mbeg, mfill, c->run_seg, c->run_mask);
+  if (L > 0) LAUNCH(k_merge<1>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, mbeg, mfill, c->run_seg, c->run_mask, kind);
   tmp.release(lk); tmp.release(lk2); tmp.release(lv); tmp.release(lv2); tmp.release(frags); tmp.release(lw_off);
   tmp.release(ph); tmp.release(pg); tmp.release(li); tmp.release(tix); tmp.release(tix2); tmp.release(key2s);
 
@@ -758,7 +885,7 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   int64_t KT = 0; int64_t NK = 0;
   if (NB > 0) {
     LAUNCH(k_kset<0>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, c->run_seg, c->run_mask,
-           pbeg, pcnt, c->rec_polys, ksize, nullptr, nullptr, nullptr);
+           pbeg, pcnt, c->rec_polys, ksize, nullptr, nullptr, nullptr, kind);
     cub::TransformInputIterator<int64_t, BigSize, const int32_t*> it_sz(ksize, BigSize());
     cub::TransformInputIterator<int32_t, BigFlag, const int32_t*> it_b(ksize, BigFlag());
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, it_sz, koff, NB, st); }), "scan K");
@@ -783,7 +910,7 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   }
   if (NB > 0) {
     LAUNCH(k_kset<1>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, c->run_seg, c->run_mask,
-           pbeg, pcnt, c->rec_polys, ksize, koff, c->sets + M, c->runs);
+           pbeg, pcnt, c->rec_polys, ksize, koff, c->sets + M, c->runs, kind);
     LAUNCH(k_kset_rng, NB, NB, ksize, koff, kidx, NG, M, c->set_rng, c->runs);
   }
   if (NG > 0) LAUNCH(k_multi_recs, NG, NG, NB, c->runs);
@@ -837,6 +964,16 @@ int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t*
   if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));
   *out = c;
   return SPADE_OK;
+}
+
+int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off, int32_t P,
+                 const spade_canvas_params* prm, cudaStream_t st, spade_canvas** out) {
+  return build_any(kPolygons, ring_xy, ring_off, poly_ring_off, nullptr, nullptr, P, prm, st, out);
+}
+
+int build_disk_canvas(const int32_t* center_xy, const int64_t* r2, int32_t D, const spade_canvas_params* prm,
+                      cudaStream_t st, spade_canvas** out) {
+  return build_any(kDisks, nullptr, nullptr, nullptr, center_xy, r2, D, prm, st, out);
 }
 
 }  // namespace spade

@@ -151,11 +151,19 @@ __device__ __forceinline__ int local_bit(int4 e, int X, int px, int py) {
   return (int)(crX ^ crP ^ cuX);
 }
 
-// Exact point-in-polygon for a point on boundary pixel (or multi-owner pixel) record `rec`:
-//   inside(p, P) = [P in K] XOR parity_P(local_bit over P's edges touching the pixel),
-// the parities of all (<= 64) polygons of the pixel accumulated at once as a bit mask
+// Exact test for a point on boundary pixel (or multi-owner pixel) record `rec`:
+//   inside(p, P) = [P in K] XOR parity_P(hit over P's primitives touching the pixel),
+// the parities of all (<= 64) polygons of the pixel accumulated at once as a bit mask.  A
+// primitive's hit: polygon edge -> local_bit (edges that straddle neither y = py nor x = X
+// contribute nothing and skip the cross products); disk (KIND == kDisks) ->
+// (px-cx)^2 + (py-cy)^2 <= r2 (|px-cx|, |py-cy| < 2^31 for a point on a pixel the disk touches).
 // emit(P) is called for every polygon containing the point, in increasing polygon order.
-template <class Emit>
+__device__ __forceinline__ bool disk_hit(int4 g, int px, int py) {
+  const long long dx = (long long)px - g.x, dy = (long long)py - g.y;
+  return (unsigned long long)(dx * dx) + (unsigned long long)(dy * dy) <= (unsigned long long)disk_r2(g);
+}
+
+template <int KIND, class Emit>
 __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
   const RunRec r = cv->runs[rec];
   const int X = cv->minx + (int)((((uint32_t)px - (uint32_t)cv->minx) >> cv->s) << cv->s);
@@ -177,10 +185,14 @@ __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int p
   const int32_t* rp = cv->rec_polys + r.poly_begin;
   const int64_t e1 = r.edge_begin + r.edge_cnt;
   if (r.poly_cnt <= kMaskPolys) {
-    // each de-duplicated edge toggles the parity of every polygon that uses it
+    // each de-duplicated primitive toggles the parity of every polygon that uses it
     uint64_t m = 0;
     for (int64_t e = r.edge_begin; e < e1; ++e) {
       const int4 g = __ldg(seg + e);
+      if (KIND == kDisks) {
+        if (disk_hit(g, px, py)) m ^= __ldg(msk + e);
+        continue;
+      }
       // an edge that straddles neither the horizontal line y = py nor the vertical line x = X
       // contributes nothing (cr and cu are both 0): skip it without the cross product or its mask
       if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
@@ -192,12 +204,16 @@ __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int p
       finalize(__ldg(rp + k), 1);
     }
   } else {
-    // > kMaskPolys polygons: edges grouped by local polygon index (run_mask = index)
+    // > kMaskPolys polygons: primitives grouped by local polygon index (run_mask = index)
     int cur = -1, par = 0;
     for (int64_t e = r.edge_begin; e < e1; ++e) {
       const int4 g = __ldg(seg + e);
-      if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
-      if (!local_bit(g, X, px, py)) continue;
+      if (KIND == kDisks) {
+        if (!disk_hit(g, px, py)) continue;
+      } else {
+        if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
+        if (!local_bit(g, X, px, py)) continue;
+      }
       const int k = (int)__ldg(msk + e);
       if (k != cur) {
         if (cur >= 0 && par) finalize(__ldg(rp + cur), 1);
@@ -218,17 +234,17 @@ __device__ __forceinline__ void count_hit(unsigned int* hist, unsigned long long
 
 // Emission from the rare in-kernel paths (deferral region full, unaligned head/tail): per-lane
 // atomics.
-template <int MODE>
+template <int MODE, int KIND>
 __device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, const Out& o,
                                              int x, int y, uint32_t rec, int64_t pid) {
   if (MODE == kCountSmem || MODE == kCountGlobal) {
-    pip_eval(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, o.counts, p); });
+    pip_eval<KIND>(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, o.counts, p); });
   } else if (MODE == kSelect) {
     bool any = false;
-    pip_eval(cvg, x, y, rec, [&](int) { any = true; });
+    pip_eval<KIND>(cvg, x, y, rec, [&](int) { any = true; });
     if (any) put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, 0);
   } else {
-    pip_eval(cvg, x, y, rec, [&](int p) { put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, p); });
+    pip_eval<KIND>(cvg, x, y, rec, [&](int p) { put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, p); });
   }
 }
 
@@ -239,7 +255,7 @@ __device__ __forceinline__ void rare_emit_owner(unsigned int* hist, const Out& o
 }
 
 // One scalar point (unaligned head / tail): classify synchronously.
-template <int MODE>
+template <int MODE, int KIND>
 __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, unsigned int* hist,
                                           const Out& o, int x, int y, int64_t pid) {
   const CanvasDev cv = *cvg;
@@ -249,13 +265,13 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
   uint32_t c = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
   if (c >= cv.mix_min) c = classify_fine(*fine_ptr(cv, c, fx, fy));
   if (c == 0) return;
-  if (c & 0x80000000u) rare_emit_point<MODE>(cvg, hist, o, x, y, ~c, pid);
+  if (c & 0x80000000u) rare_emit_point<MODE, KIND>(cvg, hist, o, x, y, ~c, pid);
   else rare_emit_owner<MODE>(hist, o, (int)c - 1, pid);
 }
 
 // COUNT, in-loop variant: evaluate up to 32 queued boundary points (one per lane).  Out of line:
 // the streaming loop keeps a small register footprint.
-template <int MODE>
+template <int MODE, int KIND>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const QEntry* wq,
                                    int cnt, int lane, unsigned int* hist, unsigned long long* counts) {
   if (lane < cnt) {
@@ -264,13 +280,13 @@ __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint
     const uint32_t fx = ((uint32_t)e.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)e.y - (uint32_t)cv.miny) >> cv.s;
     const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
     const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
-    pip_eval(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, counts, q); });
+    pip_eval<KIND>(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, counts, q); });
   }
 }
 
 // SELECT/PAIRS, in-loop variant: the exact test of one queued boundary point (lane < cnt), by
 // its index into the launch's points: (number of results, first polygon).  Out of line.
-template <int MODE>
+template <int MODE, int KIND>
 __device__ __noinline__ uint2 drain_eval(const CanvasDev* __restrict__ cvg, const uint16_t* tiles,
                                          const int2* __restrict__ xy, uint32_t pidx) {
   const CanvasDev& cv = *cvg;
@@ -280,9 +296,9 @@ __device__ __noinline__ uint2 drain_eval(const CanvasDev* __restrict__ cvg, cons
   const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
   uint32_t n = 0, first = 0;
   if (MODE == kSelect) {
-    pip_eval(cvg, p.x, p.y, ~c, [&](int) { n = 1; });
+    pip_eval<KIND>(cvg, p.x, p.y, ~c, [&](int) { n = 1; });
   } else {
-    pip_eval(cvg, p.x, p.y, ~c, [&](int q) { if (n++ == 0) first = (uint32_t)q; });
+    pip_eval<KIND>(cvg, p.x, p.y, ~c, [&](int q) { if (n++ == 0) first = (uint32_t)q; });
   }
   return make_uint2(n, first);
 }
@@ -296,6 +312,7 @@ struct Slots {
 
 // A queued point with more than one result (overlapping polygons): evaluated again, results
 // written to slots k, k+1, ...  Out of line (rare).
+template <int KIND>
 __device__ __noinline__ void emit_multi(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const int2* __restrict__ xy,
                                         uint32_t pidx, const Out& o, Slots sl, uint32_t k) {
   const CanvasDev& cv = *cvg;
@@ -303,7 +320,7 @@ __device__ __noinline__ void emit_multi(const CanvasDev* __restrict__ cvg, const
   const uint32_t fx = ((uint32_t)p.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)p.y - (uint32_t)cv.miny) >> cv.s;
   const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
   const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
-  pip_eval(cvg, p.x, p.y, ~c, [&](int q) { put_result<kPairs>(o, sl.at(k++), o.id_base + pidx, q); });
+  pip_eval<KIND>(cvg, p.x, p.y, ~c, [&](int q) { put_result<kPairs>(o, sl.at(k++), o.id_base + pidx, q); });
 }
 
 // Per-CTA shared-memory layout (bytes, in order):
@@ -317,7 +334,7 @@ __host__ __device__ __forceinline__ size_t queue_bytes(int mode) {
 }
 __host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
 
-template <int MODE, int COMPACT, int QUEUE>
+template <int MODE, int COMPACT, int QUEUE, int KIND>
 __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
   const CanvasDev& cv = prm.cv;
@@ -350,11 +367,11 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     const int64_t ntail = prm.n - tail0;
     if (lane < prm.head) {
       const int2 p = prm.xy[lane];
-      scalar_point<MODE>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + lane);
+      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + lane);
     } else if (lane >= 4 && lane - 4 < ntail) {
       const int64_t i = tail0 + (lane - 4);
       const int2 p = prm.xy[i];
-      scalar_point<MODE>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + i);
+      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + i);
     }
   }
 
@@ -401,7 +418,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   auto drain_out = [&](const uint32_t* q, int cnt, uint32_t later_batches) {
     uint2 r = make_uint2(0u, 0u);
     const uint32_t pidx = lane < cnt ? q[lane] : 0u;
-    if (lane < cnt) r = drain_eval<MODE>(prm.cvg, tiles, prm.xy, pidx);
+    if (lane < cnt) r = drain_eval<MODE, KIND>(prm.cvg, tiles, prm.xy, pidx);
     uint32_t incl = r.x;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -413,7 +430,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     const Slots sl = reserve(wtot, later_batches);
     const uint32_t k = incl - r.x;
     if (r.x == 1) put_result<MODE>(prm.o, sl.at(k), prm.o.id_base + pidx, (int)r.y);
-    else if (MODE == kPairs && r.x > 1) emit_multi(prm.cvg, tiles, prm.xy, pidx, prm.o, sl, k);
+    else if (MODE == kPairs && r.x > 1) emit_multi<KIND>(prm.cvg, tiles, prm.xy, pidx, prm.o, sl, k);
   };
   // phases A + B of one batch: c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
   auto classify = [&](const Vec4 v) {
@@ -471,7 +488,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         if (qn >= 32) {
           do {
             if (MODE == kSelect || MODE == kPairs) drain_out(wqi + qn - 32, 32, (nvec - 1 - base) / (nctaid_x() * chunk));
-            else drain<MODE>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+            else drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
             qn -= 32;
           } while (qn >= 32);
           __syncwarp();
@@ -497,7 +514,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
             dreg[d] = DEntry{p.x, p.y, ~c[q], pidx};
           } else {
             if (d < prm.defer_cap) dreg[d] = DEntry{0, 0, kHole, 0u};
-            rare_emit_point<MODE>(prm.cvg, myhist, prm.o, p.x, p.y, ~c[q], prm.o.id_base + pidx);
+            rare_emit_point<MODE, KIND>(prm.cvg, myhist, prm.o, p.x, p.y, ~c[q], prm.o.id_base + pidx);
           }
           ++d;
         }
@@ -596,7 +613,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
           int qn = s_qn[warp];
           if (qn >= 32) {
             do {
-              drain<MODE>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+              drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
               qn -= 32;
             } while (qn >= 32);
             __syncwarp();
@@ -633,7 +650,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   }
   if (QUEUE && (MODE == kCountSmem || MODE == kCountGlobal)) {
     __syncwarp();
-    if (s_qn[warp] > 0) drain<MODE>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.o.counts);
+    if (s_qn[warp] > 0) drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.o.counts);
   }
   __syncthreads();
   if (!QUEUE && tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
@@ -650,7 +667,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 // many blocks (one point per thread), exact test over the pixel's edges (pip_eval).  COUNT:
 // shared-memory histogram (or global atomics); SELECT/PAIRS: per-block count pass, block scan,
 // one global atomic, write pass.
-template <int MODE>
+template <int MODE, int KIND>
 __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                   uint32_t cap, const unsigned int* __restrict__ fill, int nreg, Out o,
                                                   int smem_hist) {
@@ -681,14 +698,14 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
     const bool act = e.rec != kHole;
     const int64_t pid = o.id_base + (int64_t)e.pidx;
     if (MODE == kCountSmem || MODE == kCountGlobal) {
-      if (act) pip_eval(cvg, e.x, e.y, e.rec, [&](int q) {
+      if (act) pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) {
         if (sh) atomicAdd(&dh[q], 1u); else atomicAdd(o.counts + q, 1ull);
       });
     } else {
       int nres = 0, first = -1;
       if (act) {
-        if (MODE == kSelect) { bool any = false; pip_eval(cvg, e.x, e.y, e.rec, [&](int) { any = true; }); nres = any; }
-        else pip_eval(cvg, e.x, e.y, e.rec, [&](int q) { if (nres++ == 0) first = q; });
+        if (MODE == kSelect) { bool any = false; pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int) { any = true; }); nres = any; }
+        else pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) { if (nres++ == 0) first = q; });
       }
       int excl, tot;
       BS(tmp).ExclusiveSum(nres, excl, tot);
@@ -701,7 +718,7 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
         } else if (nres == 1) {                    // the common case: no second evaluation
           put_result<MODE>(o, pos, pid, first);
         } else {
-          pip_eval(cvg, e.x, e.y, e.rec, [&](int q) { put_result<MODE>(o, pos++, pid, q); });
+          pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) { put_result<MODE>(o, pos++, pid, q); });
         }
       }
       __syncthreads();
@@ -875,10 +892,10 @@ void keep_pool_memory() {
   cudaGetLastError();
 }
 
-template <int MODE, int COMPACT, int QUEUE>
+template <int MODE, int COMPACT, int QUEUE, int KIND>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
   const size_t smem = tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? queue_bytes(MODE) : 0);
-  auto kern = k_probe<MODE, COMPACT, QUEUE>;
+  auto kern = k_probe<MODE, COMPACT, QUEUE, KIND>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
   const int sms = device_sm_count();
@@ -948,8 +965,8 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       const int P = c->d.num_polys;
       const int sh = ((MODE == kCountSmem || MODE == kCountGlobal) && (size_t)P * 4 <= 96 * 1024) ? 1 : 0;
       const size_t dsm = sh ? (size_t)P * 4 : 0;
-      if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
-      k_deferred<MODE><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh);
+      if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
+      k_deferred<MODE, KIND><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh);
       count_launch();
       e = cudaGetLastError();
       static const bool dbg = getenv("SPADE_DEBUG_DEFER") != nullptr;
@@ -978,7 +995,9 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
 
 template <int MODE, int QUEUE = 0>
 int launch_layout(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
-  return c->d.compact ? launch<MODE, 1, QUEUE>(c, xy, n, p, extra, st) : launch<MODE, 0, QUEUE>(c, xy, n, p, extra, st);
+  if (c->d.kind == kDisks)
+    return c->d.compact ? launch<MODE, 1, QUEUE, kDisks>(c, xy, n, p, extra, st) : launch<MODE, 0, QUEUE, kDisks>(c, xy, n, p, extra, st);
+  return c->d.compact ? launch<MODE, 1, QUEUE, kPolygons>(c, xy, n, p, extra, st) : launch<MODE, 0, QUEUE, kPolygons>(c, xy, n, p, extra, st);
 }
 
 Params base_params(const spade_canvas* c) {

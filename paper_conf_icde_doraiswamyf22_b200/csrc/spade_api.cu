@@ -13,6 +13,7 @@ namespace spade {
 
 int build_canvas(const int32_t*, const int64_t*, const int64_t*, int32_t, const spade_canvas_params*, cudaStream_t,
                  spade_canvas**);
+int build_disk_canvas(const int32_t*, const int64_t*, int32_t, const spade_canvas_params*, cudaStream_t, spade_canvas**);
 
 namespace {
 thread_local char g_err[512] = "";
@@ -89,6 +90,13 @@ int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const in
   if (!out) return set_error(SPADE_ERR_INVALID_ARG, "spade_build_canvas: out is NULL");
   *out = nullptr;
   return build_canvas(ring_xy, ring_off, poly_ring_off, num_polys, prm, (cudaStream_t)stream, out);
+}
+
+int spade_build_disk_canvas(const int32_t* center_xy, const int64_t* r2, int32_t num_disks,
+                            const spade_canvas_params* prm, spade_stream_t stream, spade_canvas** out) {
+  if (!out) return set_error(SPADE_ERR_INVALID_ARG, "spade_build_disk_canvas: out is NULL");
+  *out = nullptr;
+  return build_disk_canvas(center_xy, r2, num_disks, prm, (cudaStream_t)stream, out);
 }
 
 void spade_canvas_free(spade_canvas* c) {
@@ -209,6 +217,88 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
   cleanup();
   return SPADE_OK;
 #undef HTRY
+}
+
+// ---- kNN (knn.cu) -----------------------------------------------------------------------------
+static bool knn_q_ok(int32_t qx, int32_t qy) {
+  return qx >= -(1 << 30) && qx < (1 << 30) && qy >= -(1 << 30) && qy < (1 << 30);
+}
+
+int spade_knn_histogram(const int32_t* xy, int64_t n, int32_t qx, int32_t qy, int64_t* hist, spade_stream_t stream) {
+  if (n < 0 || (n > 0 && (!xy || !hist))) return set_error(SPADE_ERR_INVALID_ARG, "spade_knn_histogram: bad arguments");
+  if (n > 0 && ((uintptr_t)xy & 7)) return set_error(SPADE_ERR_INVALID_ARG, "spade_knn_histogram: xy must be 8-byte aligned");
+  if (!knn_q_ok(qx, qy)) return set_error(SPADE_ERR_COORD_RANGE, "spade_knn_histogram: query outside [-2^30, 2^30)");
+  return knn_hist(xy, n, qx, qy, hist, (cudaStream_t)stream);
+}
+
+int spade_knn_radius(const int64_t* hist_host, int64_t k, int64_t* r2_out, int64_t* count_out) {
+  if (!hist_host || !r2_out || !count_out || k < 0) return set_error(SPADE_ERR_INVALID_ARG, "spade_knn_radius: bad arguments");
+  int64_t acc = 0;
+  for (int b = 0; b < kKnnBins; ++b) {
+    acc += hist_host[b];
+    if (acc >= k || b == kKnnBins - 1) {
+      *r2_out = (int64_t)knn_bucket_r2(b);
+      *count_out = acc;
+      return SPADE_OK;
+    }
+  }
+  return SPADE_OK;
+}
+
+int spade_knn_select(const int32_t* xy, int64_t n, int64_t point_id_base, int32_t qx, int32_t qy, int64_t r2,
+                     int64_t* out_ids, int64_t* out_d2, int64_t capacity, int64_t* n_out, spade_stream_t stream) {
+  if (n < 0 || (n > 0 && !xy) || (capacity > 0 && (!out_ids || !out_d2)) || r2 < 0 || point_id_base < 0)
+    return set_error(SPADE_ERR_INVALID_ARG, "spade_knn_select: bad arguments");
+  if (n > 0 && ((uintptr_t)xy & 7)) return set_error(SPADE_ERR_INVALID_ARG, "spade_knn_select: xy must be 8-byte aligned");
+  if (!knn_q_ok(qx, qy)) return set_error(SPADE_ERR_COORD_RANGE, "spade_knn_select: query outside [-2^30, 2^30)");
+  return run_with_capacity(capacity, n_out, (cudaStream_t)stream, "spade_knn_select", [&](unsigned long long* t) {
+    return knn_select(xy, n, point_id_base, qx, qy, (uint64_t)r2, out_ids, out_d2, capacity, t, (cudaStream_t)stream);
+  });
+}
+
+int spade_knn_topk(const int64_t* ids, const int64_t* d2, int64_t m, int64_t k, int64_t* out_ids, int64_t* out_d2,
+                   spade_stream_t stream) {
+  if (m < 0 || k < 0 || (m > 0 && k > 0 && (!ids || !d2 || !out_ids)))
+    return set_error(SPADE_ERR_INVALID_ARG, "spade_knn_topk: bad arguments");
+  return knn_topk(ids, d2, m, k, out_ids, out_d2, (cudaStream_t)stream);
+}
+
+int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int32_t qx, int32_t qy, int64_t k, int64_t* out_ids,
+              int64_t* out_d2, int64_t* n_out, spade_stream_t stream) {
+  if (!n_out || k < 0 || n < 0 || (n > 0 && k > 0 && (!xy || !out_ids)) || point_id_base < 0)
+    return set_error(SPADE_ERR_INVALID_ARG, "spade_knn: bad arguments");
+  *n_out = 0;
+  if (!knn_q_ok(qx, qy)) return set_error(SPADE_ERR_COORD_RANGE, "spade_knn: query outside [-2^30, 2^30)");
+  if (n == 0 || k == 0) return SPADE_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  int64_t* hist = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&hist, sizeof(int64_t) * (kKnnBins + 1), st);
+  if (e != cudaSuccess) return check_cuda(e, "spade_knn");
+  int rc = check_cuda(cudaMemsetAsync(hist, 0, sizeof(int64_t) * (kKnnBins + 1), st), "spade_knn");
+  if (rc == SPADE_OK) rc = spade_knn_histogram(xy, n, qx, qy, hist, stream);
+  std::vector<int64_t> h(kKnnBins + 1, 0);
+  if (rc == SPADE_OK) {
+    rc = check_cuda(cudaMemcpyAsync(h.data(), hist, sizeof(int64_t) * (kKnnBins + 1), cudaMemcpyDeviceToHost, st), "spade_knn");
+    if (rc == SPADE_OK) rc = check_cuda(cudaStreamSynchronize(st), "spade_knn");
+  }
+  cudaFreeAsync(hist, st);
+  if (rc != SPADE_OK) return rc;
+  if (h[kKnnBins] > 0)
+    return set_error(SPADE_ERR_COORD_RANGE, "spade_knn: %lld points outside [-2^30, 2^30)", (long long)h[kKnnBins]);
+  int64_t r2 = 0, m = 0;
+  spade_knn_radius(h.data(), k, &r2, &m);
+  if (m == 0) return SPADE_OK;
+  int64_t* cand = nullptr;
+  e = cudaMallocAsync((void**)&cand, sizeof(int64_t) * 2 * (size_t)m, st);
+  if (e != cudaSuccess) return check_cuda(e, "spade_knn candidates");
+  int64_t got = 0;
+  rc = spade_knn_select(xy, n, point_id_base, qx, qy, r2, cand, cand + m, m, &got, stream);
+  if (rc == SPADE_OK && got != m) rc = set_error(SPADE_ERR_INTERNAL, "spade_knn: %lld candidates, expected %lld", (long long)got, (long long)m);
+  if (rc == SPADE_OK) rc = spade_knn_topk(cand, cand + m, m, k, out_ids, out_d2, stream);
+  if (rc == SPADE_OK) rc = check_cuda(cudaStreamSynchronize(st), "spade_knn");
+  cudaFreeAsync(cand, st);
+  if (rc == SPADE_OK) *n_out = std::min(k, m);
+  return rc;
 }
 
 int64_t spade_launch_count(void) { return g_launches.load(); }

@@ -37,6 +37,16 @@ struct RunRec {
 };
 constexpr int kMaskPolys = 64;     // records with more distinct polygons use the slow path
 
+// Canvas kinds: the constraint primitives a canvas is built from (Sec. 4.2).
+//   kPolygons: record "edges" are polygon edges (ax, ay, bx, by), exact test = local crossing parity
+//   kDisks:    record "edges" are disks (cx, cy, r2 low 32 bits, r2 high 32 bits), exact test =
+//              (px-cx)^2 + (py-cy)^2 <= r2 (closed disk, P:127 distance canvases)
+constexpr int32_t kPolygons = 0, kDisks = 1;
+
+__host__ __device__ __forceinline__ int64_t disk_r2(int4 e) {
+  return (int64_t)((uint64_t)(uint32_t)e.z | ((uint64_t)(uint32_t)e.w << 32));
+}
+
 struct CanvasDev {            // passed by value to kernels
   int32_t minx, miny;         // extent origin
   uint32_t extw, exth;        // maxx - minx, maxy - miny (points with larger offsets are outside)
@@ -57,6 +67,7 @@ struct CanvasDev {            // passed by value to kernels
   const int32_t* rec_polys;   // distinct polygons of each record
   const int32_t* sets;        // concatenated sorted owner sets
   const int2* set_rng;        // (begin, count)
+  int32_t kind;               // kPolygons / kDisks
 };
 
 }  // namespace spade
@@ -110,5 +121,14 @@ int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t b
                   int64_t cap, unsigned long long* d_total, cudaStream_t st);
 int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* opt,
                  int32_t* opl, int64_t cap, unsigned long long* d_total, cudaStream_t st);
+
+// kNN (knn.cu): squared-distance buckets = concentric circles of the paper's kNN plan
+constexpr int kKnnBins = 248;      // == SPADE_KNN_BINS
+uint64_t knn_bucket_r2(int b);
+int knn_hist(const int32_t* xy, int64_t n, int32_t qx, int32_t qy, int64_t* hist, cudaStream_t st);
+int knn_select(const int32_t* xy, int64_t n, int64_t base, int32_t qx, int32_t qy, uint64_t r2, int64_t* out_ids,
+               int64_t* out_d2, int64_t cap, unsigned long long* d_total, cudaStream_t st);
+int knn_topk(const int64_t* ids, const int64_t* d2, int64_t m, int64_t k, int64_t* out_ids, int64_t* out_d2,
+             cudaStream_t st);
 
 }  // namespace spade
