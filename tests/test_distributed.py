@@ -77,3 +77,62 @@ def test_shard_ranges_partition():
             assert rs[0][0] == 0 and rs[-1][1] == n
             assert all(rs[i][1] == rs[i + 1][0] for i in range(w - 1))
             assert max(b - a for a, b in rs) - min(b - a for a, b in rs) <= 1
+
+
+# ---- kNN over sharded points: histogram all_reduce, shared radius, candidate all_gather ----
+
+def _bucket(d2):
+    d2 = np.asarray(d2, np.int64)
+    out = d2.copy()
+    big = d2 >= 4
+    e = np.floor(np.log2(np.maximum(d2, 1))).astype(np.int64)
+    # exact floor(log2) for int64 (float rounding near powers of two)
+    e = np.where((1 << np.clip(e, 0, 62)) > d2, e - 1, e)
+    e = np.where((1 << np.clip(e + 1, 0, 62)) <= d2, e + 1, e)
+    out[big] = 4 + 4 * (e[big] - 2) + ((d2[big] >> (e[big] - 2)) & 3)
+    return out
+
+
+def _knn_worker(rank, world, port, out):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        start, stop = sd.shard_range(N, rank, world)
+        xy = _points(start, stop - start)
+        q = (400_000, 500_000)
+
+        def hist_fn(x, q_):
+            d2 = ((x.astype(np.int64) - np.array(q_)) ** 2).sum(1)
+            return torch.from_numpy(np.bincount(_bucket(d2), minlength=249).astype(np.int64))
+
+        def select_fn(x, q_, r2, base):
+            d2 = ((x.astype(np.int64) - np.array(q_)) ** 2).sum(1)
+            m = d2 <= r2
+            return torch.from_numpy(np.nonzero(m)[0].astype(np.int64) + base), torch.from_numpy(d2[m])
+
+        def topk_fn(ids, d2, k):
+            o = np.lexsort((ids.numpy(), d2.numpy()))[:k]
+            return ids[o], d2[o]
+
+        from paper_conf_icde_doraiswamyf22_b200 import knn_radius
+        res = {}
+        for k in (1, 17, 500):
+            ids, d2 = sd.knn_distributed(xy, q, k, start, hist_fn, knn_radius, select_fn, topk_fn)
+            res[k] = (ids.numpy().tolist(), d2.numpy().tolist())
+        out[rank] = res
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_knn_equals_oracle(world):
+    mgr = mp.Manager()
+    out = mgr.dict()
+    mp.spawn(_knn_worker, args=(world, _free_port(), out), nprocs=world, join=True)
+    xy = _points(0, N)
+    for k in (1, 17, 500):
+        oi, od = oracle.knn(xy, (400_000, 500_000), k)
+        for r in range(world):
+            assert out[r][k][0] == oi.tolist()
+            assert out[r][k][1] == od.tolist()
