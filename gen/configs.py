@@ -128,7 +128,7 @@ def dj(n_points: int = 1_000_000_000, n_disks: int = 100_000, meters: float = 20
     c = random_centers(n_disks, 602)
     return DiskWorkload(f"dj_taxi1B_x{n_disks // 1000}k_r{int(meters)}m_pairs", "pairs", taxi_params(601), 601,
                         n_points, {"center_xy": c, "r2": np.full(n_disks, meters_to_r2(meters), np.int64)},
-                        max_dim=16384,
+                        max_dim=8192,
                         desc=f"type 1 distance join: 1B taxi-like points x {n_disks} random points, distance <= {meters} m")
 
 
@@ -139,7 +139,7 @@ def dj2(n_points: int = 1_000_000_000, n_disks: int = 100_000) -> DiskWorkload:
     m = np.exp(rng.uniform(np.log(5.0), np.log(100.0), n_disks))
     r2 = np.array([meters_to_r2(x) for x in m], np.int64)
     return DiskWorkload(f"dj2_taxi1B_x{n_disks // 1000}k_r5to100m_count", "count", taxi_params(611), 611, n_points,
-                        {"center_xy": c, "r2": r2}, max_dim=16384,
+                        {"center_xy": c, "r2": r2}, max_dim=8192,
                         desc=f"type 2 distance join COUNT: 1B taxi-like points x {n_disks} points with radii 5..100 m")
 
 

@@ -123,6 +123,7 @@ struct Params {
   uint32_t defer_cap;
   unsigned int* defer_fill;   // [grid] entries used per CTA region
   uint32_t hcopies;           // COUNT histogram copies in shared memory (power of 2)
+  uint32_t cache_slots;       // COUNT with global counts: shared-memory count cache slots (pow 2, or 0)
   const int2* xy;
   int64_t n;
   int64_t head;               // points before the first 32-byte aligned one (0..3)
@@ -227,18 +228,18 @@ __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int p
 }
 
 template <int MODE>
-__device__ __forceinline__ void count_hit(unsigned int* hist, unsigned long long* counts, int owner) {
-  if (MODE == kCountSmem) atomicAdd(&hist[owner], 1u);
+__device__ __forceinline__ void count_hit(unsigned int* hist, uint32_t hstride, unsigned long long* counts, int owner) {
+  if (MODE == kCountSmem) atomicAdd(&hist[(uint32_t)owner * hstride], 1u);
   else atomicAdd(counts + owner, 1ull);
 }
 
 // Emission from the rare in-kernel paths (deferral region full, unaligned head/tail): per-lane
 // atomics.
 template <int MODE, int KIND>
-__device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, const Out& o,
+__device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, uint32_t hstride, const Out& o,
                                              int x, int y, uint32_t rec, int64_t pid) {
   if (MODE == kCountSmem || MODE == kCountGlobal) {
-    pip_eval<KIND>(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, o.counts, p); });
+    pip_eval<KIND>(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, hstride, o.counts, p); });
   } else if (MODE == kSelect) {
     bool any = false;
     pip_eval<KIND>(cvg, x, y, rec, [&](int) { any = true; });
@@ -249,14 +250,14 @@ __device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, 
 }
 
 template <int MODE>
-__device__ __forceinline__ void rare_emit_owner(unsigned int* hist, const Out& o, int owner, int64_t pid) {
-  if (MODE == kCountSmem || MODE == kCountGlobal) count_hit<MODE>(hist, o.counts, owner);
+__device__ __forceinline__ void rare_emit_owner(unsigned int* hist, uint32_t hstride, const Out& o, int owner, int64_t pid) {
+  if (MODE == kCountSmem || MODE == kCountGlobal) count_hit<MODE>(hist, hstride, o.counts, owner);
   else put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, owner);
 }
 
 // One scalar point (unaligned head / tail): classify synchronously.
 template <int MODE, int KIND>
-__device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, unsigned int* hist,
+__device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, unsigned int* hist, uint32_t hstride,
                                           const Out& o, int x, int y, int64_t pid) {
   const CanvasDev cv = *cvg;
   const uint32_t ux = (uint32_t)x - (uint32_t)cv.minx, uy = (uint32_t)y - (uint32_t)cv.miny;
@@ -265,22 +266,22 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
   uint32_t c = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
   if (c >= cv.mix_min) c = classify_fine(*fine_ptr(cv, c, fx, fy));
   if (c == 0) return;
-  if (c & 0x80000000u) rare_emit_point<MODE, KIND>(cvg, hist, o, x, y, ~c, pid);
-  else rare_emit_owner<MODE>(hist, o, (int)c - 1, pid);
+  if (c & 0x80000000u) rare_emit_point<MODE, KIND>(cvg, hist, hstride, o, x, y, ~c, pid);
+  else rare_emit_owner<MODE>(hist, hstride, o, (int)c - 1, pid);
 }
 
 // COUNT, in-loop variant: evaluate up to 32 queued boundary points (one per lane).  Out of line:
 // the streaming loop keeps a small register footprint.
 template <int MODE, int KIND>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const QEntry* wq,
-                                   int cnt, int lane, unsigned int* hist, unsigned long long* counts) {
+                                   int cnt, int lane, unsigned int* hist, uint32_t hstride, unsigned long long* counts) {
   if (lane < cnt) {
     const QEntry e = wq[lane];
     const CanvasDev& cv = *cvg;
     const uint32_t fx = ((uint32_t)e.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)e.y - (uint32_t)cv.miny) >> cv.s;
     const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
     const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
-    pip_eval<KIND>(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, counts, q); });
+    pip_eval<KIND>(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
   }
 }
 
@@ -346,7 +347,9 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   unsigned char* rest = smem + tbytes;
   const uint32_t P = (uint32_t)cv.num_polys;
   unsigned int* hist = (unsigned int*)rest;                       // COUNT
-  unsigned int* myhist = hist + (lane & (prm.hcopies - 1)) * (P + 1);
+  uint32_t* ctag = (uint32_t*)rest;                               // COUNT (global): cache tags
+  unsigned int* ccnt = (unsigned int*)rest + prm.cache_slots;     //                 cache counts
+  unsigned int* myhist = hist + (lane & (prm.hcopies - 1));
   __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
   __shared__ int s_qn[kNW];                     // QUEUE: per-warp queue fill
   QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : 0)) + warp * kQCap;
@@ -356,6 +359,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   for (uint32_t i = tid; i < tbytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
   if (MODE == kCountSmem)
     for (uint32_t i = tid; i < prm.hcopies * (P + 1); i += T) hist[i] = 0u;
+  if (MODE == kCountGlobal)
+    for (uint32_t i = tid; i < prm.cache_slots; i += T) { ctag[i] = 0xffffffffu; ccnt[i] = 0u; }
   if (tid == 0) s_dfill = 0;
   __syncthreads();
   DEntry* const dreg = QUEUE ? nullptr : prm.defer + (size_t)blockIdx.x * prm.defer_cap;
@@ -367,11 +372,11 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     const int64_t ntail = prm.n - tail0;
     if (lane < prm.head) {
       const int2 p = prm.xy[lane];
-      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + lane);
+      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.hcopies, prm.o, p.x, p.y, prm.o.id_base + lane);
     } else if (lane >= 4 && lane - 4 < ntail) {
       const int64_t i = tail0 + (lane - 4);
       const int2 p = prm.xy[i];
-      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.o, p.x, p.y, prm.o.id_base + i);
+      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.hcopies, prm.o, p.x, p.y, prm.o.id_base + i);
     }
   }
 
@@ -488,7 +493,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         if (qn >= 32) {
           do {
             if (MODE == kSelect || MODE == kPairs) drain_out(wqi + qn - 32, 32, (nvec - 1 - base) / (nctaid_x() * chunk));
-            else drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+            else drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts);
             qn -= 32;
           } while (qn >= 32);
           __syncwarp();
@@ -514,7 +519,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
             dreg[d] = DEntry{p.x, p.y, ~c[q], pidx};
           } else {
             if (d < prm.defer_cap) dreg[d] = DEntry{0, 0, kHole, 0u};
-            rare_emit_point<MODE, KIND>(prm.cvg, myhist, prm.o, p.x, p.y, ~c[q], prm.o.id_base + pidx);
+            rare_emit_point<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, p.x, p.y, ~c[q], prm.o.id_base + pidx);
           }
           ++d;
         }
@@ -524,11 +529,28 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     if (MODE == kCountSmem) {
       // branch-free: non-hits (0 - 1 = 0xFFFFFFFF, boundary >= 2^31 - 1) go to the trash bin P
 #pragma unroll
-      for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P)], 1u);
+      for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
     } else if (MODE == kCountGlobal) {
+      // too many polygons for a shared-memory histogram: hits are aggregated over the lanes of the
+      // warp that hit the same polygon, then counted in a direct-mapped shared-memory cache (the
+      // first polygon to claim a slot keeps it for the CTA's lifetime: hot polygons claim early),
+      // else with one global atomic.  Clustered points hit a few hot polygons whose same-address
+      // global atomics would otherwise serialise in L2.
 #pragma unroll
-      for (int q = 0; q < NPT; ++q)
-        if (c[q] != 0u && !(c[q] >> 31)) atomicAdd(prm.o.counts + (c[q] - 1u), 1ull);
+      for (int q = 0; q < NPT; ++q) {
+        const uint32_t key = (c[q] != 0u && !(c[q] >> 31)) ? c[q] - 1u : 0xffffffffu;
+        const unsigned m = __match_any_sync(0xffffffffu, key);
+        if (key != 0xffffffffu && (m & ((1u << lane) - 1u)) == 0u) {
+          bool cached = false;
+          if (prm.cache_slots) {
+            const uint32_t slot = key & (prm.cache_slots - 1u);
+            uint32_t t = ctag[slot];
+            if (t == 0xffffffffu) { t = atomicCAS(&ctag[slot], 0xffffffffu, key); if (t == 0xffffffffu) t = key; }
+            if (t == key) { atomicAdd(&ccnt[slot], (unsigned)__popc(m)); cached = true; }
+          }
+          if (!cached) atomicAdd(prm.o.counts + key, (unsigned long long)__popc(m));
+        }
+      }
     } else {
       // Output slots for this batch (Map with a scan) from the warp's current chunk: a warp
       // scan (ballots), a new chunk (one global atomic, lane 0) when the batch does not fit.
@@ -613,7 +635,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
           int qn = s_qn[warp];
           if (qn >= 32) {
             do {
-              drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.o.counts);
+              drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts);
               qn -= 32;
             } while (qn >= 32);
             __syncwarp();
@@ -624,7 +646,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
       }
       // phase C2: direct hits (branch-free: non-hits and boundary points go to the trash bin P)
 #pragma unroll
-      for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P)], 1u);
+      for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
     }
   } else {
     // only the next batch of points is prefetched; there are no CTA barriers in the loop, the 32
@@ -650,14 +672,17 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   }
   if (QUEUE && (MODE == kCountSmem || MODE == kCountGlobal)) {
     __syncwarp();
-    if (s_qn[warp] > 0) drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.o.counts);
+    if (s_qn[warp] > 0) drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts);
   }
   __syncthreads();
   if (!QUEUE && tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
+  if (MODE == kCountGlobal)
+    for (uint32_t i = tid; i < prm.cache_slots; i += T)
+      if (ccnt[i]) atomicAdd(prm.o.counts + ctag[i], (unsigned long long)ccnt[i]);
   if (MODE == kCountSmem) {
     for (uint32_t i = tid; i < P; i += T) {
       unsigned long long sum = 0;
-      for (uint32_t k = 0; k < prm.hcopies; ++k) sum += hist[k * (P + 1) + i];
+      for (uint32_t k = 0; k < prm.hcopies; ++k) sum += hist[i * prm.hcopies + k];
       if (sum) atomicAdd(prm.o.counts + i, sum);
     }
   }
@@ -698,9 +723,18 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
     const bool act = e.rec != kHole;
     const int64_t pid = o.id_base + (int64_t)e.pidx;
     if (MODE == kCountSmem || MODE == kCountGlobal) {
-      if (act) pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) {
-        if (sh) atomicAdd(&dh[q], 1u); else atomicAdd(o.counts + q, 1ull);
-      });
+      if (sh) {
+        if (act) pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) { atomicAdd(&dh[q], 1u); });
+      } else {
+        // global counts: each point's first result aggregated over the warp (see k_probe)
+        int first = -1;
+        if (act) pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) {
+          if (first < 0) first = q; else atomicAdd(o.counts + q, 1ull);
+        });
+        const unsigned m = __match_any_sync(0xffffffffu, first);
+        if (first >= 0 && (m & ((1u << (threadIdx.x & 31)) - 1u)) == 0u)
+          atomicAdd(o.counts + first, (unsigned long long)__popc(m));
+      }
     } else {
       int nres = 0, first = -1;
       if (act) {
@@ -1039,7 +1073,12 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
       return launch_layout<kCountSmem>(c, (const int2*)xy, n, p, hc * one, st);
     }
   }
-  return launch_layout<kCountGlobal>(c, (const int2*)xy, n, p, 0, st);
+  // global counts with a shared-memory count cache in the space the tiles leave
+  uint32_t slots = 0;
+  for (uint32_t ns = 16384; ns >= 1024; ns >>= 1)
+    if (tiles + (size_t)ns * 8 <= kSmemSoft) { slots = ns; break; }
+  p.cache_slots = slots;
+  return launch_layout<kCountGlobal>(c, (const int2*)xy, n, p, (size_t)slots * 8, st);
 }
 
 int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* out, int64_t cap,
