@@ -164,7 +164,9 @@ __device__ __forceinline__ bool disk_hit(int4 g, int px, int py) {
   return (unsigned long long)(dx * dx) + (unsigned long long)(dy * dy) <= (unsigned long long)disk_r2(g);
 }
 
-template <int KIND, class Emit>
+// U > 1 (the deferred kernel, one point per thread): the primitives are loaded U at a time before
+// any is tested, so a record costs ~edge_cnt / U dependent memory round trips instead of edge_cnt.
+template <int KIND, int U = 1, class Emit>
 __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
   const RunRec r = cv->runs[rec];
   const int X = cv->minx + (int)((((uint32_t)px - (uint32_t)cv->minx) >> cv->s) << cv->s);
@@ -188,16 +190,37 @@ __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int p
   if (r.poly_cnt <= kMaskPolys) {
     // each de-duplicated primitive toggles the parity of every polygon that uses it
     uint64_t m = 0;
-    for (int64_t e = r.edge_begin; e < e1; ++e) {
-      const int4 g = __ldg(seg + e);
-      if (KIND == kDisks) {
-        if (disk_hit(g, px, py)) m ^= __ldg(msk + e);
-        continue;
+    if (U > 1) {
+      for (int64_t e0 = r.edge_begin; e0 < e1; e0 += U) {
+        int4 g[U];
+        uint64_t mk[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+          const int64_t e = e0 + k < e1 ? e0 + k : e1 - 1;     // clamped: in bounds, tested once
+          g[k] = __ldg(seg + e);
+          mk[k] = __ldg(msk + e);
+        }
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+          if (e0 + k >= e1) break;
+          const bool h = KIND == kDisks ? disk_hit(g[k], px, py)
+                                        : ((((g[k].y > py) != (g[k].w > py)) || ((g[k].x > X) != (g[k].z > X))) &&
+                                           local_bit(g[k], X, px, py));
+          if (h) m ^= mk[k];
+        }
       }
-      // an edge that straddles neither the horizontal line y = py nor the vertical line x = X
-      // contributes nothing (cr and cu are both 0): skip it without the cross product or its mask
-      if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
-      if (local_bit(g, X, px, py)) m ^= __ldg(msk + e);
+    } else {
+      for (int64_t e = r.edge_begin; e < e1; ++e) {
+        const int4 g = __ldg(seg + e);
+        if (KIND == kDisks) {
+          if (disk_hit(g, px, py)) m ^= __ldg(msk + e);
+          continue;
+        }
+        // an edge that straddles neither the horizontal line y = py nor the vertical line x = X
+        // contributes nothing (cr and cu are both 0): skip it without the cross product or its mask
+        if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
+        if (local_bit(g, X, px, py)) m ^= __ldg(msk + e);
+      }
     }
     while (m) {
       const int k = __ffsll((long long)m) - 1;
@@ -712,23 +735,29 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
   }
   __syncthreads();
   const long long total = s_pre[nreg];
-  for (long long b0 = (long long)blockIdx.x * 256; b0 < total; b0 += (long long)gridDim.x * 256) {
-    const long long v = b0 + threadIdx.x;
-    DEntry e{0, 0, kHole, 0u};
+  auto fetch = [&](long long v) {                // entry v of the flattened regions (or a hole)
+    DEntry d{0, 0, kHole, 0u};
     if (v < total) {
       int lo = 0, hi = nreg;                     // region r: s_pre[r] <= v < s_pre[r + 1]
       while (hi - lo > 1) { const int mid = (lo + hi) >> 1; if (s_pre[mid] <= v) lo = mid; else hi = mid; }
-      e = defer[(size_t)lo * cap + (size_t)(v - s_pre[lo])];
+      d = defer[(size_t)lo * cap + (size_t)(v - s_pre[lo])];
     }
+    return d;
+  };
+  const long long gstride = (long long)gridDim.x * 256;
+  DEntry nxt = fetch((long long)blockIdx.x * 256 + threadIdx.x);
+  for (long long b0 = (long long)blockIdx.x * 256; b0 < total; b0 += gstride) {
+    const DEntry e = nxt;
+    nxt = fetch(b0 + gstride + threadIdx.x);     // the next point's entry in flight meanwhile
     const bool act = e.rec != kHole;
     const int64_t pid = o.id_base + (int64_t)e.pidx;
     if (MODE == kCountSmem || MODE == kCountGlobal) {
       if (sh) {
-        if (act) pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) { atomicAdd(&dh[q], 1u); });
+        if (act) pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int q) { atomicAdd(&dh[q], 1u); });
       } else {
         // global counts: each point's first result aggregated over the warp (see k_probe)
         int first = -1;
-        if (act) pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) {
+        if (act) pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int q) {
           if (first < 0) first = q; else atomicAdd(o.counts + q, 1ull);
         });
         const unsigned m = __match_any_sync(0xffffffffu, first);
@@ -738,8 +767,8 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
     } else {
       int nres = 0, first = -1;
       if (act) {
-        if (MODE == kSelect) { bool any = false; pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int) { any = true; }); nres = any; }
-        else pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) { if (nres++ == 0) first = q; });
+        if (MODE == kSelect) { bool any = false; pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int) { any = true; }); nres = any; }
+        else pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int q) { if (nres++ == 0) first = q; });
       }
       int excl, tot;
       BS(tmp).ExclusiveSum(nres, excl, tot);
