@@ -438,7 +438,8 @@ def main():
         cb.pop("seconds", None)
         cb.pop("sum_counts", None)
         line["cpu_baseline"] = cb
-        line["cpu_rtree_baseline"] = cpu_rtree_rate(w, a.cpu_seconds / 2)
+        if not is_dist:
+            line["cpu_rtree_baseline"] = cpu_rtree_rate(w, a.cpu_seconds / 2)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if ws > 1:
