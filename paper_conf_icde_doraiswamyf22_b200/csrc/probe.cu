@@ -108,8 +108,9 @@ struct Out {
 template <int MODE>
 __device__ __forceinline__ void put_result(const Out& o, int64_t pos, int64_t id, int poly) {
   if (pos < o.cap) {
-    o.out_ids[pos] = id;
-    if (MODE == kPairs) o.out_poly[pos] = poly;
+    // streaming stores (evict-first): the output must not push the canvas out of L2
+    __stcs((long long*)o.out_ids + pos, (long long)id);
+    if (MODE == kPairs) __stcs(o.out_poly + pos, poly);
   } else if (pos - o.cap < o.ovf_cap) {
     o.ovf_ids[pos - o.cap] = id;
     if (MODE == kPairs) o.ovf_poly[pos - o.cap] = poly;
