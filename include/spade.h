@@ -189,6 +189,22 @@ SPADE_API int spade_knn_topk(const int64_t* ids, const int64_t* d2, int64_t m, i
 SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int32_t qx, int32_t qy, int64_t k,
               int64_t* out_ids, int64_t* out_d2, int64_t* n_out, spade_stream_t stream);
 
+/* Probe-path tuning (A/B runs and tests; results never depend on it).  Sets option `name` for
+ * this process; returns INVALID_ARG for an unknown name or value.  Initial values come from the
+ * environment variable SPADE_<NAME> (upper case), else the default:
+ *   "defer"        0 (default) / 1: boundary points always go to the deferral kernel
+ *                  (no in-loop warp queues)
+ *   "count_global" 0 (default) / 1: COUNT with global counters even when the per-polygon
+ *                  shared-memory histogram fits
+ *   "global_queue" 0 (default) / 1: in-loop exact tests also for global-counter COUNT
+ *   "cache_slots"  16384 (default): max shared-memory count-cache slots of global-counter COUNT
+ *                  (power of 2 >= 1024, or 0 = no cache)
+ *   "coop"         0 (default, off) / -1 (auto) / 4 / 8 / 16: lanes per deferred point in
+ *                  COUNT's cooperative exact-test kernel (measured slower than one point per
+ *                  thread on C5 / dj2: fewer points in flight)
+ *   "debug_defer"  0 (default) / 1: print deferral statistics to stderr (synchronises) */
+SPADE_API int spade_set_option(const char* name, int64_t value);
+
 /* Number of kernels this library has launched in this process (for the bench's gpu_launches). */
 SPADE_API int64_t spade_launch_count(void);
 

@@ -85,6 +85,8 @@ def load(path: str | None = None):
     lib.spade_knn_topk.restype = ctypes.c_int
     lib.spade_knn.argtypes = [P, i64, i64, i32, i32, i64, P, P, ctypes.POINTER(i64), P]
     lib.spade_knn.restype = ctypes.c_int
+    lib.spade_set_option.argtypes = [ctypes.c_char_p, i64]
+    lib.spade_set_option.restype = ctypes.c_int
     lib.spade_launch_count.argtypes = []
     lib.spade_launch_count.restype = i64
     lib.spade_status_string.argtypes = [ctypes.c_int]
@@ -97,7 +99,7 @@ def load(path: str | None = None):
 
 EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canvas_free", "spade_canvas_info", "spade_join_count",
                     "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_knn_histogram",
-                    "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_launch_count",
+                    "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_set_option", "spade_launch_count",
                     "spade_status_string", "spade_last_error"]
 
 
@@ -128,6 +130,11 @@ def _dev(a, dtype, shape_last=None):
     if shape_last is not None:
         t = t.reshape(-1, shape_last)
     return t
+
+
+def set_option(name: str, value: int) -> None:
+    """Probe-path tuning option (include/spade.h spade_set_option); results never depend on it."""
+    _check(load().spade_set_option(name.encode(), int(value)), f"set_option({name})")
 
 
 def launch_count() -> int:

@@ -592,6 +592,57 @@ __global__ void k_compact(const int32_t* __restrict__ fine, int W, int H, int b,
 struct BigSize { __host__ __device__ int64_t operator()(int32_t v) const { return v >= 2 ? v : 0; } };
 struct BigFlag { __host__ __device__ int32_t operator()(int32_t v) const { return v >= 2 ? 1 : 0; } };
 
+// K-B6: packed records (spade_internal.cuh "Rec").  Blob size in 16-byte units and layout flags:
+// polygon primitives are stored relative to the pixel's lower-left corner as int16 when all four
+// coordinates fit, masks as bytes when the pixel has <= 8 polygons.
+__device__ __forceinline__ bool fits16(int64_t v) { return v >= -32768 && v <= 32767; }
+__global__ void k_blob_size(int64_t NR, int64_t NB, const RunRec* __restrict__ runs, const int64_t* __restrict__ pix_of,
+                            Geo g, const int4* __restrict__ rseg, int kind, int64_t* __restrict__ bsz,
+                            uint32_t* __restrict__ bflags) {
+  for (int64_t r = blockIdx.x * (int64_t)kBT + threadIdx.x; r < NR; r += (int64_t)gridDim.x * kBT) {
+    if (r >= NB) { bsz[r] = 0; bflags[r] = 0; continue; }          // multi-owner record: no data
+    const RunRec x = runs[r];
+    const int64_t p = pix_of[r];
+    const int64_t X = g.minx + (p % g.W) * g.S, Y = g.miny + (p / g.W) * g.S;
+    bool sh = kind == kPolygons;
+    for (int64_t e = x.edge_begin; e < x.edge_begin + x.edge_cnt && sh; ++e) {
+      const int4 q = rseg[e];
+      sh = fits16(q.x - X) && fits16(q.y - Y) && fits16(q.z - X) && fits16(q.w - Y);
+    }
+    const bool by = x.poly_cnt <= 8;
+    const int64_t bytes = (((int64_t)x.poly_cnt * 4 + 15) & ~15ll) + (int64_t)x.edge_cnt * ((sh ? 8 : 16) + (by ? 1 : 8));
+    bsz[r] = (bytes + 15) >> 4;
+    bflags[r] = (sh ? kRecShort : 0u) | (by ? kRecByte : 0u);
+  }
+}
+
+__global__ void k_blob_pack(int64_t NR, int64_t NB, const RunRec* __restrict__ runs, const int64_t* __restrict__ pix_of,
+                            Geo g, const int4* __restrict__ rseg, const uint64_t* __restrict__ rmask,
+                            const int32_t* __restrict__ rec_polys, const int64_t* __restrict__ boff,
+                            const uint32_t* __restrict__ bflags, Rec* __restrict__ recs, uint4* __restrict__ blob) {
+  for (int64_t r = blockIdx.x * (int64_t)kBT + threadIdx.x; r < NR; r += (int64_t)gridDim.x * kBT) {
+    const RunRec x = runs[r];
+    if (r >= NB) { recs[r] = Rec{0u, x.term, 0, 0u}; continue; }
+    const uint32_t fl = bflags[r];
+    recs[r] = Rec{(uint32_t)boff[r], x.term, x.edge_cnt, (uint32_t)x.poly_cnt | fl};
+    unsigned char* b = (unsigned char*)(blob + boff[r]);
+    int32_t* pp = (int32_t*)b;
+    for (int k = 0; k < x.poly_cnt; ++k) pp[k] = rec_polys[x.poly_begin + k];
+    unsigned char* eb = b + (((int64_t)x.poly_cnt * 4 + 15) & ~15ll);
+    const bool sh = fl & kRecShort, by = fl & kRecByte;
+    unsigned char* mb = eb + (int64_t)x.edge_cnt * (sh ? 8 : 16);
+    const int64_t p = pix_of[r];
+    const int X = (int)(g.minx + (p % g.W) * g.S), Y = (int)(g.miny + (p / g.W) * g.S);
+    for (int k = 0; k < x.edge_cnt; ++k) {
+      const int4 q = rseg[x.edge_begin + k];
+      if (sh) ((short4*)eb)[k] = make_short4((short)(q.x - X), (short)(q.y - Y), (short)(q.z - X), (short)(q.w - Y));
+      else ((int4*)eb)[k] = q;
+      const uint64_t m = rmask[x.edge_begin + k];
+      if (by) mb[k] = (unsigned char)m; else ((uint64_t*)mb)[k] = m;
+    }
+  }
+}
+
 int bits_for(int64_t v) {  // bits to hold values 0..v
   int b = 1;
   while (b < 63 && (v >> b) != 0) ++b;
@@ -806,9 +857,9 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
     TRYF(cudaMemcpyAsync(&D32, pg + L - 1, 4, cudaMemcpyDeviceToHost, st), "D");
     TRYF(cudaStreamSynchronize(st), "sync polys");
   }
-  if (cudaMalloc(&c->rec_polys, sizeof(int32_t) * std::max<int64_t>(D32, 1)) != cudaSuccess)
-    return fail(set_error(SPADE_ERR_OOM, "build: record polygon lists"));
-  if (L > 0) LAUNCH(k_recpolys, L, lk2, L, ph, pg, c->rec_polys);
+  int32_t* rec_polys;
+  ALLOC(rec_polys, D32, "record polygon lists");
+  if (L > 0) LAUNCH(k_recpolys, L, lk2, L, ph, pg, rec_polys);
   if (NB > 0) LAUNCH(k_polyrange, NB, NB, le_beg, le_cnt, pg, pbeg, pcnt);
   int64_t LM = 0;
   TRYF(cudaMemsetAsync(mcnt, 0, sizeof(int32_t) * std::max<int64_t>(NB, 1), st), "memset");
@@ -827,10 +878,9 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
     TRYF(cudaStreamSynchronize(st), "sync merged");
     LM = lb + lc;
   }
-  if (cudaMalloc(&c->run_seg, sizeof(int4) * std::max<int64_t>(LM, 1)) != cudaSuccess ||
-      cudaMalloc(&c->run_mask, sizeof(uint64_t) * std::max<int64_t>(LM, 1)) != cudaSuccess)
-    return fail(set_error(SPADE_ERR_OOM, "build: local edge arrays"));
-  if (L > 0) LAUNCH(k_merge<1>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, mbeg, mfill, c->run_seg, c->run_mask, kind);
+  int4* run_seg; uint64_t* run_mask;
+  ALLOC(run_seg, LM, "local edge arrays"); ALLOC(run_mask, LM, "local edge arrays");
+  if (L > 0) LAUNCH(k_merge<1>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, mbeg, mfill, run_seg, run_mask, kind);
   tmp.release(lk); tmp.release(lk2); tmp.release(lv); tmp.release(lv2); tmp.release(frags); tmp.release(lw_off);
   tmp.release(ph); tmp.release(pg); tmp.release(li); tmp.release(tix); tmp.release(tix2); tmp.release(key2s);
 
@@ -884,8 +934,8 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   ALLOC(ksize, NB, "K sizes"); ALLOC(kidx, NB, "K sizes"); ALLOC(koff, NB + 1, "K offsets");
   int64_t KT = 0; int64_t NK = 0;
   if (NB > 0) {
-    LAUNCH(k_kset<0>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, c->run_seg, c->run_mask,
-           pbeg, pcnt, c->rec_polys, ksize, nullptr, nullptr, nullptr, kind);
+    LAUNCH(k_kset<0>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, run_seg, run_mask,
+           pbeg, pcnt, rec_polys, ksize, nullptr, nullptr, nullptr, kind);
     cub::TransformInputIterator<int64_t, BigSize, const int32_t*> it_sz(ksize, BigSize());
     cub::TransformInputIterator<int32_t, BigFlag, const int32_t*> it_b(ksize, BigFlag());
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, it_sz, koff, NB, st); }), "scan K");
@@ -901,19 +951,40 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   // final set storage: [corner owner sets (M entries, NG ranges)] ++ [K sets with |K| >= 2]
   if (cudaMalloc(&c->sets, sizeof(int32_t) * std::max<int64_t>(M + KT, 1)) != cudaSuccess ||
       cudaMalloc(&c->set_rng, sizeof(int2) * std::max<int64_t>(NG + NK, 1)) != cudaSuccess ||
-      cudaMalloc(&c->runs, sizeof(RunRec) * std::max<int64_t>(NB + NG, 1)) != cudaSuccess ||
       cudaMalloc(&c->fine, sizeof(int32_t) * WH) != cudaSuccess)
     return fail(set_error(SPADE_ERR_OOM, "build: records"));
+  RunRec* runs;
+  ALLOC(runs, NB + NG, "records");
   if (M > 0) {
     TRYF(cudaMemcpyAsync(c->sets, csets, sizeof(int32_t) * M, cudaMemcpyDeviceToDevice, st), "copy sets");
     TRYF(cudaMemcpyAsync(c->set_rng, crng, sizeof(int2) * NG, cudaMemcpyDeviceToDevice, st), "copy sets");
   }
   if (NB > 0) {
-    LAUNCH(k_kset<1>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, c->run_seg, c->run_mask,
-           pbeg, pcnt, c->rec_polys, ksize, koff, c->sets + M, c->runs, kind);
-    LAUNCH(k_kset_rng, NB, NB, ksize, koff, kidx, NG, M, c->set_rng, c->runs);
+    LAUNCH(k_kset<1>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, run_seg, run_mask,
+           pbeg, pcnt, rec_polys, ksize, koff, c->sets + M, runs, kind);
+    LAUNCH(k_kset_rng, NB, NB, ksize, koff, kidx, NG, M, c->set_rng, runs);
   }
-  if (NG > 0) LAUNCH(k_multi_recs, NG, NG, NB, c->runs);
+  if (NG > 0) LAUNCH(k_multi_recs, NG, NG, NB, runs);
+
+  // --- K-B6 packed records: one 16-B record + one contiguous blob per boundary pixel ---
+  {
+    const int64_t NR = NB + NG;
+    int64_t *bsz, *boff;
+    uint32_t* bflags;
+    ALLOC(bsz, NR, "record blobs"); ALLOC(boff, NR + 1, "record blobs"); ALLOC(bflags, NR, "record blobs");
+    LAUNCH(k_blob_size, NR, NR, NB, runs, pix_of, g, run_seg, kind, bsz, bflags);
+    TRYF(cudaMemsetAsync(boff, 0, 8, st), "memset");
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, bsz, boff + 1, NR, st); }), "scan blobs");
+    int64_t units = 0;
+    TRYF(cudaMemcpyAsync(&units, boff + NR, 8, cudaMemcpyDeviceToHost, st), "blob size");
+    TRYF(cudaStreamSynchronize(st), "sync blobs");
+    if (units >= (1ll << 32)) return fail(set_error(SPADE_ERR_INVALID_ARG, "boundary index too large (%lld x 16 B)", (long long)units));
+    if (cudaMalloc(&c->recs, sizeof(Rec) * std::max<int64_t>(NR, 1)) != cudaSuccess ||
+        cudaMalloc(&c->blob, 16 * std::max<int64_t>(units, 1)) != cudaSuccess)
+      return fail(set_error(SPADE_ERR_OOM, "build: packed records"));
+    c->blob_bytes = 16 * units;
+    LAUNCH(k_blob_pack, NR, NR, NB, runs, pix_of, g, run_seg, run_mask, rec_polys, boff, bflags, c->recs, c->blob);
+  }
   LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, c->fine);
 
   // --- K-B5 coarse tiles (+ compact fine layout) ---
@@ -957,8 +1028,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   d.compact = compact ? 1 : 0;
   d.mix_min = compact ? kTileMixedCompact : kTileMixed;
   d.cfine = c->cfine;
-  d.fine = c->fine; d.coarse = c->coarse; d.runs = c->runs; d.run_seg = c->run_seg; d.run_mask = c->run_mask;
-  d.rec_polys = c->rec_polys;
+  d.fine = c->fine; d.coarse = c->coarse; d.recs = c->recs; d.blob = c->blob;
   d.sets = c->sets; d.set_rng = c->set_rng;
   if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
   if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));

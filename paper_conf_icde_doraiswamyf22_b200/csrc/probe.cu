@@ -20,6 +20,7 @@
 //     with 64-bit global atomics; SELECT/PAIRS: CTA-aggregated output reservation (one global
 //     atomic per 4096-point batch), slot-major coalesced stores.
 #include <cstdint>
+#include <climits>
 #include <algorithm>
 #include <cstdlib>
 #include <vector>
@@ -73,6 +74,11 @@ __device__ __forceinline__ uint32_t ld_fine(const int32_t* p, uint64_t pol) {
   return r;
 }
 
+__device__ __forceinline__ uint32_t ctaid_x() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%ctaid.x;" : "=r"(r));
+  return r;
+}
 __device__ __forceinline__ uint32_t nctaid_x() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%nctaid.x;" : "=r"(r));
@@ -165,90 +171,163 @@ __device__ __forceinline__ bool disk_hit(int4 g, int px, int py) {
   return (unsigned long long)(dx * dx) + (unsigned long long)(dy * dy) <= (unsigned long long)disk_r2(g);
 }
 
-// U > 1 (the deferred kernel, one point per thread): the primitives are loaded U at a time before
-// any is tested, so a record costs ~edge_cnt / U dependent memory round trips instead of edge_cnt.
-template <int KIND, int U = 1, class Emit>
-__device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
-  const RunRec r = cv->runs[rec];
-  const int X = cv->minx + (int)((((uint32_t)px - (uint32_t)cv->minx) >> cv->s) << cv->s);
-  int tn, tb = 0;
-  const bool tsingle = r.term >= 0;
-  if (tsingle) tn = 1;
-  else if (r.term == kEmpty) tn = 0;
-  else { int2 g = cv->set_rng[-2 - r.term]; tb = g.x; tn = g.y; }
-  const int32_t* sets = cv->sets;
-  auto term_at = [&](int i) { return tsingle ? r.term : sets[tb + i]; };
-  int ti = 0;
-  auto finalize = [&](int P, int par) {
-    while (ti < tn && term_at(ti) < P) emit(term_at(ti++));
-    if (ti < tn && term_at(ti) == P) { par ^= 1; ++ti; }
-    if (par) emit(P);
-  };
-  const int4* seg = cv->run_seg;
-  const uint64_t* msk = cv->run_mask;
-  const int32_t* rp = cv->rec_polys + r.poly_begin;
-  const int64_t e1 = r.edge_begin + r.edge_cnt;
-  if (r.poly_cnt <= kMaskPolys) {
-    // each de-duplicated primitive toggles the parity of every polygon that uses it
-    uint64_t m = 0;
-    if (U > 1) {
-      for (int64_t e0 = r.edge_begin; e0 < e1; e0 += U) {
-        int4 g[U];
-        uint64_t mk[U];
+__device__ __forceinline__ int4 ld_prim(const short4* p) { const short4 v = __ldg(p); return make_int4(v.x, v.y, v.z, v.w); }
+__device__ __forceinline__ int4 ld_prim(const int4* p) { return __ldg(p); }
+__device__ __forceinline__ uint64_t ld_mask(const uint8_t* p) { return __ldg(p); }
+__device__ __forceinline__ uint64_t ld_mask(const uint64_t* p) { return __ldg(p); }
+
+// Hit of one primitive for point (px, py) in the pixel whose left side is x = X (the primitive
+// and the point in the same coordinates: absolute, or relative to the pixel corner).  An edge that
+// straddles neither y = py nor x = X contributes nothing (cr and cu both 0): two compares.
+template <int KIND>
+__device__ __forceinline__ bool prim_hit(int4 g, int X, int px, int py) {
+  if (KIND == kDisks) return disk_hit(g, px, py);
+  return (((g.y > py) != (g.w > py)) || ((g.x > X) != (g.z > X))) && local_bit(g, X, px, py);
+}
+
+// XOR of the toggle masks of the hit primitives.  U > 1 (the deferred kernel, one point per
+// thread): the primitives are loaded U at a time before any is tested, so a record costs
+// ~ne / U dependent round trips instead of ne.
+template <int KIND, int U, class PT, class MT>
+__device__ __forceinline__ uint64_t hit_mask(const PT* __restrict__ seg, const MT* __restrict__ msk, int ne, int X, int px, int py) {
+  uint64_t m = 0;
+  if (U > 1) {
+    for (int e0 = 0; e0 < ne; e0 += U) {
+      int4 g[U];
+      uint64_t mk[U];
 #pragma unroll
-        for (int k = 0; k < U; ++k) {
-          const int64_t e = e0 + k < e1 ? e0 + k : e1 - 1;     // clamped: in bounds, tested once
-          g[k] = __ldg(seg + e);
-          mk[k] = __ldg(msk + e);
-        }
+      for (int k = 0; k < U; ++k) {
+        const int e = e0 + k < ne ? e0 + k : ne - 1;     // clamped: in bounds, tested once
+        g[k] = ld_prim(seg + e);
+        mk[k] = ld_mask(msk + e);
+      }
 #pragma unroll
-        for (int k = 0; k < U; ++k) {
-          if (e0 + k >= e1) break;
-          const bool h = KIND == kDisks ? disk_hit(g[k], px, py)
-                                        : ((((g[k].y > py) != (g[k].w > py)) || ((g[k].x > X) != (g[k].z > X))) &&
-                                           local_bit(g[k], X, px, py));
-          if (h) m ^= mk[k];
-        }
+      for (int k = 0; k < U; ++k) {
+        if (e0 + k >= ne) break;
+        if (prim_hit<KIND>(g[k], X, px, py)) m ^= mk[k];
       }
-    } else {
-      for (int64_t e = r.edge_begin; e < e1; ++e) {
-        const int4 g = __ldg(seg + e);
-        if (KIND == kDisks) {
-          if (disk_hit(g, px, py)) m ^= __ldg(msk + e);
-          continue;
-        }
-        // an edge that straddles neither the horizontal line y = py nor the vertical line x = X
-        // contributes nothing (cr and cu are both 0): skip it without the cross product or its mask
-        if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
-        if (local_bit(g, X, px, py)) m ^= __ldg(msk + e);
-      }
-    }
-    while (m) {
-      const int k = __ffsll((long long)m) - 1;
-      m &= m - 1;
-      finalize(__ldg(rp + k), 1);
     }
   } else {
-    // > kMaskPolys polygons: primitives grouped by local polygon index (run_mask = index)
-    int cur = -1, par = 0;
-    for (int64_t e = r.edge_begin; e < e1; ++e) {
-      const int4 g = __ldg(seg + e);
-      if (KIND == kDisks) {
-        if (!disk_hit(g, px, py)) continue;
-      } else {
-        if (((g.y > py) == (g.w > py)) && ((g.x > X) == (g.z > X))) continue;
-        if (!local_bit(g, X, px, py)) continue;
-      }
-      const int k = (int)__ldg(msk + e);
-      if (k != cur) {
-        if (cur >= 0 && par) finalize(__ldg(rp + cur), 1);
-        cur = k; par = 0;
-      }
-      par ^= 1;
-    }
-    if (cur >= 0 && par) finalize(__ldg(rp + cur), 1);
+    for (int e = 0; e < ne; ++e)
+      if (prim_hit<KIND>(ld_prim(seg + e), X, px, py)) m ^= ld_mask(msk + e);
   }
-  while (ti < tn) emit(term_at(ti++));
+  return m;
+}
+
+// > kMaskPolys polygons: primitives grouped by local polygon index (mask = index)
+template <int KIND, class PT, class Fin>
+__device__ __forceinline__ void hit_grouped(const PT* __restrict__ seg, const uint64_t* __restrict__ msk, int ne, int X, int px,
+                                            int py, const int32_t* __restrict__ rp, Fin&& finalize) {
+  int cur = -1, par = 0;
+  for (int e = 0; e < ne; ++e) {
+    if (!prim_hit<KIND>(ld_prim(seg + e), X, px, py)) continue;
+    const int k = (int)__ldg(msk + e);
+    if (k != cur) {
+      if (cur >= 0 && par) finalize(__ldg(rp + cur), 1);
+      cur = k; par = 0;
+    }
+    par ^= 1;
+  }
+  if (cur >= 0 && par) finalize(__ldg(rp + cur), 1);
+}
+
+// The record's result: [P in K] XOR parity_P, i.e. the term set K merged with the polygons whose
+// bit is set in the parity mask m (bit k = the record's k-th polygon, rp[k]); emit(P) ascending.
+// finalize(P, par) is also the hook of the > kMaskPolys path.
+template <class Emit>
+struct TermMerge {
+  const int32_t* sets;
+  int32_t term;
+  int tn, tb, ti;
+  Emit& emit;
+  __device__ __forceinline__ TermMerge(const CanvasDev* __restrict__ cv, int32_t t, Emit& e) : sets(cv->sets), term(t), tb(0), ti(0), emit(e) {
+    if (t >= 0) tn = 1;
+    else if (t == kEmpty) tn = 0;
+    else { const int2 g = cv->set_rng[-2 - t]; tb = g.x; tn = g.y; }
+  }
+  __device__ __forceinline__ int at(int i) const { return term >= 0 ? term : sets[tb + i]; }
+  __device__ __forceinline__ void operator()(int P, int par) {
+    while (ti < tn && at(ti) < P) emit(at(ti++));
+    if (ti < tn && at(ti) == P) { par ^= 1; ++ti; }
+    if (par) emit(P);
+  }
+  __device__ __forceinline__ void mask(uint64_t m, const int32_t* __restrict__ rp) {
+    while (m) { const int k = __ffsll((long long)m) - 1; m &= m - 1; (*this)(__ldg(rp + k), 1); }
+  }
+  __device__ __forceinline__ void rest() { while (ti < tn) emit(at(ti++)); }
+};
+
+// Exact test for a point on the boundary (or multi-owner) pixel of record `rec` (packed layout:
+// spade_internal.cuh "Rec"): one 16-B record fetch, then the record's polygons, primitives and
+// masks from one contiguous blob.  emit(P) for every polygon containing the point, ascending.
+template <int KIND, int U = 1, class Emit>
+__device__ __forceinline__ void pip_eval_rec(const CanvasDev* __restrict__ cv, int px, int py, const Rec r, Emit&& emit) {
+  TermMerge<Emit> fin(cv, r.term, emit);
+  const int ne = r.ecnt;
+  if (ne > 0) {
+    const int pc = (int)(r.pinfo & kRecPcnt);
+    const unsigned char* blob = (const unsigned char*)(cv->blob + r.blob);
+    const int32_t* rp = (const int32_t*)blob;
+    const unsigned char* eb = blob + ((pc * 4 + 15) & ~15);
+    const int X = cv->minx + (int)((((uint32_t)px - (uint32_t)cv->minx) >> cv->s) << cv->s);
+    if (KIND == kPolygons && (r.pinfo & kRecShort)) {
+      // primitives relative to the pixel corner (X, Y): the point moves with them
+      const int Y = cv->miny + (int)((((uint32_t)py - (uint32_t)cv->miny) >> cv->s) << cv->s);
+      const short4* seg = (const short4*)eb;
+      const unsigned char* mb = eb + (size_t)ne * 8;
+      if (pc <= kMaskPolys)
+        fin.mask((r.pinfo & kRecByte) ? hit_mask<KIND, U>(seg, (const uint8_t*)mb, ne, 0, px - X, py - Y)
+                                      : hit_mask<KIND, U>(seg, (const uint64_t*)mb, ne, 0, px - X, py - Y), rp);
+      else
+        hit_grouped<KIND>(seg, (const uint64_t*)mb, ne, 0, px - X, py - Y, rp, fin);
+    } else {
+      const int4* seg = (const int4*)eb;
+      const unsigned char* mb = eb + (size_t)ne * 16;
+      if (pc <= kMaskPolys)
+        fin.mask((r.pinfo & kRecByte) ? hit_mask<KIND, U>(seg, (const uint8_t*)mb, ne, X, px, py)
+                                      : hit_mask<KIND, U>(seg, (const uint64_t*)mb, ne, X, px, py), rp);
+      else
+        hit_grouped<KIND>(seg, (const uint64_t*)mb, ne, X, px, py, rp, fin);
+    }
+  }
+  fin.rest();
+}
+template <int KIND, int U = 1, class Emit>
+__device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
+  pip_eval_rec<KIND, U>(cv, px, py, cv->recs[rec], emit);
+}
+
+// Cooperative exact test: the G lanes of a group share one point (same px, py, rec in every lane);
+// lane gl tests primitives gl, gl + G, ... and the parity masks are XOR-reduced over the group
+// (every lane of the warp must call this).  Returns the group's mask; `big` = the record has more
+// than kMaskPolys polygons (the caller then evaluates it serially with pip_eval).
+template <int KIND, int G>
+__device__ __forceinline__ uint64_t group_mask(const CanvasDev* __restrict__ cv, bool act, int px, int py, const Rec& r, int gl, bool& big) {
+  uint64_t m = 0;
+  const int pc = (int)(r.pinfo & kRecPcnt);
+  big = act && pc > kMaskPolys;
+  if (act && !big && r.ecnt > 0) {
+    const int ne = r.ecnt;
+    const unsigned char* eb = (const unsigned char*)(cv->blob + r.blob) + ((pc * 4 + 15) & ~15);
+    const int X = cv->minx + (int)((((uint32_t)px - (uint32_t)cv->minx) >> cv->s) << cv->s);
+    if (KIND == kPolygons && (r.pinfo & kRecShort)) {
+      const int Y = cv->miny + (int)((((uint32_t)py - (uint32_t)cv->miny) >> cv->s) << cv->s);
+      const short4* seg = (const short4*)eb;
+      const unsigned char* mb = eb + (size_t)ne * 8;
+      const bool by = r.pinfo & kRecByte;
+      for (int k = gl; k < ne; k += G)
+        if (prim_hit<KIND>(ld_prim(seg + k), 0, px - X, py - Y)) m ^= by ? ld_mask((const uint8_t*)mb + k) : ld_mask((const uint64_t*)mb + k);
+    } else {
+      const int4* seg = (const int4*)eb;
+      const unsigned char* mb = eb + (size_t)ne * 16;
+      const bool by = r.pinfo & kRecByte;
+      for (int k = gl; k < ne; k += G)
+        if (prim_hit<KIND>(ld_prim(seg + k), X, px, py)) m ^= by ? ld_mask((const uint8_t*)mb + k) : ld_mask((const uint64_t*)mb + k);
+    }
+  }
+#pragma unroll
+  for (int off = G / 2; off > 0; off >>= 1) m ^= __shfl_xor_sync(0xffffffffu, m, off);
+  return m;
 }
 
 template <int MODE>
@@ -261,6 +340,20 @@ __device__ __forceinline__ void count_hit(unsigned int* hist, uint32_t hstride, 
 // atomics.
 template <int MODE, int KIND>
 __device__ __noinline__ void rare_emit_point(const CanvasDev* __restrict__ cvg, unsigned int* hist, uint32_t hstride, const Out& o,
+                                             int x, int y, uint32_t rec, int64_t pid) {
+  if (MODE == kCountSmem || MODE == kCountGlobal) {
+    pip_eval<KIND>(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, hstride, o.counts, p); });
+  } else if (MODE == kSelect) {
+    bool any = false;
+    pip_eval<KIND>(cvg, x, y, rec, [&](int) { any = true; });
+    if (any) put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, 0);
+  } else {
+    pip_eval<KIND>(cvg, x, y, rec, [&](int p) { put_result<MODE>(o, (int64_t)atomicAdd(o.total, 1ull), pid, p); });
+  }
+}
+
+template <int MODE, int KIND>
+__device__ __forceinline__ void emit_point_inl(const CanvasDev* __restrict__ cvg, unsigned int* hist, uint32_t hstride, const Out& o,
                                              int x, int y, uint32_t rec, int64_t pid) {
   if (MODE == kCountSmem || MODE == kCountGlobal) {
     pip_eval<KIND>(cvg, x, y, rec, [&](int p) { count_hit<MODE>(hist, hstride, o.counts, p); });
@@ -376,7 +469,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   unsigned int* myhist = hist + (lane & (prm.hcopies - 1));
   __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
   __shared__ int s_qn[kNW];                     // QUEUE: per-warp queue fill
-  QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : 0)) + warp * kQCap;
+  QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : MODE == kCountGlobal ? prm.cache_slots * 8 : 0)) +
+               warp * kQCap;
   uint32_t* wqi = (uint32_t*)rest + warp * kQCap;                 // SELECT/PAIRS queue
   if (QUEUE && lane == 0) s_qn[warp] = 0;
 
@@ -602,9 +696,9 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     }
   };
   const uint32_t first = blockIdx.x * chunk;
-  if (QUEUE && MODE == kCountSmem) {
-    // COUNT with in-loop exact tests (the C3 configuration): written out without the lambdas,
-    // which cost this register-bound variant a spill
+  if (MODE == kCountSmem || MODE == kCountGlobal) {
+    // COUNT (in-loop exact tests: the C3 configuration; or deferred: C5): written out without the
+    // lambdas, which cost these register-bound variants a spill of the loop state
     Vec4 nxt;
     if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
     // (the stride is re-read from the special register each batch: kept live, it spilled)
@@ -637,7 +731,34 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
       }
       // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
       const uint32_t orc = c[0] | c[1] | c[2] | c[3];
-      {
+      if (!QUEUE) {
+        // phase C1 (COUNT, deferred): boundary points -> this CTA's deferral region (one smem
+        // atomic per lane that has any, a 16-B store per point); region full: tested right here
+        if ((int)orc < 0) {
+          uint32_t bnd = 0;
+#pragma unroll
+          for (int q = 0; q < NPT; ++q) bnd |= (c[q] >> 31) << q;
+          const uint32_t nb = __popc(bnd);
+          uint32_t d = atomicAdd(&s_dfill, nb);
+          const bool fits = d + nb <= prm.defer_cap;
+#pragma unroll
+          for (int q = 0; q < NPT; ++q) {
+            if ((bnd >> q) & 1u) {
+              const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+              const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+              // (the region's address is re-derived here: kept live, it spilled)
+              DEntry* const dr = prm.defer + (size_t)ctaid_x() * prm.defer_cap;
+              if (fits) {
+                dr[d] = DEntry{x, y, ~c[q], 0u};
+              } else {
+                if (d < prm.defer_cap) dr[d] = DEntry{0, 0, kHole, 0u};
+                emit_point_inl<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, x, y, ~c[q], 0);
+              }
+              ++d;
+            }
+          }
+        }
+      } else {
         // phase C1 (COUNT): boundary points -> warp queue (one smem atomic per lane that has any),
         // drained 32 at a time from the top, in the loop: the ALU-heavy exact tests overlap the
         // memory-bound stream of the other warps
@@ -668,9 +789,31 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
           __syncwarp();
         }
       }
-      // phase C2: direct hits (branch-free: non-hits and boundary points go to the trash bin P)
+      if (MODE == kCountSmem) {
+        // phase C2: direct hits (branch-free: non-hits and boundary points go to the trash bin P)
 #pragma unroll
-      for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
+        for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
+      } else {
+        // phase C2, too many polygons for a shared-memory histogram: hits aggregated over the
+        // lanes of the warp that hit the same polygon, then counted in a direct-mapped shared-memory
+        // cache (the first polygon to claim a slot keeps it: hot polygons claim early), else with
+        // one global atomic (same-address global atomics of clustered points serialise in L2)
+#pragma unroll
+        for (int q = 0; q < NPT; ++q) {
+          const uint32_t key = (c[q] != 0u && !(c[q] >> 31)) ? c[q] - 1u : 0xffffffffu;
+          const unsigned m = __match_any_sync(0xffffffffu, key);
+          if (key != 0xffffffffu && (m & ((1u << lane) - 1u)) == 0u) {
+            bool cached = false;
+            if (prm.cache_slots) {
+              const uint32_t slot = key & (prm.cache_slots - 1u);
+              uint32_t t = ctag[slot];
+              if (t == 0xffffffffu) { t = atomicCAS(&ctag[slot], 0xffffffffu, key); if (t == 0xffffffffu) t = key; }
+              if (t == key) { atomicAdd(&ccnt[slot], (unsigned)__popc(m)); cached = true; }
+            }
+            if (!cached) atomicAdd(prm.o.counts + key, (unsigned long long)__popc(m));
+          }
+        }
+      }
     }
   } else {
     // only the next batch of points is prefetched; there are no CTA barriers in the loop, the 32
@@ -712,12 +855,79 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   }
 }
 
+// COUNT's second kernel, cooperative: the deferred boundary points of every CTA region, flattened;
+// each group of G lanes tests one point (group_mask), its first lane merges the result and counts
+// it (shared-memory histogram when the P bins fit, else warp-aggregated global atomics).
+template <int MODE, int KIND, int G>
+__global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
+                                                            uint32_t cap, const unsigned int* __restrict__ fill, int nreg,
+                                                            unsigned long long* __restrict__ counts, int smem_hist) {
+  constexpr int T = 1024, GPB = T / G;
+  __shared__ long long s_pre[1025];              // exclusive prefix of the region fills
+  extern __shared__ unsigned int dh[];
+  const int P = cvg->num_polys;
+  const int lane = threadIdx.x & 31, gl = lane & (G - 1), grp = threadIdx.x / G;
+  if (smem_hist)
+    for (int i = threadIdx.x; i < P; i += T) dh[i] = 0u;
+  if (threadIdx.x == 0) {                        // nreg <= 1024 regions (one per probe CTA)
+    long long a = 0;
+    for (int r = 0; r < nreg; ++r) { s_pre[r] = a; a += fill[r]; }
+    s_pre[nreg] = a;
+  }
+  __syncthreads();
+  const long long total = s_pre[nreg];
+  auto fetch = [&](long long v) {                // entry v of the flattened regions (or a hole)
+    DEntry d{0, 0, kHole, 0u};
+    if (v < total) {
+      int lo = 0, hi = nreg;
+      while (hi - lo > 1) { const int mid = (lo + hi) >> 1; if (s_pre[mid] <= v) lo = mid; else hi = mid; }
+      d = defer[(size_t)lo * cap + (size_t)(v - s_pre[lo])];
+    }
+    return d;
+  };
+  const long long gstride = (long long)gridDim.x * GPB;
+  DEntry nxt = fetch((long long)blockIdx.x * GPB + grp);
+  for (long long b0 = (long long)blockIdx.x * GPB; b0 < total; b0 += gstride) {   // warp-uniform bound
+    const DEntry e = nxt;
+    nxt = fetch(b0 + gstride + grp);             // the group's next point in flight meanwhile
+    const bool act = e.rec != kHole;
+    Rec r{0u, kEmpty, 0, 0u};
+    if (act) r = cvg->recs[e.rec];
+    bool big;
+    const uint64_t m = group_mask<KIND, G>(cvg, act, e.x, e.y, r, gl, big);
+    int first = -1;
+    if (act && gl == 0) {
+      auto emit = [&](int q) {
+        if (smem_hist) atomicAdd(&dh[q], 1u);
+        else if (first < 0) first = q;
+        else atomicAdd(counts + q, 1ull);
+      };
+      if (big) {
+        pip_eval<KIND>(cvg, e.x, e.y, e.rec, emit);
+      } else {
+        TermMerge<decltype(emit)> fin(cvg, r.term, emit);
+        fin.mask(m, (const int32_t*)(cvg->blob + r.blob));
+        fin.rest();
+      }
+    }
+    if (!smem_hist) {                            // each point's first result aggregated over the warp
+      const unsigned mm = __match_any_sync(0xffffffffu, first);
+      if (first >= 0 && (mm & ((1u << lane) - 1u)) == 0u) atomicAdd(counts + first, (unsigned long long)__popc(mm));
+    }
+  }
+  if (smem_hist) {
+    __syncthreads();
+    for (int q = threadIdx.x; q < P; q += T)
+      if (dh[q]) atomicAdd(counts + q, (unsigned long long)dh[q]);
+  }
+}
+
 // Second kernel: the deferred boundary points of every CTA region, flattened and spread over
 // many blocks (one point per thread), exact test over the pixel's edges (pip_eval).  COUNT:
 // shared-memory histogram (or global atomics); SELECT/PAIRS: per-block count pass, block scan,
 // one global atomic, write pass.
 template <int MODE, int KIND>
-__global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
+__global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                   uint32_t cap, const unsigned int* __restrict__ fill, int nreg, Out o,
                                                   int smem_hist) {
   using BS = cub::BlockScan<int, 256>;
@@ -746,19 +956,27 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
     return d;
   };
   const long long gstride = (long long)gridDim.x * 256;
+  // software pipeline: the entry two points ahead and the record of the next point are in flight
+  // while the current point is tested
+  auto rec_of = [&](const DEntry& d) { return d.rec != kHole ? cvg->recs[d.rec] : Rec{0u, kEmpty, 0, 0u}; };
   DEntry nxt = fetch((long long)blockIdx.x * 256 + threadIdx.x);
+  DEntry nxt2 = fetch((long long)blockIdx.x * 256 + gstride + threadIdx.x);
+  Rec nrec = rec_of(nxt);
   for (long long b0 = (long long)blockIdx.x * 256; b0 < total; b0 += gstride) {
     const DEntry e = nxt;
-    nxt = fetch(b0 + gstride + threadIdx.x);     // the next point's entry in flight meanwhile
+    const Rec rc = nrec;
+    nxt = nxt2;
+    nxt2 = fetch(b0 + 2 * gstride + threadIdx.x);
+    nrec = rec_of(nxt);
     const bool act = e.rec != kHole;
     const int64_t pid = o.id_base + (int64_t)e.pidx;
     if (MODE == kCountSmem || MODE == kCountGlobal) {
       if (sh) {
-        if (act) pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int q) { atomicAdd(&dh[q], 1u); });
+        if (act) pip_eval_rec<KIND, 4>(cvg, e.x, e.y, rc, [&](int q) { atomicAdd(&dh[q], 1u); });
       } else {
         // global counts: each point's first result aggregated over the warp (see k_probe)
         int first = -1;
-        if (act) pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int q) {
+        if (act) pip_eval_rec<KIND, 4>(cvg, e.x, e.y, rc, [&](int q) {
           if (first < 0) first = q; else atomicAdd(o.counts + q, 1ull);
         });
         const unsigned m = __match_any_sync(0xffffffffu, first);
@@ -768,8 +986,8 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
     } else {
       int nres = 0, first = -1;
       if (act) {
-        if (MODE == kSelect) { bool any = false; pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int) { any = true; }); nres = any; }
-        else pip_eval<KIND, 4>(cvg, e.x, e.y, e.rec, [&](int q) { if (nres++ == 0) first = q; });
+        if (MODE == kSelect) { bool any = false; pip_eval_rec<KIND, 4>(cvg, e.x, e.y, rc, [&](int) { any = true; }); nres = any; }
+        else pip_eval_rec<KIND, 4>(cvg, e.x, e.y, rc, [&](int q) { if (nres++ == 0) first = q; });
       }
       int excl, tot;
       BS(tmp).ExclusiveSum(nres, excl, tot);
@@ -782,7 +1000,7 @@ __global__ void __launch_bounds__(256) k_deferred(const CanvasDev* __restrict__ 
         } else if (nres == 1) {                    // the common case: no second evaluation
           put_result<MODE>(o, pos, pid, first);
         } else {
-          pip_eval<KIND>(cvg, e.x, e.y, e.rec, [&](int q) { put_result<MODE>(o, pos++, pid, q); });
+          pip_eval_rec<KIND>(cvg, e.x, e.y, rc, [&](int q) { put_result<MODE>(o, pos++, pid, q); });
         }
       }
       __syncthreads();
@@ -1029,11 +1247,26 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       const int P = c->d.num_polys;
       const int sh = ((MODE == kCountSmem || MODE == kCountGlobal) && (size_t)P * 4 <= 96 * 1024) ? 1 : 0;
       const size_t dsm = sh ? (size_t)P * 4 : 0;
-      if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
-      k_deferred<MODE, KIND><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh);
+      const int coop = options().coop;
+      bool launched = false;
+      if constexpr (MODE == kCountSmem || MODE == kCountGlobal) if (coop != 0) {
+        // cooperative groups sized to the records' mean primitive count (4 / 8 / 16 lanes)
+        const double epr = c->num_runs ? (double)c->num_run_edges / (double)c->num_runs : 1.0;
+        const int G = coop > 0 ? coop : (epr > 10.0 ? 16 : epr > 4.0 ? 8 : 4);
+        const int hs = (size_t)P * 4 <= 200 * 1024 ? 1 : 0;
+        const size_t hsm = hs ? (size_t)P * 4 : 0;
+        auto kd = G >= 16 ? k_deferred_count<MODE, KIND, 16> : G >= 8 ? k_deferred_count<MODE, KIND, 8> : k_deferred_count<MODE, KIND, 4>;
+        cudaFuncSetAttribute(kd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(hsm, 1));
+        kd<<<sms, 1024, hsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o.counts, hs);
+        launched = true;
+      }
+      if (!launched) {
+        if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
+        k_deferred<MODE, KIND><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh);
+      }
       count_launch();
       e = cudaGetLastError();
-      static const bool dbg = getenv("SPADE_DEBUG_DEFER") != nullptr;
+      const bool dbg = options().debug_defer != 0;
       if (dbg && e == cudaSuccess) {           // diagnostics only: synchronises
         std::vector<unsigned int> f(grid);
         cudaMemcpyAsync(f.data(), dfill, sizeof(unsigned int) * grid, cudaMemcpyDeviceToHost, st);
@@ -1075,8 +1308,7 @@ Params base_params(const spade_canvas* c) {
 // SELECT/PAIRS: boundary points tested in the loop (warp queues) when the queues fit beside the
 // tiles; SPADE_DEFER=1 forces the deferral kernel (A/B switch)
 bool use_queue(const spade_canvas* c, int mode) {
-  static const int force_defer = [] { const char* e = getenv("SPADE_DEFER"); return e ? atoi(e) : 0; }();
-  return !force_defer && tiles_bytes_for(c->d.Wc, c->d.Hc) + queue_bytes(mode) <= kSmemSoft;
+  return !options().defer && tiles_bytes_for(c->d.Wc, c->d.Hc) + queue_bytes(mode) <= kSmemSoft;
 }
 
 }  // namespace
@@ -1090,22 +1322,33 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   const size_t tiles = tiles_bytes_for(c->d.Wc, c->d.Hc);
   const size_t one = (size_t)(c->d.num_polys + 1) * 4;
   const size_t queue = queue_bytes(kCountSmem);
-  static const int force_defer = [] { const char* e = getenv("SPADE_DEFER"); return e ? atoi(e) : 0; }();
-  for (uint32_t hc = 8; hc >= 1; hc >>= 1) {
+  const int force_defer = options().defer, force_global = options().count_global;
+  for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {
     if (!force_defer && tiles + hc * one + queue <= kSmemSoft) {
       p.hcopies = hc;
       return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hc * one, st);
     }
   }
-  for (uint32_t hc = 8; hc >= 1; hc >>= 1) {
+  for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {
     if (tiles + hc * one <= kSmemSoft || (hc == 1 && tiles + one <= 227 * 1024)) {
       p.hcopies = hc;
       return launch_layout<kCountSmem>(c, (const int2*)xy, n, p, hc * one, st);
     }
   }
   // global counts with a shared-memory count cache in the space the tiles leave
+  // (boundary points tested in the loop when the warp queues fit too)
+  const int max_slots = options().cache_slots;
+  // (measured on C5 / dj2: in-loop tests 3-12% slower than deferral; opt in with SPADE_GLOBAL_QUEUE=1)
+  const int global_queue = options().global_queue;
+  const size_t gq = (force_defer || !global_queue) ? SIZE_MAX / 2 : queue;
   uint32_t slots = 0;
-  for (uint32_t ns = 16384; ns >= 1024; ns >>= 1)
+  for (uint32_t ns = (uint32_t)max_slots; ns >= 1024; ns >>= 1)
+    if (tiles + gq + (size_t)ns * 8 <= kSmemSoft) { slots = ns; break; }
+  if (slots || tiles + gq <= kSmemSoft) {
+    p.cache_slots = slots;
+    return launch_layout<kCountGlobal, 1>(c, (const int2*)xy, n, p, (size_t)slots * 8, st);
+  }
+  for (uint32_t ns = (uint32_t)max_slots; ns >= 1024; ns >>= 1)
     if (tiles + (size_t)ns * 8 <= kSmemSoft) { slots = ns; break; }
   p.cache_slots = slots;
   return launch_layout<kCountGlobal>(c, (const int2*)xy, n, p, (size_t)slots * 8, st);

@@ -2,6 +2,8 @@
 // error detail, launch accounting, the capacity protocol of the Map operator (PAPER.md P:167-175:
 // 1-pass Map when n_max fits, else count first and retry) and the host-resident streaming join.
 #include <cstdarg>
+#include <cstdlib>
+#include <string>
 #include <cstdio>
 #include <cstring>
 #include <atomic>
@@ -83,6 +85,18 @@ int run_with_capacity(int64_t capacity, int64_t* n_out, cudaStream_t st, const c
 
 using namespace spade;
 
+namespace spade {
+static int env_int(const char* name, int dflt) {
+  const char* e = getenv(name);
+  return e ? atoi(e) : dflt;
+}
+Options& options() {
+  static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
+                   env_int("SPADE_CACHE_SLOTS", 16384), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0)};
+  return o;
+}
+}  // namespace spade
+
 extern "C" {
 
 int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off,
@@ -102,7 +116,7 @@ int spade_build_disk_canvas(const int32_t* center_xy, const int64_t* r2, int32_t
 void spade_canvas_free(spade_canvas* c) {
   if (!c) return;
   cudaDeviceSynchronize();
-  cudaFree(c->fine); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->runs); cudaFree(c->run_seg); cudaFree(c->run_mask); cudaFree(c->rec_polys);
+  cudaFree(c->fine); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->recs); cudaFree(c->blob);
   cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->d_dev);
   delete c;
 }
@@ -302,6 +316,24 @@ int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int32_t qx, i
 }
 
 int64_t spade_launch_count(void) { return g_launches.load(); }
+
+
+int spade_set_option(const char* name, int64_t value) {
+  using spade::set_error;
+  if (!name) return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: name is NULL");
+  spade::Options& o = spade::options();
+  const std::string n(name);
+  const bool bit = value == 0 || value == 1;
+  if (n == "defer" && bit) o.defer = (int)value;
+  else if (n == "count_global" && bit) o.count_global = (int)value;
+  else if (n == "global_queue" && bit) o.global_queue = (int)value;
+  else if (n == "debug_defer" && bit) o.debug_defer = (int)value;
+  else if (n == "cache_slots" && (value == 0 || (value >= 1024 && value <= (1 << 16) && (value & (value - 1)) == 0)))
+    o.cache_slots = (int)value;
+  else if (n == "coop" && (value == -1 || value == 0 || value == 4 || value == 8 || value == 16)) o.coop = (int)value;
+  else return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: bad option %s = %lld", name, (long long)value);
+  return SPADE_OK;
+}
 
 const char* spade_status_string(int code) {
   switch (code) {

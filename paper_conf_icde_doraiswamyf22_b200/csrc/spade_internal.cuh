@@ -21,7 +21,8 @@ constexpr int32_t kMultiMark = INT32_MIN;     // transient during the fill only
 // the tile's pixels are the m-th block of 2^b x 2^b int32 in cfine (only mixed tiles stored).
 constexpr uint16_t kTileEmpty = 0, kTileMixed = 0xFFFF, kTileMixedCompact = 0x8000;
 
-// Boundary-index record.  For a boundary pixel: the distinct polygons whose edges touch the
+// Boundary-index record as the build derives it (build intermediate; packed into Rec below).
+// For a boundary pixel: the distinct polygons whose edges touch the
 // closed pixel, rec_polys[poly_begin, +poly_cnt) (ascending), the de-duplicated edges
 // [edge_begin, +edge_cnt) in run_seg with run_mask = XOR of (1 << local polygon index) over the
 // polygons using that segment (an edge shared by two polygons is stored once; poly_cnt > 64:
@@ -36,6 +37,21 @@ struct RunRec {
   int32_t poly_cnt;
 };
 constexpr int kMaskPolys = 64;     // records with more distinct polygons use the slow path
+
+// The probe's record (16 B): the build's RunRec packed for one dependent fetch.  `blob` is the
+// record's data in 16-byte units from CanvasDev::blob:
+//   int32 polys[pcnt]                      (padded to 16 B)
+//   primitives[ecnt]: short4 (ax,ay,bx,by) relative to the pixel's lower-left corner when every
+//                     coordinate fits in int16 (kRecShort), else int4 absolute
+//   masks[ecnt]:      uint8 when pcnt <= 8 (kRecByte), else uint64 (toggle mask / local index)
+// Multi-owner records have no blob (ecnt = pcnt = 0).
+struct Rec {
+  uint32_t blob;
+  int32_t term;
+  int32_t ecnt;
+  uint32_t pinfo;             // pcnt | kRecShort | kRecByte
+};
+constexpr uint32_t kRecShort = 1u << 31, kRecByte = 1u << 30, kRecPcnt = (1u << 30) - 1u;
 
 // Canvas kinds: the constraint primitives a canvas is built from (Sec. 4.2).
 //   kPolygons: record "edges" are polygon edges (ax, ay, bx, by), exact test = local crossing parity
@@ -61,10 +77,8 @@ struct CanvasDev {            // passed by value to kernels
   const int32_t* fine;        // dense W x H canvas (always present)
   const int32_t* cfine;       // compact mixed-tile blocks (compact layout only)
   const uint16_t* coarse;
-  const RunRec* runs;         // records: boundary pixels, then multi-owner pixels
-  const int4* run_seg;        // (ax, ay, bx, by) of the edges touching each boundary pixel
-  const uint64_t* run_mask;   // polygon toggle mask (or local polygon index) per edge
-  const int32_t* rec_polys;   // distinct polygons of each record
+  const Rec* recs;            // records: boundary pixels, then multi-owner pixels
+  const uint4* blob;          // packed record data (Rec::blob)
   const int32_t* sets;        // concatenated sorted owner sets
   const int2* set_rng;        // (begin, count)
   int32_t kind;               // kPolygons / kDisks
@@ -82,10 +96,9 @@ struct spade_canvas {
   int32_t* fine = nullptr;
   int32_t* cfine = nullptr;
   uint16_t* coarse = nullptr;
-  spade::RunRec* runs = nullptr;
-  int4* run_seg = nullptr;
-  uint64_t* run_mask = nullptr;
-  int32_t* rec_polys = nullptr;
+  spade::Rec* recs = nullptr;
+  uint4* blob = nullptr;
+  int64_t blob_bytes = 0;
   int32_t* sets = nullptr;
   int2* set_rng = nullptr;
   spade::CanvasDev* d_dev = nullptr;   // copy of d in device memory (out-of-line exact test)
@@ -114,6 +127,12 @@ int set_error(int code, const char* fmt, ...);
 int check_cuda(cudaError_t e, const char* what);
 void count_launch(int n = 1);
 int device_sm_count();
+
+// probe-path options (spade_set_option; include/spade.h)
+struct Options {
+  int defer, count_global, global_queue, cache_slots, coop, debug_defer;
+};
+Options& options();
 
 // probe launchers (probe.cu)
 int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts, cudaStream_t st);

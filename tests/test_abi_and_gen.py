@@ -67,3 +67,16 @@ def test_config_polygon_sets_have_the_stated_shapes():
     assert len(c4["poly_ring_off"]) - 1 == 50 * 42 + 100
     c2 = configs.c2(10).polys
     assert len(c2["ring_xy"]) == 1000
+
+
+def test_set_option_validates_names_and_values_without_a_gpu():
+    """spade_set_option (probe-path tuning, include/spade.h) is host-only: valid settings are
+    accepted, unknown names and out-of-range values are INVALID_ARG."""
+    import paper_conf_icde_doraiswamyf22_b200 as sp
+    lib = sp.load()
+    for name, value in [("defer", 1), ("defer", 0), ("coop", 8), ("coop", -1), ("cache_slots", 4096),
+                        ("cache_slots", 16384), ("count_global", 0), ("global_queue", 0), ("debug_defer", 0)]:
+        assert lib.spade_set_option(name.encode(), value) == 0, name
+    for name, value in [("coop", 3), ("cache_slots", 1000), ("defer", 2), ("nope", 0)]:
+        assert lib.spade_set_option(name.encode(), value) == -1, name
+    assert lib.spade_set_option(None, 0) == -1
