@@ -202,6 +202,9 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *   "coop"         0 (default, off) / -1 (auto) / 4 / 8 / 16: lanes per deferred point in
  *                  COUNT's cooperative exact-test kernel (measured slower than one point per
  *                  thread on C5 / dj2: fewer points in flight)
+ *   "pipe"         -1 (default, auto: > 50% mixed tiles and a per-polygon histogram that would
+ *                  fill shared memory) / 0 / 1: COUNT with the cp.async-pipelined probe
+ *                  (fine-pixel gathers staged in shared memory, global counters)
  *   "debug_defer"  0 (default) / 1: print deferral statistics to stderr (synchronises) */
 SPADE_API int spade_set_option(const char* name, int64_t value);
 

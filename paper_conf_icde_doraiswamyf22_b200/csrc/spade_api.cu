@@ -92,7 +92,8 @@ static int env_int(const char* name, int dflt) {
 }
 Options& options() {
   static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
-                   env_int("SPADE_CACHE_SLOTS", 16384), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0)};
+                   env_int("SPADE_CACHE_SLOTS", 16384), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
+                   env_int("SPADE_PIPE", -1)};
   return o;
 }
 }  // namespace spade
@@ -330,6 +331,7 @@ int spade_set_option(const char* name, int64_t value) {
   else if (n == "debug_defer" && bit) o.debug_defer = (int)value;
   else if (n == "cache_slots" && (value == 0 || (value >= 1024 && value <= (1 << 16) && (value & (value - 1)) == 0)))
     o.cache_slots = (int)value;
+  else if (n == "pipe" && (value == -1 || bit)) o.pipe = (int)value;
   else if (n == "coop" && (value == -1 || value == 0 || value == 4 || value == 8 || value == 16)) o.coop = (int)value;
   else return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: bad option %s = %lld", name, (long long)value);
   return SPADE_OK;

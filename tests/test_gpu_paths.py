@@ -16,7 +16,7 @@ from tests.helpers import lattice, random_polyset, sorted_pairs
 
 pytestmark = pytest.mark.gpu
 
-DEFAULTS = {"defer": 0, "count_global": 0, "global_queue": 0, "cache_slots": 16384, "coop": 0}
+DEFAULTS = {"defer": 0, "count_global": 0, "global_queue": 0, "cache_slots": 16384, "coop": 0, "pipe": -1}
 
 COUNT_PATHS = [
     {},
@@ -30,6 +30,10 @@ COUNT_PATHS = [
     {"count_global": 1, "cache_slots": 1024, "coop": 16},
     {"count_global": 1, "global_queue": 1},
     {"count_global": 1, "global_queue": 1, "cache_slots": 0},
+    {"pipe": 1},
+    {"pipe": 1, "count_global": 1},
+    {"pipe": 1, "count_global": 1, "cache_slots": 0},
+    {"pipe": 0, "defer": 1},
 ]
 
 
