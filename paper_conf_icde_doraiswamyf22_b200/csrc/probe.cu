@@ -1205,8 +1205,12 @@ __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict
 // and must end up in [T0, M).  k_fixup (one block) sorts the holes, sets *total = M and lists
 // (a) the hole slots below M (destinations, in order) and (b) the runs of result slots at or past
 // M (sources, in order); k_move copies the k-th source into the k-th destination.
-constexpr int kFixT = 1024, kFixItems = 5;
+constexpr int kFixT = 512, kFixItems = 10;
 constexpr int kMaxHoles = kFixT * kFixItems;    // warps per launch (grid <= 160 CTAs)
+#ifndef SPADE_FIX_RADIX_BITS
+#define SPADE_FIX_RADIX_BITS 5
+#endif
+constexpr int kFixRadixBits = SPADE_FIX_RADIX_BITS;   // digit width of the hole sort's passes
 struct FixMeta {
   long long M, nmove;
 };
@@ -1216,7 +1220,7 @@ struct FixMeta {
 template <typename Key>
 __device__ __forceinline__ void sort_holes(unsigned long long (&start)[kFixItems], int (&len)[kFixItems],
                                            unsigned long long lo, int bits, void* tmp) {
-  using Sort = cub::BlockRadixSort<Key, kFixT, kFixItems, int>;
+  using Sort = cub::BlockRadixSort<Key, kFixT, kFixItems, int, kFixRadixBits>;
   Key key[kFixItems];
 #pragma unroll
   for (int i = 0; i < kFixItems; ++i) key[i] = (Key)(start[i] - lo);
@@ -1229,8 +1233,8 @@ __global__ void __launch_bounds__(kFixT) k_fixup(const longlong2* __restrict__ h
                                                  int64_t cap, long long* __restrict__ dst_start,
                                                  long long* __restrict__ dst_pre, long long* __restrict__ src_start,
                                                  long long* __restrict__ src_pre, FixMeta* meta) {
-  using Sort32 = cub::BlockRadixSort<unsigned int, kFixT, kFixItems, int>;
-  using Sort64 = cub::BlockRadixSort<unsigned long long, kFixT, kFixItems, int>;
+  using Sort32 = cub::BlockRadixSort<unsigned int, kFixT, kFixItems, int, kFixRadixBits>;
+  using Sort64 = cub::BlockRadixSort<unsigned long long, kFixT, kFixItems, int, kFixRadixBits>;
   using Scan = cub::BlockScan<long long, kFixT>;
   using Red = cub::BlockReduce<unsigned long long, kFixT>;
   __shared__ union {
@@ -1327,11 +1331,20 @@ __device__ __forceinline__ int find_run(const long long* __restrict__ pre, int n
   return lo;
 }
 
+// (the two prefix arrays are copied to shared memory first: the per-slot searches would otherwise
+// be ~26 dependent L2 round trips, the whole kernel's duration for small outputs)
 template <int MODE>
-__global__ void k_move(Out o, const long long* __restrict__ dst_start, const long long* __restrict__ dst_pre,
-                       const long long* __restrict__ src_start, const long long* __restrict__ src_pre,
-                       const FixMeta* __restrict__ meta) {
+__global__ void __launch_bounds__(1024) k_move(Out o, const long long* __restrict__ dst_start, const long long* __restrict__ dst_pre_g,
+                                               const long long* __restrict__ src_start, const long long* __restrict__ src_pre_g,
+                                               const FixMeta* __restrict__ meta) {
+  extern __shared__ long long pre_s[];
+  long long* dst_pre = pre_s;
+  long long* src_pre = pre_s + kMaxHoles;
   const FixMeta m = *meta;
+  if (m.nmove == 0) return;
+  for (int i = threadIdx.x; i < kMaxHoles; i += blockDim.x) dst_pre[i] = dst_pre_g[i];
+  for (int i = threadIdx.x; i < kMaxHoles + 1; i += blockDim.x) src_pre[i] = src_pre_g[i];
+  __syncthreads();
   for (long long k = blockIdx.x * (long long)blockDim.x + threadIdx.x; k < m.nmove;
        k += (long long)gridDim.x * blockDim.x) {
     const int di = find_run(dst_pre, kMaxHoles, k);
@@ -1471,7 +1484,9 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     if (kOut && e == cudaSuccess) {
       k_fixup<<<1, kFixT, 0, st>>>(p.o.holes, grid * kNW, p.o.total, p.o.cap, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
       count_launch();
-      k_move<MODE><<<sms * 4, 256, 0, st>>>(p.o, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
+      const int msm = (int)(sizeof(long long) * (2 * kMaxHoles + 1));
+      cudaFuncSetAttribute(k_move<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, msm);
+      k_move<MODE><<<sms, 1024, msm, st>>>(p.o, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
       count_launch();
       e = cudaGetLastError();
     }
