@@ -197,7 +197,7 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *   "count_global" 0 (default) / 1: COUNT with global counters even when the per-polygon
  *                  shared-memory histogram fits
  *   "global_queue" 0 (default) / 1: in-loop exact tests also for global-counter COUNT
- *   "cache_slots"  16384 (default): max shared-memory count-cache slots of global-counter COUNT
+ *   "cache_slots"  4096 (default): max shared-memory count-cache slots of global-counter COUNT
  *                  (power of 2 >= 1024, or 0 = no cache)
  *   "coop"         0 (default, off) / -1 (auto) / 4 / 8 / 16: lanes per deferred point in
  *                  COUNT's cooperative exact-test kernel (measured slower than one point per

@@ -147,6 +147,22 @@ struct Params {
   Out o;
 };
 
+// COUNT with global counters, one hit of polygon `key`: the shared-memory count cache (direct
+// mapped; the first polygon to claim a slot keeps it for the CTA's lifetime, so hot polygons of
+// clustered points claim early), else one global atomic.  Same-slot lanes of a warp serialise in
+// the shared-memory atomic unit (cheaper than aggregating them with __match_any_sync first:
+// C5 13.6 -> 11.6 ms).
+__device__ __forceinline__ void count_cached(uint32_t* ctag, unsigned int* ccnt, uint32_t cslots,
+                                             unsigned long long* counts, uint32_t key) {
+  if (cslots) {
+    const uint32_t sl = key & (cslots - 1u);
+    uint32_t t = ctag[sl];
+    if (t == 0xffffffffu) { t = atomicCAS(&ctag[sl], 0xffffffffu, key); if (t == 0xffffffffu) t = key; }
+    if (t == key) { atomicAdd(&ccnt[sl], 1u); return; }
+  }
+  atomicAdd(counts + key, 1ull);
+}
+
 // Point class after the fine gather: c = fine pixel value + 1, i.e. 0 = no polygon,
 // 1 .. 2^31-1 = owner + 1, and >= 2^31 = record ~c (boundary / multi-owner pixel).  Uniform
 // coarse tiles give the same encoding directly (tile value = owner + 1, 0 = empty).
@@ -658,26 +674,10 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #pragma unroll
       for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
     } else if (MODE == kCountGlobal) {
-      // too many polygons for a shared-memory histogram: hits are aggregated over the lanes of the
-      // warp that hit the same polygon, then counted in a direct-mapped shared-memory cache (the
-      // first polygon to claim a slot keeps it for the CTA's lifetime: hot polygons claim early),
-      // else with one global atomic.  Clustered points hit a few hot polygons whose same-address
-      // global atomics would otherwise serialise in L2.
+      // too many polygons for a shared-memory histogram: the count cache
 #pragma unroll
-      for (int q = 0; q < NPT; ++q) {
-        const uint32_t key = (c[q] != 0u && !(c[q] >> 31)) ? c[q] - 1u : 0xffffffffu;
-        const unsigned m = __match_any_sync(0xffffffffu, key);
-        if (key != 0xffffffffu && (m & ((1u << lane) - 1u)) == 0u) {
-          bool cached = false;
-          if (prm.cache_slots) {
-            const uint32_t slot = key & (prm.cache_slots - 1u);
-            uint32_t t = ctag[slot];
-            if (t == 0xffffffffu) { t = atomicCAS(&ctag[slot], 0xffffffffu, key); if (t == 0xffffffffu) t = key; }
-            if (t == key) { atomicAdd(&ccnt[slot], (unsigned)__popc(m)); cached = true; }
-          }
-          if (!cached) atomicAdd(prm.o.counts + key, (unsigned long long)__popc(m));
-        }
-      }
+      for (int q = 0; q < NPT; ++q)
+        if (c[q] != 0u && !(c[q] >> 31)) count_cached(ctag, ccnt, prm.cache_slots, prm.o.counts, c[q] - 1u);
     } else {
       // Output slots for this batch (Map with a scan) from the warp's current chunk: a warp
       // scan (ballots), a new chunk (one global atomic, lane 0) when the batch does not fit.
@@ -803,25 +803,10 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #pragma unroll
         for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
       } else {
-        // phase C2, too many polygons for a shared-memory histogram: hits aggregated over the
-        // lanes of the warp that hit the same polygon, then counted in a direct-mapped shared-memory
-        // cache (the first polygon to claim a slot keeps it: hot polygons claim early), else with
-        // one global atomic (same-address global atomics of clustered points serialise in L2)
+        // phase C2, too many polygons for a shared-memory histogram: the count cache
 #pragma unroll
-        for (int q = 0; q < NPT; ++q) {
-          const uint32_t key = (c[q] != 0u && !(c[q] >> 31)) ? c[q] - 1u : 0xffffffffu;
-          const unsigned m = __match_any_sync(0xffffffffu, key);
-          if (key != 0xffffffffu && (m & ((1u << lane) - 1u)) == 0u) {
-            bool cached = false;
-            if (prm.cache_slots) {
-              const uint32_t slot = key & (prm.cache_slots - 1u);
-              uint32_t t = ctag[slot];
-              if (t == 0xffffffffu) { t = atomicCAS(&ctag[slot], 0xffffffffu, key); if (t == 0xffffffffu) t = key; }
-              if (t == key) { atomicAdd(&ccnt[slot], (unsigned)__popc(m)); cached = true; }
-            }
-            if (!cached) atomicAdd(prm.o.counts + key, (unsigned long long)__popc(m));
-          }
-        }
+        for (int q = 0; q < NPT; ++q)
+          if (c[q] != 0u && !(c[q] >> 31)) count_cached(ctag, ccnt, prm.cache_slots, prm.o.counts, c[q] - 1u);
       }
     }
   } else {
@@ -930,6 +915,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
   const uint32_t first = blockIdx.x * T, stride = nctaid_x() * T;
   const uint32_t nb = first < nvec ? (nvec - first + stride - 1) / stride : 0u;   // batches of this CTA
   const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(ring) + 4u * tid;
+  const uint32_t cslots = prm.cache_slots;
   Vec4 nxt;
   if (nb) {
     if (first + tid < nvec) nxt = ld_stream(vp + first + tid);
@@ -1003,20 +989,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
         for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
       } else {
 #pragma unroll
-        for (int q = 0; q < NPT; ++q) {
-          const uint32_t key = (c[q] != 0u && !(c[q] >> 31)) ? c[q] - 1u : 0xffffffffu;
-          const unsigned m = __match_any_sync(0xffffffffu, key);
-          if (key != 0xffffffffu && (m & ((1u << lane) - 1u)) == 0u) {
-            bool cached = false;
-            if (prm.cache_slots) {
-              const uint32_t sl = key & (prm.cache_slots - 1u);
-              uint32_t t = ctag[sl];
-              if (t == 0xffffffffu) { t = atomicCAS(&ctag[sl], 0xffffffffu, key); if (t == 0xffffffffu) t = key; }
-              if (t == key) { atomicAdd(&ccnt[sl], (unsigned)__popc(m)); cached = true; }
-            }
-            if (!cached) atomicAdd(prm.o.counts + key, (unsigned long long)__popc(m));
-          }
-        }
+        for (int q = 0; q < NPT; ++q)
+          if (c[q] != 0u && !(c[q] >> 31)) count_cached(ctag, ccnt, cslots, prm.o.counts, c[q] - 1u);
       }
     }
   }

@@ -92,7 +92,7 @@ static int env_int(const char* name, int dflt) {
 }
 Options& options() {
   static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
-                   env_int("SPADE_CACHE_SLOTS", 16384), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
+                   env_int("SPADE_CACHE_SLOTS", 4096), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
                    env_int("SPADE_PIPE", -1)};
   return o;
 }

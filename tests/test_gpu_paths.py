@@ -16,7 +16,7 @@ from tests.helpers import lattice, random_polyset, sorted_pairs
 
 pytestmark = pytest.mark.gpu
 
-DEFAULTS = {"defer": 0, "count_global": 0, "global_queue": 0, "cache_slots": 16384, "coop": 0, "pipe": -1}
+DEFAULTS = {"defer": 0, "count_global": 0, "global_queue": 0, "cache_slots": 4096, "coop": 0, "pipe": -1}
 
 COUNT_PATHS = [
     {},
