@@ -431,6 +431,45 @@ def main():
                            "api": "spade_join_count_host (pinned host buffer per rank) + all_reduce",
                            "steps": a.e2e_steps, "ok": int(hc.sum()) == total_pts,
                            "timing": "host wall clock around the synchronous API call, max over ranks"}
+    elif not a.no_e2e and not a.profile and op in ("pairs", "select"):
+        # SELECT / PAIRS from pinned host memory into pinned host result arrays
+        # (spade_select_host / spade_join_pairs_host: chunked H2D, probe and result D2H overlapped)
+        host = torch.empty((n, 2), dtype=torch.int32, pin_memory=True)
+        host.copy_(xy)
+        del xy
+        torch.cuda.empty_cache()
+        cap = n
+        hpt = torch.empty(cap, dtype=torch.int64, pin_memory=True)
+        hpl = torch.empty(cap, dtype=torch.int32, pin_memory=True) if op == "pairs" else None
+
+        def e2e_call():
+            if op == "pairs":
+                r = sp.join_pairs_host(cv, host, rank * n, capacity=cap, out=(hpt, hpl))
+                return len(r[0])
+            return len(sp.select_host(cv, host, rank * n, capacity=cap, out=hpt))
+
+        m = e2e_call()   # warm-up
+        times = []
+        for _ in range(a.e2e_steps):
+            if ws > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            s0 = time.perf_counter()
+            m = e2e_call()
+            dt = time.perf_counter() - s0
+            if ws > 1:
+                tt = torch.tensor([dt], dtype=torch.float64, device=dev)
+                dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+                dt = tt.item()
+            times.append(dt)
+        if rank == 0:
+            per = 12 if op == "pairs" else 8
+            line["e2e"] = {"value": total_pts / statistics.median(times), "unit": "points/s",
+                           "h2d_bytes_per_step": n * 8, "d2h_bytes_per_step": m * per,
+                           "api": f"spade_{'join_pairs' if op == 'pairs' else 'select'}_host (pinned host "
+                                  "points -> pinned host results, per rank)",
+                           "steps": a.e2e_steps, "results": m, "ok": m == n_results[0],
+                           "timing": "host wall clock around the synchronous API call, max over ranks"}
     elif rank == 0 and not a.profile:
         line["e2e"] = None
     if rank == 0 and not a.no_cpu_baseline and not a.profile and ws == 1:

@@ -147,6 +147,24 @@ SPADE_API int spade_join_pairs(const spade_canvas* c, const int32_t* xy, int64_t
 SPADE_API int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t n,
                           int64_t* counts_host, spade_stream_t stream);
 
+/* Host-resident SELECT / PAIRS (out-of-core point streams, Sec. 5.3; the
+ * I/O-GPU pipelining of P:480): as spade_select / spade_join_pairs, but xy_host and the outputs
+ * are HOST arrays (pinned memory gives full PCIe bandwidth; pageable works, slower).  The points
+ * are streamed in chunks (spade_set_option "host_chunk", default 2^25 points): the H2D copy of
+ * chunk k+1, the probe of chunk k and the D2H copy of chunk k-1's results run on three internal
+ * streams.  Results come in chunk order, unspecified order within a chunk.  Capacity protocol as
+ * spade_select: `capacity` < total -> SPADE_ERR_CAPACITY with *n_out = total (the first
+ * `capacity` results are written); n_max = n for select and for pairs over
+ * non-overlapping polygons.  Device memory used: 2 staging + 2 result buffers of one
+ * chunk each (a chunk whose PAIRS exceed one chunk is re-run with a larger buffer).
+ * Synchronises `stream` before return.  Errors: INVALID_ARG, CAPACITY, CUDA, OOM. */
+SPADE_API int spade_select_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, int64_t point_id_base,
+                                int64_t* out_ids_host, int64_t capacity, int64_t* n_out, spade_stream_t stream);
+SPADE_API int spade_join_pairs_host(const spade_canvas* c, const int32_t* xy_host, int64_t n,
+                                    int64_t point_id_base, int64_t* out_point_ids_host,
+                                    int32_t* out_poly_ids_host, int64_t capacity, int64_t* n_out,
+                                    spade_stream_t stream);
+
 /* ---- kNN selection over points (Sec. 5.2), in the paper's three steps ------------
  * The circles of step 1 are concentric around the query q with squared radii
  *   r2_b = the largest squared distance of bucket b,  b = 0 .. SPADE_KNN_BINS-1, where
@@ -205,7 +223,9 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *   "pipe"         -1 (default, auto: > 50% mixed tiles and a per-polygon histogram that would
  *                  fill shared memory) / 0 / 1: COUNT with the cp.async-pipelined probe
  *                  (fine-pixel gathers staged in shared memory, global counters)
- *   "debug_defer"  0 (default) / 1: print deferral statistics to stderr (synchronises) */
+ *   "debug_defer"  0 (default) / 1: print deferral statistics to stderr (synchronises)
+ *   "host_chunk"   2^25 (default): points per staging chunk of the host-resident calls
+ *                  (256 .. 2^28) */
 SPADE_API int spade_set_option(const char* name, int64_t value);
 
 /* Number of kernels this library has launched in this process (for the bench's gpu_launches). */

@@ -75,6 +75,10 @@ def load(path: str | None = None):
     lib.spade_join_pairs.restype = ctypes.c_int
     lib.spade_join_count_host.argtypes = [P, P, i64, P, P]
     lib.spade_join_count_host.restype = ctypes.c_int
+    lib.spade_select_host.argtypes = [P, P, i64, i64, P, i64, ctypes.POINTER(i64), P]
+    lib.spade_select_host.restype = ctypes.c_int
+    lib.spade_join_pairs_host.argtypes = [P, P, i64, i64, P, P, i64, ctypes.POINTER(i64), P]
+    lib.spade_join_pairs_host.restype = ctypes.c_int
     lib.spade_knn_histogram.argtypes = [P, i64, i32, i32, P, P]
     lib.spade_knn_histogram.restype = ctypes.c_int
     lib.spade_knn_radius.argtypes = [P, i64, ctypes.POINTER(i64), ctypes.POINTER(i64)]
@@ -98,7 +102,7 @@ def load(path: str | None = None):
 
 
 EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canvas_free", "spade_canvas_info", "spade_join_count",
-                    "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_knn_histogram",
+                    "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_select_host", "spade_join_pairs_host", "spade_knn_histogram",
                     "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_set_option", "spade_launch_count",
                     "spade_status_string", "spade_last_error"]
 
@@ -292,6 +296,70 @@ def join_count_host(canvas: Canvas, xy_host, counts_host=None, stream=None) -> n
                                    counts_host.ctypes.data_as(ctypes.c_void_p), _stream(stream))
     _check(rc, "spade_join_count_host")
     return counts_host
+
+
+def _host_points(xy_host):
+    if hasattr(xy_host, "data_ptr"):      # torch CPU tensor (pinned for full bandwidth)
+        assert not xy_host.is_cuda and xy_host.is_contiguous()
+        return xy_host, xy_host.data_ptr(), xy_host.numel() // 2
+    xy_host = np.ascontiguousarray(xy_host, dtype=np.int32)
+    return xy_host, xy_host.ctypes.data, xy_host.size // 2
+
+
+def _host_out(out, cap, dtype):
+    """Caller's host output array (numpy or CPU tensor, pinned for full bandwidth) if it holds
+    `cap` elements, else a new numpy array; returns (array, address)."""
+    if out is not None:
+        if hasattr(out, "data_ptr"):
+            assert not out.is_cuda and out.is_contiguous() and out.numel() >= cap
+            return out, out.data_ptr()
+        if out.size >= cap:
+            return out, out.ctypes.data
+    a = np.empty(max(cap, 1), dtype=dtype)
+    return a, a.ctypes.data
+
+
+def select_host(canvas: Canvas, xy_host, point_id_base: int = 0, capacity: int | None = None, stream=None,
+                out=None):
+    """SELECT over HOST-resident points (spade_select_host): int64 ids (numpy, or `out`'s type
+    when a large enough host array / pinned CPU tensor is given), chunk order.
+    capacity=None is n_max = n; a too-small capacity retries with the reported size."""
+    _torch()
+    keep, ptr, n = _host_points(xy_host)
+    cap = n if capacity is None else capacity
+    for attempt in range(2):
+        out, optr = _host_out(out if attempt == 0 else None, cap, np.int64)
+        n_out = ctypes.c_int64()
+        rc = load().spade_select_host(canvas.handle, ctypes.c_void_p(ptr), n, point_id_base,
+                                      ctypes.c_void_p(optr), cap, ctypes.byref(n_out), _stream(stream))
+        if rc == SPADE_ERR_CAPACITY:
+            cap = n_out.value
+            continue
+        _check(rc, "spade_select_host")
+        return out[: n_out.value]
+    raise SpadeError(SPADE_ERR_CAPACITY, "select_host: capacity retry failed")
+
+
+def join_pairs_host(canvas: Canvas, xy_host, point_id_base: int = 0, capacity: int | None = None, stream=None,
+                    out=None):
+    """PAIRS over HOST-resident points (spade_join_pairs_host): (int64 point ids, int32 polygon
+    ids) host arrays; `out` = (pt, pl) preallocated host arrays / pinned CPU tensors."""
+    _torch()
+    keep, ptr, n = _host_points(xy_host)
+    cap = n if capacity is None else capacity
+    for attempt in range(2):
+        pt, ptp = _host_out(out[0] if out is not None and attempt == 0 else None, cap, np.int64)
+        pl, plp = _host_out(out[1] if out is not None and attempt == 0 else None, cap, np.int32)
+        n_out = ctypes.c_int64()
+        rc = load().spade_join_pairs_host(canvas.handle, ctypes.c_void_p(ptr), n, point_id_base,
+                                          ctypes.c_void_p(ptp), ctypes.c_void_p(plp), cap,
+                                          ctypes.byref(n_out), _stream(stream))
+        if rc == SPADE_ERR_CAPACITY:
+            cap = n_out.value
+            continue
+        _check(rc, "spade_join_pairs_host")
+        return pt[: n_out.value], pl[: n_out.value]
+    raise SpadeError(SPADE_ERR_CAPACITY, "join_pairs_host: capacity retry failed")
 
 
 # ---- kNN selection (spade_knn*, P:216-226): circles -> aggregation -> distance select -> sort ----

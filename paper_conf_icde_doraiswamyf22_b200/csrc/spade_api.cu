@@ -93,7 +93,7 @@ static int env_int(const char* name, int dflt) {
 Options& options() {
   static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
                    env_int("SPADE_CACHE_SLOTS", 4096), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
-                   env_int("SPADE_PIPE", -1)};
+                   env_int("SPADE_PIPE", -1), (int64_t)1 << 25};
   return o;
 }
 }  // namespace spade
@@ -176,7 +176,7 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
   if (P > 0 && !counts_host) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_count_host: counts_host is NULL");
   if (n == 0 || P == 0) return SPADE_OK;
   cudaStream_t st = (cudaStream_t)stream;
-  const int64_t kChunk = 1ll << 25;             // 32 Mi points = 256 MiB per staging buffer
+  const int64_t kChunk = options().host_chunk;  // default 32 Mi points = 256 MiB per staging buffer
   const int64_t chunk = std::min(kChunk, n);
   int32_t* stage[2] = {nullptr, nullptr};
   int64_t* d_counts = nullptr;
@@ -232,6 +232,163 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
   cleanup();
   return SPADE_OK;
 #undef HTRY
+}
+
+// Host-resident points, SELECT / PAIRS: the Map of P:167-175 applied chunk by chunk to a point
+// stream that lives on the host (NEXT(3)).  Three streams overlap:
+//   cs  H2D of chunk k+1 into staging buffer (k+1)&1
+//   ks  probe of chunk k into device result buffer k&1, then its result count D2H (pinned word)
+//   ds  D2H of chunk k-1's results into the caller's host arrays at the running offset
+// The host waits only on chunk k-1's count, after chunk k's probe is already enqueued.  A chunk
+// whose results exceed its device buffer (possible for PAIRS with overlapping polygons) is re-run
+// with a buffer of the reported size (the 2-pass Map).  Results beyond `capacity` are
+// counted but not copied; the call then returns SPADE_ERR_CAPACITY with *n_out = the total.
+// Output order: chunk order; within a chunk unspecified (as the device calls).
+static int map_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, int64_t base, int64_t* out_ids,
+                    int32_t* out_polys, int64_t capacity, int64_t* n_out, cudaStream_t st, const char* fn) {
+  const bool pairs = out_polys != nullptr || std::string(fn) == "spade_join_pairs_host";
+  const int64_t chunk = std::min(options().host_chunk, n);
+  int32_t* stage[2] = {nullptr, nullptr};
+  int64_t* d_ids[2] = {nullptr, nullptr};
+  int32_t* d_polys[2] = {nullptr, nullptr};
+  int64_t cap_b[2] = {chunk, chunk};
+  unsigned long long* d_tot = nullptr;   // [2] device result counters
+  unsigned long long* h_tot = nullptr;   // [2] pinned copies
+  cudaStream_t cs = nullptr, ks = nullptr, ds = nullptr;
+  cudaEvent_t copied[2] = {}, consumed[2] = {}, probed[2] = {}, drained[2] = {};
+  cudaError_t e = cudaSuccess;
+  auto cleanup = [&]() {
+    for (cudaStream_t s : {ks, cs, ds})
+      if (s) cudaStreamSynchronize(s);
+    for (int i = 0; i < 2; ++i) {
+      cudaFree(stage[i]); cudaFree(d_ids[i]); cudaFree(d_polys[i]);
+      for (cudaEvent_t ev : {copied[i], consumed[i], probed[i], drained[i]})
+        if (ev) cudaEventDestroy(ev);
+    }
+    cudaFree(d_tot);
+    if (h_tot) cudaFreeHost(h_tot);
+    for (cudaStream_t s : {ks, cs, ds})
+      if (s) cudaStreamDestroy(s);
+  };
+#define MTRY(call, what) do { e = (call); if (e != cudaSuccess) { int r_ = check_cuda(e, what); cleanup(); return r_; } } while (0)
+#define MRC(expr) do { int r_ = (expr); if (r_ != SPADE_OK) { cleanup(); return r_; } } while (0)
+  for (int i = 0; i < 2; ++i) {
+    MTRY(cudaMalloc(&stage[i], chunk * 8), "staging");
+    MTRY(cudaMalloc(&d_ids[i], chunk * 8), "result buffer");
+    if (pairs) MTRY(cudaMalloc(&d_polys[i], chunk * 4), "result buffer");
+  }
+  MTRY(cudaMalloc(&d_tot, 2 * sizeof(unsigned long long)), "counter");
+  MTRY(cudaHostAlloc(&h_tot, 2 * sizeof(unsigned long long), cudaHostAllocDefault), "pinned counter");
+  MTRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking), "stream");
+  MTRY(cudaStreamCreateWithFlags(&ks, cudaStreamNonBlocking), "stream");
+  MTRY(cudaStreamCreateWithFlags(&ds, cudaStreamNonBlocking), "stream");
+  for (int i = 0; i < 2; ++i)
+    for (cudaEvent_t* ev : {&copied[i], &consumed[i], &probed[i], &drained[i]})
+      MTRY(cudaEventCreateWithFlags(ev, cudaEventDisableTiming), "event");
+  MTRY(cudaEventRecord(consumed[0], st), "event");   // order after prior work on the caller's stream
+  for (cudaStream_t s : {cs, ks, ds}) MTRY(cudaStreamWaitEvent(s, consumed[0], 0), "wait");
+
+  auto probe = [&](int b, int64_t off, int64_t m) -> int {
+    cudaError_t e2 = cudaMemsetAsync(d_tot + b, 0, sizeof(unsigned long long), ks);
+    if (e2 != cudaSuccess) return check_cuda(e2, fn);
+    int rc = pairs ? launch_pairs(c, stage[b], m, base + off, d_ids[b], d_polys[b], cap_b[b], d_tot + b, ks)
+                   : launch_select(c, stage[b], m, base + off, d_ids[b], cap_b[b], d_tot + b, ks);
+    if (rc != SPADE_OK) return rc;
+    e2 = cudaMemcpyAsync(h_tot + b, d_tot + b, sizeof(unsigned long long), cudaMemcpyDeviceToHost, ks);
+    if (e2 == cudaSuccess) e2 = cudaEventRecord(probed[b], ks);
+    return check_cuda(e2, fn);
+  };
+  int64_t total = 0;
+  // drain chunk j (buffer b): wait for its count, re-run on overflow, copy its results out
+  auto drain = [&](int b, int64_t off, int64_t m) -> int {
+    cudaError_t e2 = cudaEventSynchronize(probed[b]);
+    if (e2 != cudaSuccess) return check_cuda(e2, fn);
+    int64_t cnt = (int64_t)h_tot[b];
+    if (cnt > cap_b[b]) {                       // 2-pass Map for this chunk
+      e2 = cudaStreamSynchronize(ds);
+      if (e2 == cudaSuccess) e2 = cudaStreamSynchronize(ks);
+      if (e2 != cudaSuccess) return check_cuda(e2, fn);
+      cudaFree(d_ids[b]); d_ids[b] = nullptr;
+      cudaFree(d_polys[b]); d_polys[b] = nullptr;
+      e2 = cudaMalloc(&d_ids[b], cnt * 8);
+      if (e2 == cudaSuccess && pairs) e2 = cudaMalloc(&d_polys[b], cnt * 4);
+      if (e2 != cudaSuccess) return check_cuda(e2, fn);
+      cap_b[b] = cnt;
+      int rc = probe(b, off, m);
+      if (rc != SPADE_OK) return rc;
+      e2 = cudaEventSynchronize(probed[b]);
+      if (e2 != cudaSuccess) return check_cuda(e2, fn);
+      cnt = (int64_t)h_tot[b];
+    }
+    const int64_t keep = std::max<int64_t>(0, std::min(cnt, capacity - total));
+    e2 = cudaStreamWaitEvent(ds, probed[b], 0);
+    if (e2 == cudaSuccess && keep > 0)
+      e2 = cudaMemcpyAsync(out_ids + total, d_ids[b], keep * 8, cudaMemcpyDeviceToHost, ds);
+    if (e2 == cudaSuccess && keep > 0 && pairs)
+      e2 = cudaMemcpyAsync(out_polys + total, d_polys[b], keep * 4, cudaMemcpyDeviceToHost, ds);
+    if (e2 == cudaSuccess) e2 = cudaEventRecord(drained[b], ds);
+    total += cnt;
+    return check_cuda(e2, fn);
+  };
+  int64_t prev_off = -1, prev_m = 0;
+  int64_t k = 0;
+  for (int64_t off = 0; off < n; off += chunk, ++k) {
+    const int b = (int)(k & 1);
+    const int64_t m = std::min(chunk, n - off);
+    if (k >= 2) {
+      MTRY(cudaStreamWaitEvent(cs, consumed[b], 0), "wait");   // staging b free (probe k-2 done)
+      MTRY(cudaStreamWaitEvent(ks, drained[b], 0), "wait");    // results b copied out (chunk k-2)
+    }
+    MTRY(cudaMemcpyAsync(stage[b], xy_host + 2 * off, m * 8, cudaMemcpyHostToDevice, cs), "H2D");
+    MTRY(cudaEventRecord(copied[b], cs), "event");
+    MTRY(cudaStreamWaitEvent(ks, copied[b], 0), "wait");
+    MRC(probe(b, off, m));
+    MTRY(cudaEventRecord(consumed[b], ks), "event");
+    if (prev_off >= 0) MRC(drain(b ^ 1, prev_off, prev_m));
+    prev_off = off;
+    prev_m = m;
+  }
+  if (prev_off >= 0) MRC(drain((int)((k - 1) & 1), prev_off, prev_m));
+  MTRY(cudaStreamSynchronize(ds), "sync");
+  MTRY(cudaStreamSynchronize(ks), "sync");
+  MTRY(cudaEventRecord(consumed[0], ks), "event");   // make the caller's stream observe completion
+  MTRY(cudaStreamWaitEvent(st, consumed[0], 0), "wait");
+  cleanup();
+  *n_out = total;
+  if (total > capacity)
+    return set_error(SPADE_ERR_CAPACITY, "%s: %lld results exceed capacity %lld", fn, (long long)total,
+                     (long long)capacity);
+  return SPADE_OK;
+#undef MRC
+#undef MTRY
+}
+
+int spade_select_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, int64_t point_id_base,
+                      int64_t* out_ids_host, int64_t capacity, int64_t* n_out, spade_stream_t stream) {
+  int rc = check_points(c, xy_host, n, "spade_select_host");
+  if (rc) return rc;
+  if (!n_out) return set_error(SPADE_ERR_INVALID_ARG, "spade_select_host: n_out is NULL");
+  if (capacity < 0) return set_error(SPADE_ERR_INVALID_ARG, "spade_select_host: negative capacity");
+  if (capacity > 0 && !out_ids_host) return set_error(SPADE_ERR_INVALID_ARG, "spade_select_host: out_ids_host is NULL");
+  *n_out = 0;
+  if (n == 0) return SPADE_OK;
+  return map_host(c, xy_host, n, point_id_base, out_ids_host, nullptr, capacity, n_out, (cudaStream_t)stream,
+                  "spade_select_host");
+}
+
+int spade_join_pairs_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, int64_t point_id_base,
+                          int64_t* out_point_ids_host, int32_t* out_poly_ids_host, int64_t capacity, int64_t* n_out,
+                          spade_stream_t stream) {
+  int rc = check_points(c, xy_host, n, "spade_join_pairs_host");
+  if (rc) return rc;
+  if (!n_out) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_pairs_host: n_out is NULL");
+  if (capacity < 0) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_pairs_host: negative capacity");
+  if (capacity > 0 && (!out_point_ids_host || !out_poly_ids_host))
+    return set_error(SPADE_ERR_INVALID_ARG, "spade_join_pairs_host: output arrays are NULL");
+  *n_out = 0;
+  if (n == 0) return SPADE_OK;
+  return map_host(c, xy_host, n, point_id_base, out_point_ids_host, out_poly_ids_host, capacity, n_out,
+                  (cudaStream_t)stream, "spade_join_pairs_host");
 }
 
 // ---- kNN (knn.cu) -----------------------------------------------------------------------------
@@ -332,6 +489,7 @@ int spade_set_option(const char* name, int64_t value) {
   else if (n == "cache_slots" && (value == 0 || (value >= 1024 && value <= (1 << 16) && (value & (value - 1)) == 0)))
     o.cache_slots = (int)value;
   else if (n == "pipe" && (value == -1 || bit)) o.pipe = (int)value;
+  else if (n == "host_chunk" && value >= 256 && value <= ((int64_t)1 << 28)) o.host_chunk = value;
   else if (n == "coop" && (value == -1 || value == 0 || value == 4 || value == 8 || value == 16)) o.coop = (int)value;
   else return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: bad option %s = %lld", name, (long long)value);
   return SPADE_OK;

@@ -150,6 +150,53 @@ def test_host_streaming_count_matches_oracle(spade):
     np.testing.assert_array_equal(acc - 7, got)
 
 
+@pytest.mark.parametrize("chunk", [256, 4096, 1 << 25])
+def test_host_streaming_select_pairs_match_oracle(spade, chunk):
+    """spade_select_host / spade_join_pairs_host (NEXT(3): host-resident point streams, P:232-248,
+    P:480): chunked H2D, probe and result D2H on three streams; results in chunk order."""
+    import torch
+    w = configs.c1()
+    xy = np.concatenate([gen.points_host(w.points, w.point_seed, 0, 200_000), configs.c1_edge_points(w.polys)])
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    spade.set_option("host_chunk", chunk)
+    try:
+        ids = spade.select_host(cv, xy, point_id_base=77)
+        pt, pl = spade.join_pairs_host(cv, torch.from_numpy(xy).pin_memory(), point_id_base=77)
+        # capacity protocol: too small -> retried with the reported total
+        pt2, pl2 = spade.join_pairs_host(cv, xy, point_id_base=77, capacity=5)
+    finally:
+        spade.set_option("host_chunk", 1 << 25)
+    np.testing.assert_array_equal(np.sort(ids), oracle.select(xy, w.polys, point_id_base=77))
+    opt, opl = oracle.join_pairs(xy, w.polys, point_id_base=77)
+    for a, b in ((pt, pl), (pt2, pl2)):
+        got = sorted_pairs(a, b)
+        np.testing.assert_array_equal(got[0], opt)
+        np.testing.assert_array_equal(got[1], opl)
+        assert np.all(np.diff((a - 77) // min(chunk, len(xy))) >= 0)     # chunk order
+    assert np.all(np.diff((ids - 77) // min(chunk, len(xy))) >= 0)
+
+
+def test_host_streaming_pairs_chunk_overflow(spade):
+    """Three identical squares: every chunk yields 3x its points in pairs, more than the per-chunk
+    device buffer, so each chunk takes the 2-pass Map re-run."""
+    sq = np.array([[0, 0], [1000, 0], [1000, 1000], [0, 1000]], np.int32)
+    polys = {"ring_xy": np.concatenate([sq] * 3), "ring_off": np.array([0, 4, 8, 12], np.int64),
+             "poly_ring_off": np.array([0, 1, 2, 3], np.int64)}
+    rng = np.random.default_rng(3)
+    xy = rng.integers(-100, 1100, size=(50_000, 2)).astype(np.int32)
+    cv = spade.Canvas(polys)
+    spade.set_option("host_chunk", 1000)
+    try:
+        pt, pl = spade.join_pairs_host(cv, xy, point_id_base=0, capacity=3 * len(xy))
+    finally:
+        spade.set_option("host_chunk", 1 << 25)
+    opt, opl = oracle.join_pairs(xy, polys)
+    got = sorted_pairs(pt, pl)
+    np.testing.assert_array_equal(got[0], opt)
+    np.testing.assert_array_equal(got[1], opl)
+    assert len(pt) > 2 * len(xy)
+
+
 def test_invalid_arguments_are_reported(spade):
     import ctypes
     import torch
