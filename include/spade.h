@@ -224,6 +224,9 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  fill shared memory) / 0 / 1: COUNT with the cp.async-pipelined probe
  *                  (fine-pixel gathers staged in shared memory, global counters)
  *   "debug_defer"  0 (default) / 1: print deferral statistics to stderr (synchronises)
+ *   "defer_xy"     0 (default) / 1: the pipelined probe's deferral entries carry the point
+ *                  (re-read from L2 at classification) instead of k_deferred re-reading it
+ *                  (measured neutral on C5 / dj2: 11.6 vs 11.6-12.3 ms)
  *   "host_chunk"   2^25 (default): points per staging chunk of the host-resident calls
  *                  (256 .. 2^28) */
 SPADE_API int spade_set_option(const char* name, int64_t value);

@@ -140,6 +140,7 @@ struct Params {
   unsigned int* defer_fill;   // [grid] entries used per CTA region
   uint32_t hcopies;           // COUNT histogram copies in shared memory (power of 2)
   uint32_t cache_slots;       // COUNT with global counts: shared-memory count cache slots (pow 2, or 0)
+  uint32_t defer_xy;          // pipelined probe: deferral entries carry the point (re-read from L2)
   const int2* xy;
   int64_t n;
   int64_t head;               // points before the first 32-byte aligned one (0..3)
@@ -970,11 +971,14 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
         const bool fits = d + nbd <= prm.defer_cap;
         DEntry* const dr = prm.defer + (size_t)ctaid_x() * prm.defer_cap;
         const uint32_t pbase = (uint32_t)prm.head + 4u * (first + j * stride + tid);
+        // the batch was streamed D - 1 batches ago (evict-first): its points are still in L2, so
+        // the entry carries them and k_deferred does not re-read them from DRAM
 #pragma unroll
         for (int q = 0; q < NPT; ++q) {
           if ((bnd >> q) & 1u) {
             if (fits) {
-              dr[d] = DEntry{0, 0, ~c[q], pbase + q};
+              const int2 pt = prm.defer_xy ? __ldcg(prm.xy + pbase + q) : make_int2(0, 0);
+              dr[d] = DEntry{pt.x, pt.y, ~c[q], pbase + q};
             } else {
               if (d < prm.defer_cap) dr[d] = DEntry{0, 0, kHole, 0u};
               const int2 p = __ldg(prm.xy + pbase + q);
@@ -1415,6 +1419,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       p.o.holes = (longlong2*)(scratch + offs[4]);
     }
     p.defer = dbuf;
+    p.defer_xy = PIPE ? (uint32_t)options().defer_xy : 0u;
     p.defer_cap = (uint32_t)per;
     p.defer_fill = dfill;
     kern<<<grid, kT, smem, st>>>(p);
@@ -1434,13 +1439,14 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
         const size_t hsm = hs ? (size_t)P * 4 : 0;
         auto kd = G >= 16 ? k_deferred_count<MODE, KIND, 16> : G >= 8 ? k_deferred_count<MODE, KIND, 8> : k_deferred_count<MODE, KIND, 4>;
         cudaFuncSetAttribute(kd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(hsm, 1));
-        kd<<<sms, 1024, hsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o.counts, hs, PIPE ? p.xy : nullptr);
+        kd<<<sms, 1024, hsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o.counts, hs,
+                                   PIPE && !p.defer_xy ? p.xy : nullptr);
         launched = true;
       }
       if (!launched) {
         if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
         k_deferred<MODE, KIND><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh,
-                                                           PIPE ? p.xy : nullptr);
+                                                           PIPE && !p.defer_xy ? p.xy : nullptr);
       }
       count_launch();
       e = cudaGetLastError();
