@@ -227,6 +227,9 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *   "defer_xy"     0 (default) / 1: the pipelined probe's deferral entries carry the point
  *                  (re-read from L2 at classification) instead of k_deferred re-reading it
  *                  (measured neutral on C5 / dj2: 11.6 vs 11.6-12.3 ms)
+ *   "l2_frac_pct"  100 (default) / 1..100: percent of the fine-canvas lines (by address) gathered
+ *                  with L2::evict_last, the rest evict_unchanged (measured: 50/25/12 neutral on
+ *                  C5, 1-5% slower on C4 / dj)
  *   "host_chunk"   2^25 (default): points per staging chunk of the host-resident calls
  *                  (256 .. 2^28) */
 SPADE_API int spade_set_option(const char* name, int64_t value);

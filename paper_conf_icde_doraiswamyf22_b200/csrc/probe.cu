@@ -63,9 +63,12 @@ __device__ __forceinline__ Vec4 ld_stream(const Vec4* p) {
   return r;
 }
 
-__device__ __forceinline__ uint64_t policy_evict_last() {
+// L2 policy of the fine-canvas gathers: evict_last for a fraction `f` of the lines (by address),
+// evict_unchanged for the rest (f = 1: every gather evict_last)
+__device__ __forceinline__ uint64_t policy_evict_last(float f) {
   uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  if (f >= 1.0f) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  else asm volatile("createpolicy.fractional.L2::evict_last.L2::evict_unchanged.b64 %0, %1;" : "=l"(pol) : "f"(f));
   return pol;
 }
 __device__ __forceinline__ uint32_t ld_fine(const int32_t* p, uint64_t pol) {
@@ -141,6 +144,7 @@ struct Params {
   uint32_t hcopies;           // COUNT histogram copies in shared memory (power of 2)
   uint32_t cache_slots;       // COUNT with global counts: shared-memory count cache slots (pow 2, or 0)
   uint32_t defer_xy;          // pipelined probe: deferral entries carry the point (re-read from L2)
+  float l2_frac;              // fraction of fine-canvas lines gathered with L2::evict_last
   const int2* xy;
   int64_t n;
   int64_t head;               // points before the first 32-byte aligned one (0..3)
@@ -508,7 +512,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   if (tid == 0) s_dfill = 0;
   __syncthreads();
   DEntry* const dreg = QUEUE ? nullptr : prm.defer + (size_t)blockIdx.x * prm.defer_cap;
-  const uint64_t pol = policy_evict_last();
+  const uint64_t pol = policy_evict_last(prm.l2_frac);
 
   // unaligned head and tail (< 8 points): CTA 0, warp 0
   if (blockIdx.x == 0 && warp == 0) {
@@ -891,7 +895,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
     for (uint32_t i = tid; i < prm.cache_slots; i += T) { ctag[i] = 0xffffffffu; ccnt[i] = 0u; }
   if (tid == 0) s_dfill = 0;
   __syncthreads();
-  const uint64_t pol = policy_evict_last();
+  const uint64_t pol = policy_evict_last(prm.l2_frac);
 
   if (blockIdx.x == 0 && tid < 32) {               // unaligned head and tail (< 8 points)
     const int64_t tail0 = prm.head + 4 * prm.nvec;
@@ -1420,6 +1424,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     }
     p.defer = dbuf;
     p.defer_xy = PIPE ? (uint32_t)options().defer_xy : 0u;
+    p.l2_frac = (float)options().l2_frac_pct * 0.01f;
     p.defer_cap = (uint32_t)per;
     p.defer_fill = dfill;
     kern<<<grid, kT, smem, st>>>(p);
