@@ -35,9 +35,10 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5", "dj", "dj2", "knn"],
+    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5", "dj", "dj2", "knn", "ov"],
                     help="c3 (default) = the metric's join+COUNT config; c2 select, c4 pairs, c5 40k polygons; "
-                         "dj / dj2 distance joins (type 1 pairs / type 2 count), knn kNN selection")
+                         "dj / dj2 distance joins (type 1 pairs / type 2 count), knn kNN selection, "
+                         "ov overlap-heavy polygon set (1,000 overlapping stars)")
     ap.add_argument("--points-per-gpu", type=int, default=None, help="default: the config's size (1B; C2 100M)")
     ap.add_argument("--impl", default="spade", choices=["spade", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)

@@ -151,5 +151,28 @@ def knn(n_points: int = 1_000_000_000, k: int = 50) -> DiskWorkload:
                         query=(int(q[0]), int(q[1])), desc=f"kNN selection: {k} nearest of 1B taxi-like points")
 
 
+def ov(n_points: int = 1_000_000_000, n_polys: int = 1000) -> Workload:
+    """Overlap-heavy polygon set (the layered canvases of P:148 / P:200 and
+    the layer index of P:270-274): n_polys concave star query regions (48..160 vertices) centred on
+    points drawn from the taxi distribution itself, radii log-uniform in [2^15, 2^20] grid units,
+    so the stars pile up over the dense clusters (tens of polygons deep there).  COUNT per
+    polygon; a point joins every polygon containing it (reading C3), so sum(counts) = pairs."""
+    tp = taxi_params(701)
+    rng = np.random.default_rng(702)
+    import gen
+    ctr = gen.points_host(tp, 703, 0, n_polys).astype(np.int64)
+    polys = []
+    for i in range(n_polys):
+        r = float(2.0 ** rng.uniform(15, 20))
+        n = int(rng.integers(48, 161))
+        cx = min(max(int(ctr[i, 0]), int(r)), DOMAIN - 1 - int(r))
+        cy = min(max(int(ctr[i, 1]), int(r)), DOMAIN - 1 - int(r))
+        polys.append([pg.star(rng, n, cx, cy, r, r * rng.uniform(0.5, 1.0), rmin=0.4, smooth=0.05)])
+    return Workload(f"ov_taxi1B_x{n_polys // 1000}k_overlapping_stars_count", "count", tp, 701, n_points,
+                    pg.assemble(polys), max_dim=8192,
+                    desc=f"overlap-heavy join COUNT: 1B taxi-like points x {n_polys} overlapping star polygons")
+
+
 ALL = {"c1": c1, "c2": c2, "c3": c3, "c4": c4, "c5": c5}
+OVERLAP = {"ov": ov}
 DISTANCE = {"dj": dj, "dj2": dj2, "knn": knn}

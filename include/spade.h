@@ -230,6 +230,10 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *   "l2_frac_pct"  100 (default) / 1..100: percent of the fine-canvas lines (by address) gathered
  *                  with L2::evict_last, the rest evict_unchanged (measured: 50/25/12 neutral on
  *                  C5, 1-5% slower on C4 / dj)
+ *   "multi_agg"    1 (default) / 0: COUNT counts points on multi-owner pixels (overlapping
+ *                  polygons, no edge in the pixel) once per pixel record and spreads the record
+ *                  counts over the owner sets afterwards (the paper's partial-aggregate plan,
+ *                  P:214), instead of one increment per (point, polygon)
  *   "host_chunk"   2^25 (default): points per staging chunk of the host-resident calls
  *                  (256 .. 2^28) */
 SPADE_API int spade_set_option(const char* name, int64_t value);

@@ -145,12 +145,31 @@ struct Params {
   uint32_t cache_slots;       // COUNT with global counts: shared-memory count cache slots (pow 2, or 0)
   uint32_t defer_xy;          // pipelined probe: deferral entries carry the point (re-read from L2)
   float l2_frac;              // fraction of fine-canvas lines gathered with L2::evict_last
+  unsigned int* rec_cnt;      // COUNT over overlapping polygons: points per multi-owner record, or null
+  uint32_t multi_base;        // first multi-owner record id (records >= it have no edges)
   const int2* xy;
   int64_t n;
   int64_t head;               // points before the first 32-byte aligned one (0..3)
   int64_t nvec;               // aligned 4-point vectors after the head
   Out o;
 };
+
+// COUNT, multi-owner pixels (overlapping polygons, no edge in the pixel): the point's polygons
+// are exactly the record's owner set, so the point is counted once per record here and the
+// per-record counts are spread over the owner sets after the probe (k_multi_expand) — the
+// paper's aggregation plan for points: partial aggregates per canvas location, then combined
+// per polygon.  One global atomic per such point instead of one per (point, polygon).
+template <int MODE, class C>
+__device__ __forceinline__ void count_multi_owner(const Params& prm, C& c) {
+  if (!(MODE == kCountSmem || MODE == kCountGlobal) || prm.rec_cnt == nullptr) return;
+  if ((int)(c[0] | c[1] | c[2] | c[3]) >= 0) return;
+#pragma unroll
+  for (int q = 0; q < kNPT; ++q)
+    if ((c[q] >> 31) && ~c[q] >= prm.multi_base) {
+      atomicAdd(prm.rec_cnt + (~c[q] - prm.multi_base), 1u);
+      c[q] = 0u;
+    }
+}
 
 // COUNT with global counters, one hit of polygon `key`: the shared-memory count cache (direct
 // mapped; the first polygon to claim a slot keeps it for the CTA's lifetime, so hot polygons of
@@ -613,7 +632,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     return f;
   };
   // phase C of one batch: the sinks.  getxy(q): coordinates of point q of this thread.
-  auto process = [&](uint32_t base, const U4 c, auto getxy) {
+  auto process = [&](uint32_t base, U4 c, auto getxy) {
+    count_multi_owner<MODE>(prm, c);
     const uint32_t orc = c[0] | c[1] | c[2] | c[3];
     if (QUEUE) {
       // phase C1 (COUNT): boundary points -> warp queue (one smem atomic per lane that has any),
@@ -744,6 +764,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         }
       }
       // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
+      count_multi_owner<MODE>(prm, c);
       const uint32_t orc = c[0] | c[1] | c[2] | c[3];
       if (!QUEUE) {
         // phase C1 (COUNT, deferred): boundary points -> this CTA's deferral region (one smem
@@ -965,6 +986,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
         asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(slot + q * (T * 4)) : "memory");
         c[q] = v + 1u;                               // 0 none | owner + 1 | >= 2^31 record ~c
       }
+      count_multi_owner<MODE>(prm, c);
       const uint32_t orc = c[0] | c[1] | c[2] | c[3];
       if ((int)orc < 0) {
         uint32_t bnd = 0;
@@ -1356,6 +1378,22 @@ void keep_pool_memory() {
   cudaGetLastError();
 }
 
+// Spread the per-record counts of multi-owner pixels over their owner sets (see count_multi_owner).
+__global__ void __launch_bounds__(256) k_multi_expand(const CanvasDev* __restrict__ cvg, const unsigned int* __restrict__ rec_cnt,
+                                                     uint32_t multi_base, uint32_t num_multi, unsigned long long* counts) {
+  for (uint32_t i = blockIdx.x * 256 + threadIdx.x; i < num_multi; i += gridDim.x * 256) {
+    const unsigned int k = rec_cnt[i];
+    if (k == 0u) continue;
+    const int32_t term = cvg->recs[multi_base + i].term;
+    if (term >= 0) {
+      atomicAdd(counts + term, (unsigned long long)k);
+    } else if (term != kEmpty) {
+      const int2 g = cvg->set_rng[-2 - term];
+      for (int j = 0; j < g.y; ++j) atomicAdd(counts + cvg->sets[g.x + j], (unsigned long long)k);
+    }
+  }
+}
+
 template <int MODE, int COMPACT, int QUEUE, int KIND, int PIPE = 0>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
   const size_t smem = PIPE ? tiles_bytes_for(c->d.Wc, c->d.Hc) + ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes()
@@ -1367,6 +1405,15 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
   const int sms = device_sm_count();
   keep_pool_memory();
+  // COUNT over a canvas with multi-owner pixels: per-record counters (count_multi_owner)
+  constexpr bool kCnt = MODE == kCountSmem || MODE == kCountGlobal;
+  const uint32_t num_multi = kCnt && options().multi_agg ? (uint32_t)(c->num_records - c->num_runs) : 0u;
+  unsigned int* rec_cnt = nullptr;
+  if (num_multi > 0) {
+    e = cudaMallocAsync((void**)&rec_cnt, sizeof(unsigned int) * num_multi, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(rec_cnt, 0, sizeof(unsigned int) * num_multi, st);
+    if (e != cudaSuccess) return check_cuda(e, "multi-owner counters");
+  }
   // launches of fewer than 2^31 points (32-bit vector indices and point offsets)
   const int64_t kMax = (1ll << 31) - 64;
   for (int64_t off = 0; off < n; off += kMax) {
@@ -1424,6 +1471,8 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     }
     p.defer = dbuf;
     p.defer_xy = PIPE ? (uint32_t)options().defer_xy : 0u;
+    p.rec_cnt = rec_cnt;
+    p.multi_base = (uint32_t)c->num_runs;
     p.l2_frac = (float)options().l2_frac_pct * 0.01f;
     p.defer_cap = (uint32_t)per;
     p.defer_fill = dfill;
@@ -1476,7 +1525,18 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       e = cudaGetLastError();
     }
     if (scratch) cudaFreeAsync(scratch, st);
-    if (e != cudaSuccess) return check_cuda(e, "probe launch");
+    if (e != cudaSuccess) {
+      if (rec_cnt) cudaFreeAsync(rec_cnt, st);
+      return check_cuda(e, "probe launch");
+    }
+  }
+  if (rec_cnt) {
+    const int g = (int)std::min<int64_t>((int64_t)sms * 8, ((int64_t)num_multi + 255) / 256);
+    k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, rec_cnt, (uint32_t)c->num_runs, num_multi, base.o.counts);
+    count_launch();
+    e = cudaGetLastError();
+    cudaFreeAsync(rec_cnt, st);
+    if (e != cudaSuccess) return check_cuda(e, "multi-owner expand");
   }
   return SPADE_OK;
 }

@@ -105,3 +105,40 @@ def test_full_size_count_c5_one_gpu_shard(sp):
     idx = _sample(n, 300, 29)
     got = lab[torch.as_tensor(idx, device="cuda")].cpu().numpy().astype(np.int64)
     np.testing.assert_array_equal(got, _oracle_labels(w, idx + 3 * n))
+
+
+def test_full_size_overlap_heavy_ov(sp):
+    """NEXT(4)'s scenario: 1,000 overlapping stars (~32 polygons per point on average).  COUNT of
+    a 50M-point slice equals the histogram of its PAIRS output; sampled points' pairs equal the
+    oracle's; COUNT over the full 1B points equals the sum of its 50M-point slices."""
+    import torch
+    w = configs.ov()
+    n = w.n_points
+    cv = sp.Canvas(w.polys, max_dim=w.max_dim)
+    m = 50_000_000
+    xy = _device_points(w, m, start=7 * m)
+    counts = sp.join_count(cv, xy)
+    pt, pl = sp.join_pairs(cv, xy, point_id_base=7 * m, capacity=int(counts.sum()))
+    assert len(pt) == int(counts.sum())
+    assert torch.equal(torch.bincount(pl.long(), minlength=cv.num_polys), counts)
+    idx = _sample(m, 200, 31)
+    o = torch.argsort(pt)
+    pts, pls = pt[o], pl[o]
+    lo = torch.searchsorted(pts, torch.as_tensor(idx + 7 * m, device="cuda"))
+    hi = torch.searchsorted(pts, torch.as_tensor(idx + 7 * m, device="cuda"), right=True)
+    xs = gen.points_at(w.points, w.point_seed, idx + 7 * m)
+    opt, opl = oracle.join_pairs(xs, w.polys)
+    lo, hi = lo.cpu().numpy(), hi.cpu().numpy()
+    for k in range(len(idx)):
+        got = np.sort(pls[lo[k]:hi[k]].cpu().numpy().astype(np.int64))
+        np.testing.assert_array_equal(got, np.sort(opl[opt == k]))
+    del pt, pl, pts, pls, o
+    total = torch.zeros(cv.num_polys, dtype=torch.int64, device="cuda")
+    full = torch.zeros(cv.num_polys, dtype=torch.int64, device="cuda")
+    for s in range(0, n, 200_000_000):
+        xs_d = _device_points(w, min(200_000_000, n - s), start=s)
+        sp.join_count(cv, xs_d, total)
+        del xs_d
+    xy_full = _device_points(w, n)
+    sp.join_count(cv, xy_full, full)
+    assert torch.equal(total, full)

@@ -197,6 +197,15 @@ def test_host_streaming_pairs_chunk_overflow(spade):
     assert len(pt) > 2 * len(xy)
 
 
+def test_overlap_heavy_polygon_set(spade):
+    """1,000 overlapping stars (configs.ov, NEXT(4)'s scenario): ~32 polygons per point on average,
+    owner sets of dozens of polygons per pixel; all ops bit-exact against the oracle."""
+    w = configs.ov()
+    xy = gen.points_host(w.points, w.point_seed, 0, 30_000)
+    for md in (1024, 8192):
+        check_all(spade, w.polys, xy, max_dim=md, base=11)
+
+
 def test_invalid_arguments_are_reported(spade):
     import ctypes
     import torch
