@@ -234,6 +234,10 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  polygons, no edge in the pixel) once per pixel record and spreads the record
  *                  counts over the owner sets afterwards (the paper's partial-aggregate plan,
  *                  P:214), instead of one increment per (point, polygon)
+ *   "k_agg"        -1 (default, auto: owner-set entries > 1/2 per record) / 0 / 1: COUNT counts
+ *                  boundary points once per pixel record for the record's corner set K (spread
+ *                  over K afterwards) plus a +1 / -1 per polygon of odd edge parity, instead of
+ *                  merging K per point
  *   "host_chunk"   2^25 (default): points per staging chunk of the host-resident calls
  *                  (256 .. 2^28) */
 SPADE_API int spade_set_option(const char* name, int64_t value);

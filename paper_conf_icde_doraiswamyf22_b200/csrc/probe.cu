@@ -147,6 +147,7 @@ struct Params {
   float l2_frac;              // fraction of fine-canvas lines gathered with L2::evict_last
   unsigned int* rec_cnt;      // COUNT over overlapping polygons: points per multi-owner record, or null
   uint32_t multi_base;        // first multi-owner record id (records >= it have no edges)
+  unsigned int* kcnt;         // COUNT with K aggregation: points per boundary record, or null
   const int2* xy;
   int64_t n;
   int64_t head;               // points before the first 32-byte aligned one (0..3)
@@ -309,9 +310,50 @@ struct TermMerge {
 // Exact test for a point on the boundary (or multi-owner) pixel of record `rec` (packed layout:
 // spade_internal.cuh "Rec"): one 16-B record fetch, then the record's polygons, primitives and
 // masks from one contiguous blob.  emit(P) for every polygon containing the point, ascending.
+template <int KIND, int U, class Fin>
+__device__ __forceinline__ void pip_edges_rec(const CanvasDev* __restrict__ cv, int px, int py, const Rec r, Fin& fin);
+
 template <int KIND, int U = 1, class Emit>
 __device__ __forceinline__ void pip_eval_rec(const CanvasDev* __restrict__ cv, int px, int py, const Rec r, Emit&& emit) {
   TermMerge<Emit> fin(cv, r.term, emit);
+  pip_edges_rec<KIND, U>(cv, px, py, r, fin);
+  fin.rest();
+}
+
+// COUNT with K aggregation: the record's term set K is counted once per point in a per-record
+// counter (spread over K after the probe, like multi-owner pixels) and only the edge parity is
+// evaluated per point: polygon P with odd parity contributes -1 if P is in K (the point leaves
+// it) else +1.  Per point O(hit polygons) instead of O(|K|) (overlapping polygon sets).
+template <class Emit>
+struct DeltaFin {
+  const int32_t* sets;
+  int32_t term;
+  int tb, tn;
+  Emit& emit;
+  __device__ __forceinline__ DeltaFin(const CanvasDev* __restrict__ cv, int32_t t, Emit& e) : sets(cv->sets), term(t), tb(0), tn(0), emit(e) {
+    if (t < -1) { const int2 g = cv->set_rng[-2 - t]; tb = g.x; tn = g.y; }
+  }
+  __device__ __forceinline__ bool inK(int P) const {
+    if (term >= 0) return P == term;
+    int lo = 0, hi = tn;                         // sorted set: lower bound
+    while (lo < hi) { const int mid = (lo + hi) >> 1; if (__ldg(sets + tb + mid) < P) lo = mid + 1; else hi = mid; }
+    return lo < tn && __ldg(sets + tb + lo) == P;
+  }
+  __device__ __forceinline__ void operator()(int P, int par) { if (par) emit(P, inK(P) ? -1 : 1); }
+  __device__ __forceinline__ void mask(uint64_t m, const int32_t* __restrict__ rp) {
+    while (m) { const int k = __ffsll((long long)m) - 1; m &= m - 1; (*this)(__ldg(rp + k), 1); }
+  }
+};
+template <int KIND, int U = 1, class Emit>
+__device__ __forceinline__ void pip_count_delta(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, const Rec r,
+                                                unsigned int* __restrict__ kcnt, Emit&& emit) {
+  if (r.term != kEmpty) atomicAdd(kcnt + rec, 1u);
+  DeltaFin<Emit> fin(cv, r.term, emit);
+  pip_edges_rec<KIND, U>(cv, px, py, r, fin);
+}
+
+template <int KIND, int U, class Fin>
+__device__ __forceinline__ void pip_edges_rec(const CanvasDev* __restrict__ cv, int px, int py, const Rec r, Fin& fin) {
   const int ne = r.ecnt;
   if (ne > 0) {
     const int pc = (int)(r.pinfo & kRecPcnt);
@@ -339,7 +381,6 @@ __device__ __forceinline__ void pip_eval_rec(const CanvasDev* __restrict__ cv, i
         hit_grouped<KIND>(seg, (const uint64_t*)mb, ne, X, px, py, rp, fin);
     }
   }
-  fin.rest();
 }
 template <int KIND, int U = 1, class Emit>
 __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
@@ -440,14 +481,21 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
 // the streaming loop keeps a small register footprint.
 template <int MODE, int KIND>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const QEntry* wq,
-                                   int cnt, int lane, unsigned int* hist, uint32_t hstride, unsigned long long* counts) {
+                                   int cnt, int lane, unsigned int* hist, uint32_t hstride, unsigned long long* counts,
+                                   unsigned int* kcnt) {
   if (lane < cnt) {
     const QEntry e = wq[lane];
     const CanvasDev& cv = *cvg;
     const uint32_t fx = ((uint32_t)e.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)e.y - (uint32_t)cv.miny) >> cv.s;
     const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
     const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
-    pip_eval<KIND>(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
+    if (kcnt)
+      pip_count_delta<KIND>(cvg, e.x, e.y, ~c, cv.recs[~c], kcnt, [&](int q, int d) {
+        if (MODE == kCountSmem) atomicAdd(&hist[(uint32_t)q * hstride], (unsigned int)d);
+        else atomicAdd(counts + q, (unsigned long long)(long long)d);
+      });
+    else
+      pip_eval<KIND>(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
   }
 }
 
@@ -661,7 +709,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         if (qn >= 32) {
           do {
             if (MODE == kSelect || MODE == kPairs) drain_out(wqi + qn - 32, 32, (nvec - 1 - base) / (nctaid_x() * chunk));
-            else drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts);
+            else drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
             qn -= 32;
           } while (qn >= 32);
           __syncwarp();
@@ -815,7 +863,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
           int qn = s_qn[warp];
           if (qn >= 32) {
             do {
-              drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts);
+              drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
               qn -= 32;
             } while (qn >= 32);
             __syncwarp();
@@ -859,7 +907,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   }
   if (QUEUE && (MODE == kCountSmem || MODE == kCountGlobal)) {
     __syncwarp();
-    if (s_qn[warp] > 0) drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts);
+    if (s_qn[warp] > 0) drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
   }
   __syncthreads();
   if (!QUEUE && tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
@@ -869,7 +917,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   if (MODE == kCountSmem) {
     for (uint32_t i = tid; i < P; i += T) {
       unsigned long long sum = 0;
-      for (uint32_t k = 0; k < prm.hcopies; ++k) sum += hist[i * prm.hcopies + k];
+      for (uint32_t k = 0; k < prm.hcopies; ++k) sum += (unsigned long long)(long long)(int)hist[i * prm.hcopies + k];
       if (sum) atomicAdd(prm.o.counts + i, sum);
     }
   }
@@ -1033,7 +1081,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
   if (MODE == kCountSmem) {
     for (uint32_t i = tid; i < P; i += T) {
       unsigned long long sum = 0;
-      for (uint32_t k = 0; k < prm.hcopies; ++k) sum += hist[i * prm.hcopies + k];
+      for (uint32_t k = 0; k < prm.hcopies; ++k) sum += (unsigned long long)(long long)(int)hist[i * prm.hcopies + k];
       if (sum) atomicAdd(prm.o.counts + i, sum);
     }
   }
@@ -1115,7 +1163,7 @@ __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __r
 template <int MODE, int KIND>
 __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                   uint32_t cap, const unsigned int* __restrict__ fill, int nreg, Out o,
-                                                  int smem_hist, const int2* __restrict__ pxy) {
+                                                  int smem_hist, const int2* __restrict__ pxy, unsigned int* __restrict__ kcnt) {
   using BS = cub::BlockScan<int, 256>;
   __shared__ typename BS::TempStorage tmp;
   __shared__ unsigned long long s_gb;
@@ -1161,7 +1209,12 @@ __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict
     nrec = rec_of(nxt);
     const bool act = e.rec != kHole;
     const int64_t pid = o.id_base + (int64_t)e.pidx;
-    if (MODE == kCountSmem || MODE == kCountGlobal) {
+    if ((MODE == kCountSmem || MODE == kCountGlobal) && kcnt) {
+      if (act) pip_count_delta<KIND, 4>(cvg, e.x, e.y, e.rec, rc, kcnt, [&](int q, int d) {
+        if (sh) atomicAdd(&dh[q], (unsigned int)d);
+        else atomicAdd(o.counts + q, (unsigned long long)(long long)d);
+      });
+    } else if (MODE == kCountSmem || MODE == kCountGlobal) {
       if (sh) {
         if (act) pip_eval_rec<KIND, 4>(cvg, e.x, e.y, rc, [&](int q) { atomicAdd(&dh[q], 1u); });
       } else {
@@ -1200,7 +1253,7 @@ __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict
   if (sh) {
     __syncthreads();
     for (int q = threadIdx.x; q < P; q += 256)
-      if (dh[q]) atomicAdd(o.counts + q, (unsigned long long)dh[q]);
+      if (dh[q]) atomicAdd(o.counts + q, (unsigned long long)(long long)(int)dh[q]);
   }
 }
 
@@ -1414,6 +1467,21 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     if (e == cudaSuccess) e = cudaMemsetAsync(rec_cnt, 0, sizeof(unsigned int) * num_multi, st);
     if (e != cudaSuccess) return check_cuda(e, "multi-owner counters");
   }
+  // COUNT over heavily overlapping polygons (owner sets much larger than one polygon on average):
+  // boundary points counted per record for the term set K + per-point parity deltas
+  const int kagg_opt = options().k_agg;
+  const bool kagg = kCnt && c->num_runs > 0 &&
+                    (kagg_opt == 1 || (kagg_opt < 0 && 2 * c->num_set_entries > c->num_records));
+  unsigned int* kcnt = nullptr;
+  if (options().debug_defer)
+    fprintf(stderr, "[spade] records %lld (boundary %lld), set entries %lld, k_agg %d\n", (long long)c->num_records,
+            (long long)c->num_runs, (long long)c->num_set_entries, (int)kagg);
+  if (kagg) {
+    // every record: multi-owner records reach the exact-test paths too when multi_agg is off
+    e = cudaMallocAsync((void**)&kcnt, sizeof(unsigned int) * c->num_records, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(kcnt, 0, sizeof(unsigned int) * c->num_records, st);
+    if (e != cudaSuccess) return check_cuda(e, "boundary-record counters");
+  }
   // launches of fewer than 2^31 points (32-bit vector indices and point offsets)
   const int64_t kMax = (1ll << 31) - 64;
   for (int64_t off = 0; off < n; off += kMax) {
@@ -1473,6 +1541,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.defer_xy = PIPE ? (uint32_t)options().defer_xy : 0u;
     p.rec_cnt = rec_cnt;
     p.multi_base = (uint32_t)c->num_runs;
+    p.kcnt = kcnt;
     p.l2_frac = (float)options().l2_frac_pct * 0.01f;
     p.defer_cap = (uint32_t)per;
     p.defer_fill = dfill;
@@ -1500,7 +1569,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       if (!launched) {
         if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
         k_deferred<MODE, KIND><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh,
-                                                           PIPE && !p.defer_xy ? p.xy : nullptr);
+                                                           PIPE && !p.defer_xy ? p.xy : nullptr, kcnt);
       }
       count_launch();
       e = cudaGetLastError();
@@ -1527,7 +1596,19 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     if (scratch) cudaFreeAsync(scratch, st);
     if (e != cudaSuccess) {
       if (rec_cnt) cudaFreeAsync(rec_cnt, st);
+      if (kcnt) cudaFreeAsync(kcnt, st);
       return check_cuda(e, "probe launch");
+    }
+  }
+  if (kcnt) {
+    const int g = (int)std::min<int64_t>((int64_t)sms * 8, (c->num_records + 255) / 256);
+    k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, kcnt, 0u, (uint32_t)c->num_records, base.o.counts);
+    count_launch();
+    e = cudaGetLastError();
+    cudaFreeAsync(kcnt, st);
+    if (e != cudaSuccess) {
+      if (rec_cnt) cudaFreeAsync(rec_cnt, st);
+      return check_cuda(e, "boundary-record expand");
     }
   }
   if (rec_cnt) {

@@ -93,7 +93,7 @@ static int env_int(const char* name, int dflt) {
 Options& options() {
   static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
                    env_int("SPADE_CACHE_SLOTS", 4096), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
-                   env_int("SPADE_PIPE", -1), env_int("SPADE_DEFER_XY", 0), env_int("SPADE_L2_FRAC_PCT", 100), env_int("SPADE_MULTI_AGG", 1),
+                   env_int("SPADE_PIPE", -1), env_int("SPADE_DEFER_XY", 0), env_int("SPADE_L2_FRAC_PCT", 100), env_int("SPADE_MULTI_AGG", 1), env_int("SPADE_K_AGG", -1),
                    (int64_t)1 << 25};
   return o;
 }
@@ -490,6 +490,7 @@ int spade_set_option(const char* name, int64_t value) {
   else if (n == "defer_xy" && bit) o.defer_xy = (int)value;
   else if (n == "l2_frac_pct" && value >= 1 && value <= 100) o.l2_frac_pct = (int)value;
   else if (n == "multi_agg" && bit) o.multi_agg = (int)value;
+  else if (n == "k_agg" && (value == -1 || bit)) o.k_agg = (int)value;
   else if (n == "cache_slots" && (value == 0 || (value >= 1024 && value <= (1 << 16) && (value & (value - 1)) == 0)))
     o.cache_slots = (int)value;
   else if (n == "pipe" && (value == -1 || bit)) o.pipe = (int)value;

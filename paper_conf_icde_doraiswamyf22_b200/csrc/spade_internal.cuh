@@ -130,7 +130,7 @@ int device_sm_count();
 
 // probe-path options (spade_set_option; include/spade.h)
 struct Options {
-  int defer, count_global, global_queue, cache_slots, coop, debug_defer, pipe, defer_xy, l2_frac_pct, multi_agg;
+  int defer, count_global, global_queue, cache_slots, coop, debug_defer, pipe, defer_xy, l2_frac_pct, multi_agg, k_agg;
   int64_t host_chunk;  // points per staging chunk of the host-resident calls
 };
 Options& options();
