@@ -5,7 +5,7 @@
 # Usage (on the GPU box): bash tools/profile_round.sh <tag>    -> gpurun_out/<tag>_*
 T=${1:-prof}
 python bench.py > gpurun_out/${T}_bench_c3.json 2> gpurun_out/${T}_bench_c3.err
-for wl in c2 c4 c5 dj dj2 knn; do
+for wl in c2 c4 c5 dj dj2 knn ov; do
   python bench.py --workload $wl --no-e2e --steps 20 --warmup 3 --cpu-seconds 8 > gpurun_out/${T}_bench_$wl.json 2> gpurun_out/${T}_bench_$wl.err
 done
 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/${T}_launches_c3.csv \
