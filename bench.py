@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-parity", action="store_true", help="skip the oracle parity check on the sample")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU oracle sample time")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu/clocks)")
     ap.add_argument("--dense", action="store_true", help="force the dense fine-canvas layout (A/B runs)")
@@ -172,13 +173,15 @@ def cpu_oracle_rate(w, target_s, seed_offset=0):
         stride = max(1, w.n_points // m)
         xy = gen.points_at(w.points, w.point_seed, np.arange(m, dtype=np.int64) * stride + seed_offset)
         t0 = time.perf_counter()
-        _oracle_run(w, xy, nt)
+        counts = _oracle_run(w, xy, nt)
         dt = time.perf_counter() - t0
         what = (f"kNN (k={w.k}) by sorting all sampled points" if w.op == "knn" else
                 f"x {len(w.disks['r2'])} disks, brute force over all pairs")
         return {"value": m / dt, "unit": "points/s", "cores": 1 if w.op == "knn" else nt, "kind": "oracle",
                 "sample": f"{m} points = every {stride}-th global index of the workload's point stream, {what} "
-                          f"({dt:.1f} s)", "seconds": dt, "sum_counts": 0}
+                          f"({dt:.1f} s)", "seconds": dt, "sum_counts": 0,
+                "idx": np.arange(m, dtype=np.int64) * stride + seed_offset, "rate": m / dt,
+                "counts": None if w.op == "knn" else counts}
     idx = np.arange(0, 2000, dtype=np.int64) * 499 + seed_offset
     pilot = gen.points_at(w.points, w.point_seed, idx)
     t0 = time.perf_counter()
@@ -194,7 +197,8 @@ def cpu_oracle_rate(w, target_s, seed_offset=0):
     return {"value": m / dt, "unit": "points/s", "cores": nt, "kind": "oracle",
             "sample": f"{m} points = every {stride}-th global index of the workload's point stream, "
                       f"x {len(w.polys['poly_ring_off']) - 1} polygons, brute force over all pairs "
-                      f"({dt:.1f} s)", "seconds": dt, "sum_counts": int(counts.sum())}
+                      f"({dt:.1f} s)", "seconds": dt, "sum_counts": int(counts.sum()),
+            "idx": idx, "counts": counts, "rate": m / dt}
 
 
 def cpu_rtree_rate(w, target_s):
@@ -217,6 +221,50 @@ def cpu_rtree_rate(w, target_s):
     return {"value": m / dt, "unit": "points/s", "cores": nt, "kind": "rtree",
             "sample": f"{m} points = every {stride}-th global index, STR R-tree over "
                       f"{len(w.polys['poly_ring_off']) - 1} polygon bboxes + exact predicate ({dt:.1f} s)"}
+
+
+def parity_check(w, cv, sp, idx, oracle_counts=None, rate=None, pairs_seconds=5.0):
+    """The GPU path on the oracle's sample ("the GPU is run on the same
+    subsample indices for parity"): per-polygon counts of the whole sample (the oracle's, from
+    the timed cpu_baseline run when given) and the sorted (point, polygon) pairs of a prefix sized
+    to ~pairs_seconds of oracle time, bit-exact.  Inputs regenerated from the shared seeded
+    generator; expected values only from oracle/."""
+    import numpy as np
+    import torch
+    import gen
+    import oracle
+    xy = gen.points_at(w.points, w.point_seed, idx)
+    xy_d = torch.as_tensor(xy).cuda()
+    res = {"sample": int(len(idx)), "indices": f"global indices {int(idx[0])}, {int(idx[1]) if len(idx) > 1 else ''}, ... "
+                                                 f"(stride {int(idx[1] - idx[0]) if len(idx) > 1 else 0})"}
+    if getattr(w, "op", "") == "knn":
+        xy, xy_d = xy[:2_000_000], xy_d[:2_000_000]
+        res["sample"] = int(len(xy))
+        k = min(w.k, len(xy))
+        gi, gd = sp.knn(xy_d, w.query, k)
+        oi, od = oracle.knn(xy, w.query, k)
+        res.update({"checked": f"kNN (k={k}) of the sample: ids and squared distances in order",
+                    "ok": bool(np.array_equal(gi.cpu().numpy(), oi) and np.array_equal(gd.cpu().numpy(), od))})
+        return res
+    is_dist = hasattr(w, "disks")
+    count_o = (lambda x: oracle.disk_join_count(x, w.disks)) if is_dist else (lambda x: oracle.join_count(x, w.polys))
+    pairs_o = (lambda x: oracle.disk_join_pairs(x, w.disks)) if is_dist else (lambda x: oracle.join_pairs(x, w.polys))
+    if oracle_counts is None:
+        oracle_counts = count_o(xy)
+    gc = sp.join_count(cv, xy_d).cpu().numpy()
+    counts_ok = bool(np.array_equal(gc, oracle_counts))
+    kp = len(idx) if rate is None else int(max(200, min(len(idx), rate * pairs_seconds)))
+    opt, opl = pairs_o(xy[:kp])
+    cap = int(sp.join_count(cv, xy_d[:kp]).sum())
+    gpt, gpl = sp.join_pairs(cv, xy_d[:kp], capacity=max(cap, 1))
+    gpt, gpl = gpt.cpu().numpy().astype(np.int64), gpl.cpu().numpy().astype(np.int64)
+    o = np.lexsort((gpl, gpt))
+    pairs_ok = bool(np.array_equal(gpt[o], opt) and np.array_equal(gpl[o], opl))
+    res.update({"checked": f"per-{'disk' if is_dist else 'polygon'} COUNT of all {len(idx)} sample points; "
+                           f"sorted (point, {'disk' if is_dist else 'polygon'}) pairs of the first {kp}",
+                "counts_equal": counts_ok, "pairs_sample": kp, "pairs": int(len(opt)), "pairs_equal": pairs_ok,
+                "ok": counts_ok and pairs_ok})
+    return res
 
 
 def run_reference(a):
@@ -477,9 +525,19 @@ def main():
         cb = cpu_oracle_rate(w, a.cpu_seconds)
         cb.pop("seconds", None)
         cb.pop("sum_counts", None)
+        idx, ocounts, rate = cb.pop("idx"), cb.pop("counts", None), cb.pop("rate")
         line["cpu_baseline"] = cb
         if not is_dist:
             line["cpu_rtree_baseline"] = cpu_rtree_rate(w, a.cpu_seconds / 2)
+        if not a.no_parity:
+            line["parity"] = parity_check(w, cv, sp, idx, ocounts, rate)
+    elif rank == 0 and not a.profile and not a.no_parity:
+        # N > 1 (or no CPU baseline): the parity check alone, on a small strided sample of the
+        # global stream (all ranks' points), rank 0
+        import numpy as np
+        m = 2000 if w.name.startswith("c5") else 20000
+        stride = max(1, (n * ws) // m)
+        line["parity"] = parity_check(w, cv, sp, np.arange(m, dtype=np.int64) * stride + 1, None, None)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if ws > 1:

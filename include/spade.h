@@ -103,7 +103,8 @@ SPADE_API int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off
 SPADE_API int spade_build_disk_canvas(const int32_t* center_xy, const int64_t* r2, int32_t num_disks,
                             const spade_canvas_params* prm, spade_stream_t stream, spade_canvas** out);
 
-/* Release a canvas (NULL is a no-op).  Synchronises the device. */
+/* Release a canvas (NULL is a no-op).  Synchronises the canvas's device.  Every call taking a
+ * canvas runs on the device the canvas was built on (made current for the call and restored). */
 SPADE_API void spade_canvas_free(spade_canvas* c);
 
 /* Canvas statistics for reports: fine canvas W x H at 2^log2_pixel units per pixel; coarse
@@ -113,6 +114,13 @@ SPADE_API void spade_canvas_free(spade_canvas* c);
 SPADE_API int spade_canvas_info(const spade_canvas* c, int32_t* W, int32_t* H, int32_t* log2_pixel,
                       int32_t* Wc, int32_t* Hc, int32_t* log2_tile,
                       int64_t* num_runs, int64_t* num_run_edges, double* mixed_tile_frac);
+
+/* 64-bit checksum of everything the probe reads from the canvas (geometry, fine / compact /
+ * coarse levels, records, primitive blobs, owner sets), written to *out (HOST).  Equal polygon
+ * arrays give equal checksums on any device (the build is deterministic); ranks that replicate a
+ * canvas compare them (multi-GPU is the paper's future work).
+ * Synchronises `stream`.  Errors: INVALID_ARG (NULL), CUDA, OOM. */
+SPADE_API int spade_canvas_checksum(const spade_canvas* c, uint64_t* out, spade_stream_t stream);
 
 /* Aggregation: per-polygon COUNT of the points of xy[0..n) inside each polygon (P:214,
  * Sec. 5.2, "aggregation plan 2" for points: partial aggregates without materialising the join).
@@ -239,7 +247,17 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  over K afterwards) plus a +1 / -1 per polygon of odd edge parity, instead of
  *                  merging K per point
  *   "host_chunk"   2^25 (default): points per staging chunk of the host-resident calls
- *                  (256 .. 2^28) */
+ *                  (256 .. 2^28)
+ *   "max_launch_points"  2^31 - 64 (default, the maximum): points per probe sub-launch; a call
+ *                  with more points runs several sub-launches (each < 2^31 points: 32-bit point
+ *                  offsets and per-record counters; the counters are spread over the owner sets
+ *                  after every sub-launch).  Small values (>= 256) exercise the split in tests.
+ *   "defer_budget_mb"  4096 (default): device scratch per sub-launch for deferred boundary
+ *                  points (16 B per reserved entry; reserved: (2 fb + 4%) of the points, fb = the
+ *                  canvas's boundary-pixel fraction).  Calls whose reservation would exceed it
+ *                  are cut into more sub-launches, so the peak scratch of spade_join_count /
+ *                  spade_select / spade_join_pairs is <= this budget + ~0.2 GB of output
+ *                  overflow and compaction tables, whatever n is (64 .. 2^20). */
 SPADE_API int spade_set_option(const char* name, int64_t value);
 
 /* Number of kernels this library has launched in this process (for the bench's gpu_launches). */

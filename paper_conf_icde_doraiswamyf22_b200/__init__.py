@@ -67,6 +67,8 @@ def load(path: str | None = None):
     lib.spade_canvas_free.restype = None
     lib.spade_canvas_info.argtypes = [P] + [ctypes.POINTER(i32)] * 6 + [ctypes.POINTER(i64)] * 2 + [ctypes.POINTER(ctypes.c_double)]
     lib.spade_canvas_info.restype = ctypes.c_int
+    lib.spade_canvas_checksum.argtypes = [P, ctypes.POINTER(ctypes.c_uint64), P]
+    lib.spade_canvas_checksum.restype = ctypes.c_int
     lib.spade_join_count.argtypes = [P, P, i64, P, P]
     lib.spade_join_count.restype = ctypes.c_int
     lib.spade_select.argtypes = [P, P, i64, i64, P, i64, ctypes.POINTER(i64), P]
@@ -101,7 +103,8 @@ def load(path: str | None = None):
     return lib
 
 
-EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canvas_free", "spade_canvas_info", "spade_join_count",
+EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canvas_free", "spade_canvas_info",
+                    "spade_canvas_checksum", "spade_join_count",
                     "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_select_host", "spade_join_pairs_host", "spade_knn_histogram",
                     "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_set_option", "spade_launch_count",
                     "spade_status_string", "spade_last_error"]
@@ -136,6 +139,48 @@ def _dev(a, dtype, shape_last=None):
     return t
 
 
+def _dev_out(t, dtype, n: int, name: str, device=None):
+    """A caller-supplied DEVICE output buffer: must be a contiguous CUDA tensor of `dtype` with
+    at least n elements (on `device` if given); the C side writes through its raw pointer."""
+    torch = _torch()
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor")
+    if t.dtype != dtype:
+        raise ValueError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    if t.numel() < n:
+        raise ValueError(f"{name} holds {t.numel()} elements, needs >= {n}")
+    if device is not None and t.device != device:
+        raise ValueError(f"{name} is on {t.device}, the canvas on {device}")
+    return t
+
+
+def _host_buf(a, dtype, n: int, name: str):
+    """A caller-supplied HOST buffer (numpy array or CPU tensor): dtype, C-contiguous, writeable,
+    >= n elements; returns its address."""
+    if hasattr(a, "data_ptr"):
+        torch = _torch()
+        if a.is_cuda:
+            raise ValueError(f"{name} must be a host (CPU) tensor")
+        if a.dtype != {np.int64: torch.int64, np.int32: torch.int32}[dtype]:
+            raise ValueError(f"{name} must be {np.dtype(dtype).name}, got {a.dtype}")
+        if not a.is_contiguous():
+            raise ValueError(f"{name} must be contiguous")
+        if a.numel() < n:
+            raise ValueError(f"{name} holds {a.numel()} elements, needs >= {n}")
+        return a.data_ptr()
+    if not isinstance(a, np.ndarray):
+        raise ValueError(f"{name} must be a numpy array or a CPU tensor")
+    if a.dtype != np.dtype(dtype):
+        raise ValueError(f"{name} must be {np.dtype(dtype).name}, got {a.dtype}")
+    if not a.flags.c_contiguous or not a.flags.writeable:
+        raise ValueError(f"{name} must be C-contiguous and writeable")
+    if a.size < n:
+        raise ValueError(f"{name} holds {a.size} elements, needs >= {n}")
+    return a.ctypes.data
+
+
 def set_option(name: str, value: int) -> None:
     """Probe-path tuning option (include/spade.h spade_set_option); results never depend on it."""
     _check(load().spade_set_option(name.encode(), int(value)), f"set_option({name})")
@@ -152,6 +197,7 @@ class Canvas:
     def __init__(self, polys, log2_pixel: int = -1, max_dim: int = 4096, dense: bool = False, stream=None):
         torch = _torch()
         lib = load()
+        self.device = torch.device("cuda", torch.cuda.current_device())
         if polys is None:                    # filled in by Canvas.disks
             self._h, self._lib, self.num_polys = None, lib, 0
             return
@@ -217,19 +263,33 @@ class Canvas:
             pass
 
 
-def _points(xy):
+def canvas_checksum(canvas: Canvas, stream=None) -> int:
+    """64-bit checksum of the canvas arrays (spade_canvas_checksum): equal polygon sets give equal
+    checksums on every rank (the replicated-canvas check of distributed.canvas_checksums_agree)."""
+    h = ctypes.c_uint64()
+    _check(load().spade_canvas_checksum(canvas.handle, ctypes.byref(h), _stream(stream)), "spade_canvas_checksum")
+    return int(h.value)
+
+
+def _points(xy, device=None):
     torch = _torch()
     if not (isinstance(xy, torch.Tensor) and xy.is_cuda and xy.dtype == torch.int32 and xy.is_contiguous()):
-        xy = _dev(xy, torch.int32, 2)
+        xy = _dev(xy, torch.int32, 2) if device is None else \
+            (torch.as_tensor(xy) if not isinstance(xy, torch.Tensor) else xy).to(device=device, dtype=torch.int32).contiguous()
+    if device is not None and xy.device != device:
+        raise ValueError(f"points are on {xy.device}, the canvas on {device}")
+    if xy.numel() % 2:
+        raise ValueError("points must be (n, 2) int32 coordinates")
     return xy, xy.numel() // 2
 
 
 def join_count(canvas: Canvas, xy, counts=None, stream=None):
     """Per-polygon COUNT (int64[P] CUDA tensor); accumulates into `counts` if given."""
     torch = _torch()
-    xy, n = _points(xy)
+    xy, n = _points(xy, canvas.device)
     if counts is None:
-        counts = torch.zeros(canvas.num_polys, dtype=torch.int64, device="cuda")
+        counts = torch.zeros(canvas.num_polys, dtype=torch.int64, device=canvas.device)
+    _dev_out(counts, torch.int64, canvas.num_polys, "counts", canvas.device)
     rc = load().spade_join_count(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n,
                                  ctypes.c_void_p(counts.data_ptr()), _stream(stream))
     _check(rc, "spade_join_count")
@@ -241,11 +301,14 @@ def select(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None = No
     capacity=None uses n_max = n (1-pass Map); a too-small capacity retries once with the
     reported size (2-pass Map).  `out` (int64 CUDA, >= capacity) avoids the allocation."""
     torch = _torch()
-    xy, n = _points(xy)
+    xy, n = _points(xy, canvas.device)
     cap = n if capacity is None else capacity
+    if out is not None:
+        _dev_out(out, torch.int64, 0, "out", canvas.device)
     for attempt in range(2):
         if out is None or attempt > 0 or out.numel() < max(cap, 1):
-            out = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
+            out = torch.empty(max(cap, 1), dtype=torch.int64, device=canvas.device)
+        _dev_out(out, torch.int64, cap, "out", canvas.device)
         n_out = ctypes.c_int64()
         rc = load().spade_select(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n, point_id_base,
                                  ctypes.c_void_p(out.data_ptr()), cap, ctypes.byref(n_out), _stream(stream))
@@ -261,14 +324,19 @@ def join_pairs(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None 
     """(point_ids int64, poly_ids int32) CUDA tensors, order unspecified.  `out` = (pt, pl)
     preallocated CUDA tensors (>= capacity) avoids the allocation."""
     torch = _torch()
-    xy, n = _points(xy)
+    xy, n = _points(xy, canvas.device)
     cap = n if capacity is None else capacity
+    if out is not None:
+        _dev_out(out[0], torch.int64, 0, "out[0]", canvas.device)
+        _dev_out(out[1], torch.int32, 0, "out[1]", canvas.device)
     for attempt in range(2):
         if out is not None and attempt == 0 and out[0].numel() >= max(cap, 1) and out[1].numel() >= max(cap, 1):
             pt, pl = out
         else:
-            pt = torch.empty(max(cap, 1), dtype=torch.int64, device="cuda")
-            pl = torch.empty(max(cap, 1), dtype=torch.int32, device="cuda")
+            pt = torch.empty(max(cap, 1), dtype=torch.int64, device=canvas.device)
+            pl = torch.empty(max(cap, 1), dtype=torch.int32, device=canvas.device)
+        _dev_out(pt, torch.int64, cap, "out[0]", canvas.device)
+        _dev_out(pl, torch.int32, cap, "out[1]", canvas.device)
         n_out = ctypes.c_int64()
         rc = load().spade_join_pairs(canvas.handle, ctypes.c_void_p(xy.data_ptr()), n, point_id_base,
                                      ctypes.c_void_p(pt.data_ptr()), ctypes.c_void_p(pl.data_ptr()), cap,
@@ -284,23 +352,20 @@ def join_pairs(canvas: Canvas, xy, point_id_base: int = 0, capacity: int | None 
 def join_count_host(canvas: Canvas, xy_host, counts_host=None, stream=None) -> np.ndarray:
     """COUNT over HOST-resident points (numpy array or pinned CPU tensor); returns int64 numpy."""
     lib = load()
-    if hasattr(xy_host, "data_ptr"):      # torch CPU tensor (pinned for full bandwidth)
-        assert not xy_host.is_cuda and xy_host.is_contiguous()
-        ptr, n = xy_host.data_ptr(), xy_host.numel() // 2
-    else:
-        xy_host = np.ascontiguousarray(xy_host, dtype=np.int32)
-        ptr, n = xy_host.ctypes.data, xy_host.size // 2
+    keep, ptr, n = _host_points(xy_host)
     if counts_host is None:
         counts_host = np.zeros(canvas.num_polys, dtype=np.int64)
-    rc = lib.spade_join_count_host(canvas.handle, ctypes.c_void_p(ptr), n,
-                                   counts_host.ctypes.data_as(ctypes.c_void_p), _stream(stream))
+    cptr = _host_buf(counts_host, np.int64, canvas.num_polys, "counts_host")
+    rc = lib.spade_join_count_host(canvas.handle, ctypes.c_void_p(ptr), n, ctypes.c_void_p(cptr), _stream(stream))
     _check(rc, "spade_join_count_host")
     return counts_host
 
 
 def _host_points(xy_host):
     if hasattr(xy_host, "data_ptr"):      # torch CPU tensor (pinned for full bandwidth)
-        assert not xy_host.is_cuda and xy_host.is_contiguous()
+        import torch
+        if xy_host.is_cuda or not xy_host.is_contiguous() or xy_host.dtype != torch.int32 or xy_host.numel() % 2:
+            raise ValueError("host points must be a contiguous (n, 2) int32 CPU tensor")
         return xy_host, xy_host.data_ptr(), xy_host.numel() // 2
     xy_host = np.ascontiguousarray(xy_host, dtype=np.int32)
     return xy_host, xy_host.ctypes.data, xy_host.size // 2
@@ -310,11 +375,10 @@ def _host_out(out, cap, dtype):
     """Caller's host output array (numpy or CPU tensor, pinned for full bandwidth) if it holds
     `cap` elements, else a new numpy array; returns (array, address)."""
     if out is not None:
-        if hasattr(out, "data_ptr"):
-            assert not out.is_cuda and out.is_contiguous() and out.numel() >= cap
-            return out, out.data_ptr()
-        if out.size >= cap:
-            return out, out.ctypes.data
+        size = out.numel() if hasattr(out, "data_ptr") else np.asarray(out).size
+        if size >= cap:
+            return out, _host_buf(out, dtype, cap, "out")
+        _host_buf(out, dtype, 0, "out")            # type errors are reported even when too small
     a = np.empty(max(cap, 1), dtype=dtype)
     return a, a.ctypes.data
 

@@ -1021,6 +1021,9 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   c->num_run_edges = LM;
   c->num_set_entries = M + KT;
   c->mixed_tile_frac = (double)h_mixed / ((double)Wc * Hc);
+  c->num_set_ranges = NG + NK;
+  c->cfine_elems = compact ? (h_mixed << (2 * b)) : 0;
+  c->coarse_elems = NT1;
   CanvasDev& d = c->d;
   d.minx = (int32_t)g.minx; d.miny = (int32_t)g.miny;
   d.extw = (uint32_t)ew; d.exth = (uint32_t)eh;
@@ -1033,6 +1036,60 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
   if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));
   *out = c;
+  return SPADE_OK;
+}
+
+// ---- canvas checksum (replicated-canvas check across ranks) -------------------
+// Sum over the 32-bit words w_i of an array of mix(salt, i, w_i) mod 2^64: order-independent, so
+// the atomic accumulation is deterministic; any changed word changes the sum (up to 2^-64).
+__host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+__global__ void k_hash(const uint32_t* __restrict__ w, int64_t n, uint64_t salt, unsigned long long* __restrict__ acc) {
+  uint64_t h = 0;
+  for (int64_t i = blockIdx.x * (int64_t)kBT + threadIdx.x; i < n; i += (int64_t)gridDim.x * kBT)
+    h += mix64(salt ^ mix64((uint64_t)i) ^ ((uint64_t)w[i] << 17));
+  using BR = cub::BlockReduce<unsigned long long, kBT>;
+  __shared__ typename BR::TempStorage tmp;
+  const unsigned long long r = BR(tmp).Sum((unsigned long long)h);
+  if (threadIdx.x == 0 && r) atomicAdd(acc, r);
+}
+
+int canvas_checksum(const spade_canvas* c, uint64_t* out, cudaStream_t st) {
+  uint64_t h = mix64(0x5ADEull ^ (uint64_t)c->d.num_polys ^ ((uint64_t)c->d.kind << 40));
+  if (!c->empty) {
+    const CanvasDev& d = c->d;
+    const int64_t hdr[] = {d.minx, d.miny, d.extw, d.exth, d.s, d.W, d.H, d.b, d.Wc, d.Hc, d.compact, d.mix_min,
+                           c->num_runs, c->num_records, c->num_run_edges, c->num_set_entries, c->num_set_ranges};
+    for (int64_t v : hdr) h = mix64(h ^ (uint64_t)v);
+    unsigned long long* acc = nullptr;
+    cudaError_t e = cudaMallocAsync((void**)&acc, sizeof(unsigned long long), st);
+    if (e != cudaSuccess) return check_cuda(e, "spade_canvas_checksum");
+    e = cudaMemsetAsync(acc, 0, sizeof(unsigned long long), st);
+    struct A { const void* p; int64_t words; };
+    const A arrs[] = {{c->fine, (int64_t)d.W * d.H}, {c->cfine, c->cfine_elems}, {c->coarse, (c->coarse_elems + 1) / 2},
+                      {c->recs, c->num_records * (int64_t)(sizeof(Rec) / 4)}, {c->blob, c->blob_bytes / 4},
+                      {c->sets, c->num_set_entries}, {c->set_rng, 2 * c->num_set_ranges}};
+    uint64_t salt = 1;
+    for (const A& a : arrs) {
+      if (e == cudaSuccess && a.p && a.words > 0) {
+        k_hash<<<grid_for(a.words), kBT, 0, st>>>((const uint32_t*)a.p, a.words, mix64(salt), acc);
+        count_launch();
+        e = cudaGetLastError();
+      }
+      ++salt;
+    }
+    unsigned long long r = 0;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&r, acc, sizeof(r), cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    cudaFreeAsync(acc, st);
+    if (e != cudaSuccess) return check_cuda(e, "spade_canvas_checksum");
+    h = mix64(h ^ (uint64_t)r);
+  }
+  *out = h;
   return SPADE_OK;
 }
 

@@ -25,6 +25,7 @@
 #include <cstdlib>
 #include <vector>
 #include <cstdio>
+#include <atomic>
 #include <cub/block/block_scan.cuh>
 #include <cub/block/block_radix_sort.cuh>
 #include <cub/block/block_reduce.cuh>
@@ -596,7 +597,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   }
 
   const Vec4* vp = (const Vec4*)(prm.xy + prm.head);
-  const uint32_t nvec = (uint32_t)prm.nvec;      // launches hold < 2^31 points
+  const uint32_t nvec = (uint32_t)prm.nvec;      // sub-launches hold < 2^31 points (launch())
   const uint32_t chunk = (uint32_t)T;
   const uint32_t minx = (uint32_t)cv.minx, miny = (uint32_t)cv.miny;
   const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
@@ -1417,12 +1418,13 @@ __global__ void __launch_bounds__(1024) k_move(Out o, const long long* __restric
 
 // Stream-ordered scratch comes from the device's default memory pool; by default the pool hands
 // memory back to the driver at every synchronisation, which made each call re-map its scratch.
+// Set once per device (the caller's current device, which the entry points switch to the canvas's).
 void keep_pool_memory() {
-  static bool done = false;
-  if (done) return;
-  done = true;
+  static std::atomic<uint64_t> done{0};
   int dev = 0;
   cudaGetDevice(&dev);
+  const uint64_t bit = 1ull << (dev & 63);
+  if (done.fetch_or(bit) & bit) return;
   cudaMemPool_t pool;
   if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
     uint64_t thr = 16ull << 30;
@@ -1447,6 +1449,13 @@ __global__ void __launch_bounds__(256) k_multi_expand(const CanvasDev* __restric
   }
 }
 
+// Stream-ordered device scratch freed on every exit path (errors included).
+struct ScratchGuard {
+  void* p = nullptr;
+  cudaStream_t st = nullptr;
+  ~ScratchGuard() { if (p) cudaFreeAsync(p, st); }
+};
+
 template <int MODE, int COMPACT, int QUEUE, int KIND, int PIPE = 0>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
   const size_t smem = PIPE ? tiles_bytes_for(c->d.Wc, c->d.Hc) + ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes()
@@ -1461,10 +1470,14 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
   // COUNT over a canvas with multi-owner pixels: per-record counters (count_multi_owner)
   constexpr bool kCnt = MODE == kCountSmem || MODE == kCountGlobal;
   const uint32_t num_multi = kCnt && options().multi_agg ? (uint32_t)(c->num_records - c->num_runs) : 0u;
+  ScratchGuard rec_g, kcnt_g;
+  rec_g.st = kcnt_g.st = st;
   unsigned int* rec_cnt = nullptr;
   if (num_multi > 0) {
     e = cudaMallocAsync((void**)&rec_cnt, sizeof(unsigned int) * num_multi, st);
-    if (e == cudaSuccess) e = cudaMemsetAsync(rec_cnt, 0, sizeof(unsigned int) * num_multi, st);
+    if (e != cudaSuccess) return check_cuda(e, "multi-owner counters");
+    rec_g.p = rec_cnt;
+    e = cudaMemsetAsync(rec_cnt, 0, sizeof(unsigned int) * num_multi, st);
     if (e != cudaSuccess) return check_cuda(e, "multi-owner counters");
   }
   // COUNT over heavily overlapping polygons (owner sets much larger than one polygon on average):
@@ -1479,11 +1492,44 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
   if (kagg) {
     // every record: multi-owner records reach the exact-test paths too when multi_agg is off
     e = cudaMallocAsync((void**)&kcnt, sizeof(unsigned int) * c->num_records, st);
-    if (e == cudaSuccess) e = cudaMemsetAsync(kcnt, 0, sizeof(unsigned int) * c->num_records, st);
+    if (e != cudaSuccess) return check_cuda(e, "boundary-record counters");
+    kcnt_g.p = kcnt;
+    e = cudaMemsetAsync(kcnt, 0, sizeof(unsigned int) * c->num_records, st);
     if (e != cudaSuccess) return check_cuda(e, "boundary-record counters");
   }
-  // launches of fewer than 2^31 points (32-bit vector indices and point offsets)
-  const int64_t kMax = (1ll << 31) - 64;
+  // The per-record counters are uint32: they are spread over the owner sets (and cleared) after
+  // every sub-launch, each of which holds < 2^31 points, so no counter can wrap whatever n is.
+  auto expand = [&](bool clear) -> int {
+    if (kcnt) {
+      const int g = (int)std::min<int64_t>((int64_t)sms * 8, (c->num_records + 255) / 256);
+      k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, kcnt, 0u, (uint32_t)c->num_records, base.o.counts);
+      count_launch();
+      cudaError_t e2 = cudaGetLastError();
+      if (e2 == cudaSuccess && clear) e2 = cudaMemsetAsync(kcnt, 0, sizeof(unsigned int) * c->num_records, st);
+      if (e2 != cudaSuccess) return check_cuda(e2, "boundary-record expand");
+    }
+    if (rec_cnt) {
+      const int g = (int)std::min<int64_t>((int64_t)sms * 8, ((int64_t)num_multi + 255) / 256);
+      k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, rec_cnt, (uint32_t)c->num_runs, num_multi, base.o.counts);
+      count_launch();
+      cudaError_t e2 = cudaGetLastError();
+      if (e2 == cudaSuccess && clear) e2 = cudaMemsetAsync(rec_cnt, 0, sizeof(unsigned int) * num_multi, st);
+      if (e2 != cudaSuccess) return check_cuda(e2, "multi-owner expand");
+    }
+    return SPADE_OK;
+  };
+  // Sub-launches of fewer than 2^31 points (32-bit vector indices, point offsets and per-record
+  // counters).  Deferral regions are sized from the canvas's boundary-pixel fraction fb (points
+  // are not uniform, so 2 fb + 4%, at most all points; overflowing points are tested in place),
+  // 16 B per entry; a sub-launch is also cut so that its regions stay within the deferral budget
+  // (spade_set_option "defer_budget_mb"), which bounds the scratch for boundary-heavy canvases.
+  const double fb = (double)c->num_runs / ((double)c->d.W * (double)c->d.H);
+  const double frac = std::min(1.0, 2.0 * fb + 0.04);
+  int64_t kMax = std::min<int64_t>((1ll << 31) - 64, options().max_launch_points);
+  if (!QUEUE) {
+    const double budget = (double)options().defer_budget_mb * (1 << 20);
+    kMax = std::min<int64_t>(kMax, std::max<int64_t>(1 << 16, (int64_t)(budget / (16.0 * frac))));
+  }
   for (int64_t off = 0; off < n; off += kMax) {
     const int64_t m = std::min(kMax, n - off);
     Params p = base;
@@ -1495,10 +1541,6 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.o.id_base = base.o.id_base + off;
     const int64_t chunks = (p.nvec + kT - 1) / kT;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(std::min(sms, kMaxHoles / kNW), chunks));
-    // deferral regions sized from the canvas's boundary-pixel fraction fb (points are not uniform,
-    // so 2 fb + 4%, at most all points); overflowing points are tested in place (slow, rare)
-    const double fb = (double)c->num_runs / ((double)c->d.W * (double)c->d.H);
-    const double frac = std::min(1.0, 2.0 * fb + 0.04);
     const int64_t per = QUEUE ? 0 : std::min<int64_t>(std::max<int64_t>((int64_t)(frac * (double)m / grid) + 64, 1024),
                                                        (int64_t)1 << 26);
     // SELECT/PAIRS: warp output chunks of K slots (about 1/16 of a warp's points, 256..2048),
@@ -1518,10 +1560,13 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
                     kOut ? 8 * (size_t)(kMaxHoles + 1) + sizeof(FixMeta) : 0};
     size_t total_sz = 0, offs[9];
     for (int i = 0; i < 9; ++i) { offs[i] = total_sz; total_sz += (sz[i] + 255) & ~(size_t)255; }
+    ScratchGuard scr;
+    scr.st = st;
     unsigned char* scratch = nullptr;
     if (total_sz > 0) {
       e = cudaMallocAsync((void**)&scratch, total_sz, st);
       if (e != cudaSuccess) return check_cuda(e, "probe scratch");
+      scr.p = scratch;
     }
     DEntry* dbuf = QUEUE ? nullptr : (DEntry*)(scratch + offs[0]);
     unsigned int* dfill = QUEUE ? nullptr : (unsigned int*)(scratch + offs[1]);
@@ -1593,31 +1638,9 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       count_launch();
       e = cudaGetLastError();
     }
-    if (scratch) cudaFreeAsync(scratch, st);
-    if (e != cudaSuccess) {
-      if (rec_cnt) cudaFreeAsync(rec_cnt, st);
-      if (kcnt) cudaFreeAsync(kcnt, st);
-      return check_cuda(e, "probe launch");
-    }
-  }
-  if (kcnt) {
-    const int g = (int)std::min<int64_t>((int64_t)sms * 8, (c->num_records + 255) / 256);
-    k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, kcnt, 0u, (uint32_t)c->num_records, base.o.counts);
-    count_launch();
-    e = cudaGetLastError();
-    cudaFreeAsync(kcnt, st);
-    if (e != cudaSuccess) {
-      if (rec_cnt) cudaFreeAsync(rec_cnt, st);
-      return check_cuda(e, "boundary-record expand");
-    }
-  }
-  if (rec_cnt) {
-    const int g = (int)std::min<int64_t>((int64_t)sms * 8, ((int64_t)num_multi + 255) / 256);
-    k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, rec_cnt, (uint32_t)c->num_runs, num_multi, base.o.counts);
-    count_launch();
-    e = cudaGetLastError();
-    cudaFreeAsync(rec_cnt, st);
-    if (e != cudaSuccess) return check_cuda(e, "multi-owner expand");
+    if (e != cudaSuccess) return check_cuda(e, "probe launch");
+    const int rc = expand(off + m < n);
+    if (rc != SPADE_OK) return rc;
   }
   return SPADE_OK;
 }

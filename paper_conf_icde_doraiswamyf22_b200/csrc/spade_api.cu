@@ -16,6 +16,7 @@ namespace spade {
 int build_canvas(const int32_t*, const int64_t*, const int64_t*, int32_t, const spade_canvas_params*, cudaStream_t,
                  spade_canvas**);
 int build_disk_canvas(const int32_t*, const int64_t*, int32_t, const spade_canvas_params*, cudaStream_t, spade_canvas**);
+int canvas_checksum(const spade_canvas*, uint64_t*, cudaStream_t);
 
 namespace {
 thread_local char g_err[512] = "";
@@ -94,7 +95,7 @@ Options& options() {
   static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
                    env_int("SPADE_CACHE_SLOTS", 4096), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
                    env_int("SPADE_PIPE", -1), env_int("SPADE_DEFER_XY", 0), env_int("SPADE_L2_FRAC_PCT", 100), env_int("SPADE_MULTI_AGG", 1), env_int("SPADE_K_AGG", -1),
-                   (int64_t)1 << 25};
+                   (int64_t)1 << 25, (1ll << 31) - 64, 4096};
   return o;
 }
 }  // namespace spade
@@ -117,6 +118,7 @@ int spade_build_disk_canvas(const int32_t* center_xy, const int64_t* r2, int32_t
 
 void spade_canvas_free(spade_canvas* c) {
   if (!c) return;
+  DeviceGuard dg(c->device);
   cudaDeviceSynchronize();
   cudaFree(c->fine); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->recs); cudaFree(c->blob);
   cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->d_dev);
@@ -138,10 +140,17 @@ int spade_canvas_info(const spade_canvas* c, int32_t* W, int32_t* H, int32_t* lo
   return SPADE_OK;
 }
 
+int spade_canvas_checksum(const spade_canvas* c, uint64_t* out, spade_stream_t stream) {
+  if (!c || !out) return set_error(SPADE_ERR_INVALID_ARG, "spade_canvas_checksum: NULL argument");
+  DeviceGuard dg(c->device);
+  return canvas_checksum(c, out, (cudaStream_t)stream);
+}
+
 int spade_join_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts, spade_stream_t stream) {
   int rc = check_points(c, xy, n, "spade_join_count");
   if (rc) return rc;
   if (c->d.num_polys > 0 && !counts) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_count: counts is NULL");
+  DeviceGuard dg(c->device);
   return launch_count(c, xy, n, counts, (cudaStream_t)stream);
 }
 
@@ -150,6 +159,7 @@ int spade_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t po
   int rc = check_points(c, xy, n, "spade_select");
   if (rc) return rc;
   if (capacity > 0 && !out_ids) return set_error(SPADE_ERR_INVALID_ARG, "spade_select: out_ids is NULL");
+  DeviceGuard dg(c->device);
   return run_with_capacity(capacity, n_out, (cudaStream_t)stream, "spade_select", [&](unsigned long long* t) {
     return launch_select(c, xy, n, point_id_base, out_ids, capacity, t, (cudaStream_t)stream);
   });
@@ -161,6 +171,7 @@ int spade_join_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_
   if (rc) return rc;
   if (capacity > 0 && (!out_point_ids || !out_poly_ids))
     return set_error(SPADE_ERR_INVALID_ARG, "spade_join_pairs: output arrays are NULL");
+  DeviceGuard dg(c->device);
   return run_with_capacity(capacity, n_out, (cudaStream_t)stream, "spade_join_pairs", [&](unsigned long long* t) {
     return launch_pairs(c, xy, n, point_id_base, out_point_ids, out_poly_ids, capacity, t, (cudaStream_t)stream);
   });
@@ -176,6 +187,7 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
   const int P = c->d.num_polys;
   if (P > 0 && !counts_host) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_count_host: counts_host is NULL");
   if (n == 0 || P == 0) return SPADE_OK;
+  DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
   const int64_t kChunk = options().host_chunk;  // default 32 Mi points = 256 MiB per staging buffer
   const int64_t chunk = std::min(kChunk, n);
@@ -247,6 +259,7 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
 // Output order: chunk order; within a chunk unspecified (as the device calls).
 static int map_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, int64_t base, int64_t* out_ids,
                     int32_t* out_polys, int64_t capacity, int64_t* n_out, cudaStream_t st, const char* fn) {
+  DeviceGuard dg(c->device);
   const bool pairs = out_polys != nullptr || std::string(fn) == "spade_join_pairs_host";
   const int64_t chunk = std::min(options().host_chunk, n);
   int32_t* stage[2] = {nullptr, nullptr};
@@ -495,6 +508,8 @@ int spade_set_option(const char* name, int64_t value) {
     o.cache_slots = (int)value;
   else if (n == "pipe" && (value == -1 || bit)) o.pipe = (int)value;
   else if (n == "host_chunk" && value >= 256 && value <= ((int64_t)1 << 28)) o.host_chunk = value;
+  else if (n == "max_launch_points" && value >= 256 && value <= (1ll << 31) - 64) o.max_launch_points = value;
+  else if (n == "defer_budget_mb" && value >= 64 && value <= (1ll << 20)) o.defer_budget_mb = value;
   else if (n == "coop" && (value == -1 || value == 0 || value == 4 || value == 8 || value == 16)) o.coop = (int)value;
   else return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: bad option %s = %lld", name, (long long)value);
   return SPADE_OK;

@@ -91,6 +91,7 @@ struct spade_canvas {
   int device = 0;
   bool empty = true;          // no polygon vertices: everything is outside
   int64_t num_runs = 0, num_records = 0, num_run_edges = 0, num_set_entries = 0;
+  int64_t num_set_ranges = 0, cfine_elems = 0, coarse_elems = 0;   // array sizes (checksum)
   double mixed_tile_frac = 0.0;
   // owned device allocations
   int32_t* fine = nullptr;
@@ -131,7 +132,19 @@ int device_sm_count();
 // probe-path options (spade_set_option; include/spade.h)
 struct Options {
   int defer, count_global, global_queue, cache_slots, coop, debug_defer, pipe, defer_xy, l2_frac_pct, multi_agg, k_agg;
-  int64_t host_chunk;  // points per staging chunk of the host-resident calls
+  int64_t host_chunk;         // points per staging chunk of the host-resident calls
+  int64_t max_launch_points;  // points per probe sub-launch (< 2^31; smaller values: tests)
+  int64_t defer_budget_mb;    // deferral scratch per sub-launch (16 B per reserved entry)
+};
+
+// Makes the canvas's device current for the duration of an entry point (restored after).
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+    else prev = -1;
+  }
+  ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
 };
 Options& options();
 

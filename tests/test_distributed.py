@@ -136,3 +136,62 @@ def test_sharded_knn_equals_oracle(world):
         for r in range(world):
             assert out[r][k][0] == oi.tolist()
             assert out[r][k][1] == od.tolist()
+
+
+# ---- sharded outputs by default, exact-size gather on request, replicated-canvas checksums ----
+
+def _shard_worker(rank, world, port, out):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        polys = _polys()
+        start, stop = sd.shard_range(N, rank, world)
+        xy = _points(start, stop - start)
+
+        def pairs_fn(p, x, base):
+            pt, pl = oracle.join_pairs(x, p, point_id_base=base, nthreads=2)
+            return torch.from_numpy(pt), torch.from_numpy(pl.astype(np.int64))
+
+        def select_fn(p, x, base):
+            return torch.from_numpy(oracle.select(x, p, point_id_base=base, nthreads=2))
+
+        local = sd.join_pairs_distributed(polys, xy, start, pairs_fn=pairs_fn)
+        gathered = sd.join_pairs_distributed(polys, xy, start, pairs_fn=pairs_fn, gather=True, dst=world - 1)
+        ids = sd.select_distributed(polys, xy, start, select_fn=select_fn, gather=True, dst=0)
+        agree = sd.canvas_checksums_agree(polys, checksum_fn=lambda p: 0xDEADBEEFCAFEF00D)
+        differ = sd.canvas_checksums_agree(polys, checksum_fn=lambda p: 12345 + (rank == 1))
+        empty = sd.gather_variable(torch.zeros(0, dtype=torch.int64) if rank != 0 else torch.arange(5), dst=1)
+        out[rank] = {"local": (local[0].numpy().tolist(), local[1].numpy().tolist()),
+                     "gathered": None if gathered is None else (gathered[0].numpy().tolist(), gathered[1].numpy().tolist()),
+                     "ids": None if ids is None else ids.numpy().tolist(), "agree": agree, "differ": differ,
+                     "empty": None if empty is None else empty.numpy().tolist(), "range": (start, stop)}
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_outputs_gather_on_request_and_checksums(world):
+    mgr = mp.Manager()
+    out = mgr.dict()
+    mp.spawn(_shard_worker, args=(world, _free_port(), out), nprocs=world, join=True)
+    polys = _polys()
+    xy = _points(0, N)
+    rpt, rpl = oracle.join_pairs(xy, polys)
+    for r in range(world):
+        a, b = out[r]["range"]
+        lpt = np.array(out[r]["local"][0])
+        assert len(lpt) == 0 or (lpt.min() >= a and lpt.max() < b)      # sharded: own ids only
+        m = (rpt >= a) & (rpt < b)
+        o = np.lexsort((np.array(out[r]["local"][1]), lpt))
+        assert lpt[o].tolist() == rpt[m].tolist()
+        assert out[r]["agree"] is True
+        assert out[r]["differ"] is False
+        assert (out[r]["gathered"] is None) == (r != world - 1)
+        assert (out[r]["ids"] is None) == (r != 0)
+    gpt, gpl = out[world - 1]["gathered"]
+    o = np.lexsort((np.array(gpl), np.array(gpt)))
+    assert np.array(gpt)[o].tolist() == rpt.tolist()
+    assert np.array(gpl)[o].tolist() == rpl.tolist()
+    assert sorted(out[0]["ids"]) == oracle.select(xy, polys).tolist()
+    assert out[1]["empty"] == [0, 1, 2, 3, 4]

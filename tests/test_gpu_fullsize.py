@@ -90,21 +90,44 @@ def test_full_size_select_c2(sp):
     assert int(sp.join_count(cv, xy)[0]) == ids.numel()
 
 
+def _boundary_points(polys, k, seed):
+    """k points on or next to polygon boundaries: random ring vertices (shared by two or more
+    polygons of the tiling: the tie rule decides them), and vertices moved by 1..3 units (within
+    the closed pixel the edges touch).  Every one lies in a boundary pixel at any resolution >= 8
+    units, so every one takes the exact test."""
+    rng = np.random.default_rng(seed)
+    v = polys["ring_xy"][rng.integers(0, len(polys["ring_xy"]), k)].astype(np.int64)
+    d = rng.integers(-3, 4, (k, 2))
+    d[: k // 2] = 0
+    return (v + d).astype(np.int32)
+
+
 def test_full_size_count_c5_one_gpu_shard(sp):
-    """Config 5's polygon set (40k zip-code-like tiles) with one GPU's 1B-point shard."""
+    """Config 5's polygon set (40k zip-code-like tiles) with one GPU's 1B-point shard, plus 6,000
+    boundary-pixel points appended (vertices and near-vertex points): COUNT == hist(PAIRS), the
+    appended points' labels and 2,000 sampled stream points equal the oracle's."""
     import torch
     w = configs.c5()
     n = w.n_points
     cv = sp.Canvas(w.polys, max_dim=w.max_dim)
-    xy = _device_points(w, n, start=3 * n)                   # shard 3 of 8: global ids [3n, 4n)
+    nb = 6000
+    bxy = _boundary_points(w.polys, nb, 41)
+    xy = torch.empty((n + nb, 2), dtype=torch.int32, device="cuda")
+    gen.points_device(w.points, w.point_seed, 3 * n, n, out=xy[:n])   # shard 3 of 8: global ids [3n, 4n)
+    xy[n:] = torch.as_tensor(bxy, device="cuda")
     counts = sp.join_count(cv, xy)
-    assert int(counts.sum()) == n
     pt, pl = sp.join_pairs(cv, xy, point_id_base=3 * n)
     assert torch.equal(torch.bincount(pl.long(), minlength=cv.num_polys), counts)
-    lab = _labels_from_pairs(pt - 3 * n, pl, n)
-    idx = _sample(n, 300, 29)
+    lab = _labels_from_pairs(pt - 3 * n, pl, n + nb)
+    assert int((lab[:n] < 0).sum()) == 0                       # the stream lies inside the tiling
+    idx = _sample(n, 2000, 29)
     got = lab[torch.as_tensor(idx, device="cuda")].cpu().numpy().astype(np.int64)
     np.testing.assert_array_equal(got, _oracle_labels(w, idx + 3 * n))
+    bpt, bpl = oracle.join_pairs(bxy, w.polys)
+    assert len(np.unique(bpt)) == len(bpt)
+    exp = np.full(nb, -1, np.int64)
+    exp[bpt] = bpl
+    np.testing.assert_array_equal(lab[n:].cpu().numpy().astype(np.int64), exp)
 
 
 def test_full_size_overlap_heavy_ov(sp):
