@@ -360,14 +360,19 @@ __global__ void k_segkey(const uint64_t* __restrict__ key, const int32_t* __rest
 // entries sorted by (bid, hash): the first occurrence of each exact segment within its equal-key
 // run carries the XOR of the polygon bits of all its occurrences; zero masks (a segment used
 // an even number of times by the same polygons) contribute nothing and are dropped.  Records with
-// more than kMaskPolys polygons keep every entry with its local index.
+// more than kMaskPolys polygons keep every entry with its local index.  PASS 0 flags the kept
+// entries (keep[u]) and counts them per record; PASS 1 writes entry u at its rank among the kept
+// entries (kpos = exclusive scan of keep: the entries are sorted by record, so a record's kept
+// entries start at mbeg[bid]) -- positions independent of thread timing, so the canvas bytes are
+// deterministic (spade_canvas_checksum).
 template <int PASS>
 __global__ void k_merge(const uint64_t* __restrict__ key2, const int32_t* __restrict__ tix, int64_t L,
                         const int32_t* __restrict__ ev, const int32_t* __restrict__ li, const int4* __restrict__ seg,
                         const int32_t* __restrict__ pcnt, const int64_t* __restrict__ le_beg, int32_t* __restrict__ mcnt,
-                        const int64_t* __restrict__ mbeg, int32_t* __restrict__ mfill,
+                        const int64_t* __restrict__ mbeg, int32_t* __restrict__ keep, const int64_t* __restrict__ kpos,
                         int4* __restrict__ oseg, uint64_t* __restrict__ omask, int kind) {
   for (int64_t u = blockIdx.x * (int64_t)kBT + threadIdx.x; u < L; u += (int64_t)gridDim.x * kBT) {
+    if (PASS == 1 && !keep[u]) continue;
     const uint64_t k = key2[u];
     const uint32_t bid = (uint32_t)(k >> 32);
     const int4 e = seg[ev[tix[u]]];
@@ -377,19 +382,21 @@ __global__ void k_merge(const uint64_t* __restrict__ key2, const int32_t* __rest
       m = (uint64_t)li[tix[u]];
     } else {
       bool first = true;
-      for (int64_t w = u - 1; w >= 0 && key2[w] == k; --w)
-        if (same_seg(seg[ev[tix[w]]], e, kind)) { first = false; break; }
-      if (!first) continue;
+      if (PASS == 0)
+        for (int64_t w = u - 1; w >= 0 && key2[w] == k; --w)
+          if (same_seg(seg[ev[tix[w]]], e, kind)) { first = false; break; }
+      if (!first) { keep[u] = 0; continue; }
       m = 1ull << li[tix[u]];
       for (int64_t w = u + 1; w < L && key2[w] == k; ++w)
         if (same_seg(seg[ev[tix[w]]], e, kind)) m ^= 1ull << li[tix[w]];
-      if (m == 0) continue;
+      if (m == 0) { if (PASS == 0) keep[u] = 0; continue; }
     }
     if (PASS == 0) {
+      keep[u] = 1;
       atomicAdd(&mcnt[bid], 1);
     } else {
       // slow records keep the (bid, poly) order of the entries: grouped by local index
-      const int64_t pos = mbeg[bid] + (slow ? (int64_t)tix[u] - le_beg[bid] : (int64_t)atomicAdd(&mfill[bid], 1));
+      const int64_t pos = slow ? mbeg[bid] + ((int64_t)tix[u] - le_beg[bid]) : kpos[u];
       oseg[pos] = e;
       omask[pos] = m;
     }
@@ -525,12 +532,15 @@ __global__ void k_kset_rng(int64_t NB, const int32_t* __restrict__ ksize, const 
   }
 }
 
+// final encoding: boundary pixel -> -2 - (its record's header offset in the blob); multi-owner
+// corner (owner set g) -> -2 - (record NB + g's header offset)
 __global__ void k_finalize(int64_t WH, const int32_t* __restrict__ bflag, const int32_t* __restrict__ bscan,
-                           const int32_t* __restrict__ corner, int64_t NB, int32_t* __restrict__ fine) {
+                           const int32_t* __restrict__ corner, int64_t NB, const int64_t* __restrict__ boff,
+                           int32_t* __restrict__ fine) {
   for (int64_t p = blockIdx.x * (int64_t)kBT + threadIdx.x; p < WH; p += (int64_t)gridDim.x * kBT) {
-    if (bflag[p]) { fine[p] = -2 - (bscan[p] - 1); continue; }
+    if (bflag[p]) { fine[p] = (int32_t)(-2 - boff[bscan[p] - 1]); continue; }
     int32_t v = corner[p];
-    fine[p] = v >= kEmpty ? v : (int32_t)(-2 - (NB + (-2 - (int64_t)v)));   // owner set g -> record NB + g
+    fine[p] = v >= kEmpty ? v : (int32_t)(-2 - boff[NB + (-2 - (int64_t)v)]);   // owner set g -> record NB + g
   }
 }
 
@@ -592,15 +602,19 @@ __global__ void k_compact(const int32_t* __restrict__ fine, int W, int H, int b,
 struct BigSize { __host__ __device__ int64_t operator()(int32_t v) const { return v >= 2 ? v : 0; } };
 struct BigFlag { __host__ __device__ int32_t operator()(int32_t v) const { return v >= 2 ? 1 : 0; } };
 
-// K-B6: packed records (spade_internal.cuh "Rec").  Blob size in 16-byte units and layout flags:
-// polygon primitives are stored relative to the pixel's lower-left corner as int16 when all four
-// coordinates fit, masks as bytes when the pixel has <= 8 polygons.
+// K-B6: packed records (spade_internal.cuh "Rec").  Every record is one contiguous blob: a 16-B
+// header (RecHdr) followed by its data; the fine canvas holds the header's blob offset, so the
+// probe reaches a record's data with no separate record fetch.  Blob size in 16-byte units and
+// layout flags: polygon primitives are stored relative to the pixel's lower-left corner as int16
+// when all four coordinates fit, masks as bytes when the pixel has <= 8 polygons.  Multi-owner
+// records (r >= NB) are a header only: they come last, one unit each (the probe's per-record
+// counters are indexed by their unit offset minus the first one's).
 __device__ __forceinline__ bool fits16(int64_t v) { return v >= -32768 && v <= 32767; }
 __global__ void k_blob_size(int64_t NR, int64_t NB, const RunRec* __restrict__ runs, const int64_t* __restrict__ pix_of,
                             Geo g, const int4* __restrict__ rseg, int kind, int64_t* __restrict__ bsz,
                             uint32_t* __restrict__ bflags) {
   for (int64_t r = blockIdx.x * (int64_t)kBT + threadIdx.x; r < NR; r += (int64_t)gridDim.x * kBT) {
-    if (r >= NB) { bsz[r] = 0; bflags[r] = 0; continue; }          // multi-owner record: no data
+    if (r >= NB) { bsz[r] = 1; bflags[r] = 0; continue; }          // multi-owner record: header only
     const RunRec x = runs[r];
     const int64_t p = pix_of[r];
     const int64_t X = g.minx + (p % g.W) * g.S, Y = g.miny + (p / g.W) * g.S;
@@ -611,7 +625,7 @@ __global__ void k_blob_size(int64_t NR, int64_t NB, const RunRec* __restrict__ r
     }
     const bool by = x.poly_cnt <= 8;
     const int64_t bytes = (((int64_t)x.poly_cnt * 4 + 15) & ~15ll) + (int64_t)x.edge_cnt * ((sh ? 8 : 16) + (by ? 1 : 8));
-    bsz[r] = (bytes + 15) >> 4;
+    bsz[r] = 1 + ((bytes + 15) >> 4);
     bflags[r] = (sh ? kRecShort : 0u) | (by ? kRecByte : 0u);
   }
 }
@@ -622,10 +636,16 @@ __global__ void k_blob_pack(int64_t NR, int64_t NB, const RunRec* __restrict__ r
                             const uint32_t* __restrict__ bflags, Rec* __restrict__ recs, uint4* __restrict__ blob) {
   for (int64_t r = blockIdx.x * (int64_t)kBT + threadIdx.x; r < NR; r += (int64_t)gridDim.x * kBT) {
     const RunRec x = runs[r];
-    if (r >= NB) { recs[r] = Rec{0u, x.term, 0, 0u}; continue; }
+    const uint32_t data = (uint32_t)boff[r] + 1u;
+    if (r >= NB) {
+      recs[r] = Rec{data, x.term, 0, 0u};
+      blob[boff[r]] = make_uint4((uint32_t)x.term, 0u, 0u, (uint32_t)r);
+      continue;
+    }
     const uint32_t fl = bflags[r];
-    recs[r] = Rec{(uint32_t)boff[r], x.term, x.edge_cnt, (uint32_t)x.poly_cnt | fl};
-    unsigned char* b = (unsigned char*)(blob + boff[r]);
+    recs[r] = Rec{data, x.term, x.edge_cnt, (uint32_t)x.poly_cnt | fl};
+    blob[boff[r]] = make_uint4((uint32_t)x.term, (uint32_t)x.edge_cnt, (uint32_t)x.poly_cnt | fl, (uint32_t)r);
+    unsigned char* b = (unsigned char*)(blob + data);
     int32_t* pp = (int32_t*)b;
     for (int k = 0; k < x.poly_cnt; ++k) pp[k] = rec_polys[x.poly_begin + k];
     unsigned char* eb = b + (((int64_t)x.poly_cnt * 4 + 15) & ~15ll);
@@ -844,12 +864,14 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   if (NB > 0)
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, le_cnt, le_beg, NB, st); }), "scan local edges");
   // distinct polygons per boundary pixel, local indices, de-duplicated edges with toggle masks
-  int32_t *ph, *pg, *pbeg, *pcnt, *li, *tix, *tix2, *mcnt, *mfill;
+  int32_t *ph, *pg, *pbeg, *pcnt, *li, *tix, *tix2, *mcnt;
   int64_t* mbeg;
   uint64_t* key2s;
   ALLOC(ph, L, "dedup"); ALLOC(pg, L, "dedup"); ALLOC(pbeg, NB, "dedup"); ALLOC(pcnt, NB, "dedup");
   ALLOC(li, L, "dedup"); ALLOC(tix, L, "dedup"); ALLOC(tix2, L, "dedup"); ALLOC(key2s, L, "dedup");
-  ALLOC(mcnt, NB, "dedup"); ALLOC(mfill, NB, "dedup"); ALLOC(mbeg, NB + 1, "dedup");
+  ALLOC(mcnt, NB, "dedup"); ALLOC(mbeg, NB + 1, "dedup");
+  int32_t* mkeep; int64_t* mkpos;
+  ALLOC(mkeep, L, "dedup"); ALLOC(mkpos, L, "dedup");
   int32_t D32 = 0;
   if (L > 0) {
     LAUNCH(k_polyhead, L, lk2, L, ph);
@@ -863,12 +885,12 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   if (NB > 0) LAUNCH(k_polyrange, NB, NB, le_beg, le_cnt, pg, pbeg, pcnt);
   int64_t LM = 0;
   TRYF(cudaMemsetAsync(mcnt, 0, sizeof(int32_t) * std::max<int64_t>(NB, 1), st), "memset");
-  TRYF(cudaMemsetAsync(mfill, 0, sizeof(int32_t) * std::max<int64_t>(NB, 1), st), "memset");
   if (L > 0) {
     LAUNCH(k_segkey, L, lk2, lv2, L, seg, pg, pbeg, lk, li);            // lk reused for (bid, hash) keys
     LAUNCH(k_iota, L, tix, L);
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceRadixSort::SortPairs(t, sz, lk, key2s, tix, tix2, L, 0, 32 + bbits, st); }), "sort segments");
-    LAUNCH(k_merge<0>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, nullptr, nullptr, nullptr, nullptr, kind);
+    LAUNCH(k_merge<0>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, nullptr, mkeep, nullptr, nullptr, nullptr, kind);
+    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, mkeep, mkpos, L, st); }), "scan kept");
   }
   if (NB > 0) {
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, mcnt, mbeg, NB, st); }), "scan merged");
@@ -880,7 +902,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   }
   int4* run_seg; uint64_t* run_mask;
   ALLOC(run_seg, LM, "local edge arrays"); ALLOC(run_mask, LM, "local edge arrays");
-  if (L > 0) LAUNCH(k_merge<1>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, mbeg, mfill, run_seg, run_mask, kind);
+  if (L > 0) LAUNCH(k_merge<1>, L, key2s, tix2, L, lv2, li, seg, pcnt, le_beg, mcnt, mbeg, mkeep, mkpos, run_seg, run_mask, kind);
   tmp.release(lk); tmp.release(lk2); tmp.release(lv); tmp.release(lv2); tmp.release(frags); tmp.release(lw_off);
   tmp.release(ph); tmp.release(pg); tmp.release(li); tmp.release(tix); tmp.release(tix2); tmp.release(key2s);
 
@@ -966,26 +988,28 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   }
   if (NG > 0) LAUNCH(k_multi_recs, NG, NG, NB, runs);
 
-  // --- K-B6 packed records: one 16-B record + one contiguous blob per boundary pixel ---
-  {
-    const int64_t NR = NB + NG;
-    int64_t *bsz, *boff;
-    uint32_t* bflags;
-    ALLOC(bsz, NR, "record blobs"); ALLOC(boff, NR + 1, "record blobs"); ALLOC(bflags, NR, "record blobs");
-    LAUNCH(k_blob_size, NR, NR, NB, runs, pix_of, g, run_seg, kind, bsz, bflags);
-    TRYF(cudaMemsetAsync(boff, 0, 8, st), "memset");
-    TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, bsz, boff + 1, NR, st); }), "scan blobs");
-    int64_t units = 0;
-    TRYF(cudaMemcpyAsync(&units, boff + NR, 8, cudaMemcpyDeviceToHost, st), "blob size");
-    TRYF(cudaStreamSynchronize(st), "sync blobs");
-    if (units >= (1ll << 32)) return fail(set_error(SPADE_ERR_INVALID_ARG, "boundary index too large (%lld x 16 B)", (long long)units));
-    if (cudaMalloc(&c->recs, sizeof(Rec) * std::max<int64_t>(NR, 1)) != cudaSuccess ||
-        cudaMalloc(&c->blob, 16 * std::max<int64_t>(units, 1)) != cudaSuccess)
-      return fail(set_error(SPADE_ERR_OOM, "build: packed records"));
-    c->blob_bytes = 16 * units;
-    LAUNCH(k_blob_pack, NR, NR, NB, runs, pix_of, g, run_seg, run_mask, rec_polys, boff, bflags, c->recs, c->blob);
-  }
-  LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, c->fine);
+  // --- K-B6 packed records: one contiguous blob (16-B header + data) per record ---
+  const int64_t NR = NB + NG;
+  int64_t *bsz, *boff;
+  uint32_t* bflags;
+  ALLOC(bsz, NR, "record blobs"); ALLOC(boff, NR + 1, "record blobs"); ALLOC(bflags, NR, "record blobs");
+  LAUNCH(k_blob_size, NR, NR, NB, runs, pix_of, g, run_seg, kind, bsz, bflags);
+  TRYF(cudaMemsetAsync(boff, 0, 8, st), "memset");
+  TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::InclusiveSum(t, sz, bsz, boff + 1, NR, st); }), "scan blobs");
+  int64_t units = 0, multi_unit = 0;
+  TRYF(cudaMemcpyAsync(&units, boff + NR, 8, cudaMemcpyDeviceToHost, st), "blob size");
+  TRYF(cudaMemcpyAsync(&multi_unit, boff + NB, 8, cudaMemcpyDeviceToHost, st), "blob size");
+  TRYF(cudaStreamSynchronize(st), "sync blobs");
+  // fine values -2 - offset must stay >= INT32_MIN
+  if (units >= (1ll << 31) - 2) return fail(set_error(SPADE_ERR_INVALID_ARG, "boundary index too large (%lld x 16 B)", (long long)units));
+  if (cudaMalloc(&c->recs, sizeof(Rec) * std::max<int64_t>(NR, 1)) != cudaSuccess ||
+      cudaMalloc(&c->blob, 16 * std::max<int64_t>(units, 1)) != cudaSuccess)
+    return fail(set_error(SPADE_ERR_OOM, "build: packed records"));
+  c->blob_bytes = 16 * units;
+  c->multi_unit = multi_unit;
+  TRYF(cudaMemsetAsync(c->blob, 0, 16 * std::max<int64_t>(units, 1), st), "memset blob");   // padding bytes defined
+  LAUNCH(k_blob_pack, NR, NR, NB, runs, pix_of, g, run_seg, run_mask, rec_polys, boff, bflags, c->recs, c->blob);
+  LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, boff, c->fine);
 
   // --- K-B5 coarse tiles (+ compact fine layout) ---
   const int64_t NT = (int64_t)Wc * Hc;
@@ -1063,7 +1087,8 @@ int canvas_checksum(const spade_canvas* c, uint64_t* out, cudaStream_t st) {
   if (!c->empty) {
     const CanvasDev& d = c->d;
     const int64_t hdr[] = {d.minx, d.miny, d.extw, d.exth, d.s, d.W, d.H, d.b, d.Wc, d.Hc, d.compact, d.mix_min,
-                           c->num_runs, c->num_records, c->num_run_edges, c->num_set_entries, c->num_set_ranges};
+                           c->num_runs, c->num_records, c->num_run_edges, c->num_set_entries, c->num_set_ranges,
+                           c->multi_unit};
     for (int64_t v : hdr) h = mix64(h ^ (uint64_t)v);
     unsigned long long* acc = nullptr;
     cudaError_t e = cudaMallocAsync((void**)&acc, sizeof(unsigned long long), st);

@@ -147,7 +147,7 @@ struct Params {
   uint32_t defer_xy;          // pipelined probe: deferral entries carry the point (re-read from L2)
   float l2_frac;              // fraction of fine-canvas lines gathered with L2::evict_last
   unsigned int* rec_cnt;      // COUNT over overlapping polygons: points per multi-owner record, or null
-  uint32_t multi_base;        // first multi-owner record id (records >= it have no edges)
+  uint32_t multi_base;        // blob unit of the first multi-owner record header (records at or past it have no edges)
   unsigned int* kcnt;         // COUNT with K aggregation: points per boundary record, or null
   const int2* xy;
   int64_t n;
@@ -308,9 +308,20 @@ struct TermMerge {
   __device__ __forceinline__ void rest() { while (ti < tn) emit(at(ti++)); }
 };
 
+// The record whose header is at blob unit u (the fine canvas value of a boundary / multi-owner
+// pixel is -2 - u; spade_internal.cuh "Packed records").  The header load asks L2 to fetch the
+// 256-B block around it (L2::256B), so the record's data -- the next loads of the exact test --
+// comes in with the same DRAM access instead of one dependent miss per sector.
+__device__ __forceinline__ Rec load_rec(const CanvasDev* __restrict__ cv, uint32_t u, uint32_t* id = nullptr) {
+  uint4 h;
+  asm("ld.global.nc.L2::256B.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(h.x), "=r"(h.y), "=r"(h.z), "=r"(h.w) : "l"(cv->blob + u));
+  if (id) *id = h.w;
+  return Rec{u + 1u, (int32_t)h.x, (int32_t)h.y, h.z};
+}
+
 // Exact test for a point on the boundary (or multi-owner) pixel of record `rec` (packed layout:
-// spade_internal.cuh "Rec"): one 16-B record fetch, then the record's polygons, primitives and
-// masks from one contiguous blob.  emit(P) for every polygon containing the point, ascending.
+// spade_internal.cuh "Packed records"): the header, then the record's polygons, primitives and
+// masks from the same contiguous blob.  emit(P) for every polygon containing the point, ascending.
 template <int KIND, int U, class Fin>
 __device__ __forceinline__ void pip_edges_rec(const CanvasDev* __restrict__ cv, int px, int py, const Rec r, Fin& fin);
 
@@ -385,7 +396,7 @@ __device__ __forceinline__ void pip_edges_rec(const CanvasDev* __restrict__ cv, 
 }
 template <int KIND, int U = 1, class Emit>
 __device__ __forceinline__ void pip_eval(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, Emit&& emit) {
-  pip_eval_rec<KIND, U>(cv, px, py, cv->recs[rec], emit);
+  pip_eval_rec<KIND, U>(cv, px, py, load_rec(cv, rec), emit);
 }
 
 // Cooperative exact test: the G lanes of a group share one point (same px, py, rec in every lane);
@@ -490,13 +501,15 @@ __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint
     const uint32_t fx = ((uint32_t)e.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)e.y - (uint32_t)cv.miny) >> cv.s;
     const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
     const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
+    uint32_t rid = 0;
+    const Rec r = load_rec(cvg, ~c, &rid);
     if (kcnt)
-      pip_count_delta<KIND>(cvg, e.x, e.y, ~c, cv.recs[~c], kcnt, [&](int q, int d) {
+      pip_count_delta<KIND>(cvg, e.x, e.y, rid, r, kcnt, [&](int q, int d) {
         if (MODE == kCountSmem) atomicAdd(&hist[(uint32_t)q * hstride], (unsigned int)d);
         else atomicAdd(counts + q, (unsigned long long)(long long)d);
       });
     else
-      pip_eval<KIND>(cvg, e.x, e.y, ~c, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
+      pip_eval_rec<KIND>(cvg, e.x, e.y, r, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
   }
 }
 
@@ -1127,7 +1140,7 @@ __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __r
     const bool act = e.rec != kHole;
     if (act && pxy) { const int2 q = __ldg(pxy + e.pidx); e.x = q.x; e.y = q.y; }   // entry without coordinates
     Rec r{0u, kEmpty, 0, 0u};
-    if (act) r = cvg->recs[e.rec];
+    if (act) r = load_rec(cvg, e.rec);
     bool big;
     const uint64_t m = group_mask<KIND, G>(cvg, act, e.x, e.y, r, gl, big);
     int first = -1;
@@ -1194,24 +1207,26 @@ __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict
   // software pipeline: the entry two points ahead and the record of the next point are in flight
   // while the current point is tested
   // (pxy != nullptr: the entries hold no coordinates; the point is re-read by its index)
-  auto rec_of = [&](DEntry& d) {
+  auto rec_of = [&](DEntry& d, uint32_t& id) {
     if (d.rec == kHole) return Rec{0u, kEmpty, 0, 0u};
     if (pxy) { const int2 q = __ldg(pxy + d.pidx); d.x = q.x; d.y = q.y; }
-    return cvg->recs[d.rec];
+    return load_rec(cvg, d.rec, &id);
   };
   DEntry nxt = fetch((long long)blockIdx.x * 256 + threadIdx.x);
   DEntry nxt2 = fetch((long long)blockIdx.x * 256 + gstride + threadIdx.x);
-  Rec nrec = rec_of(nxt);
+  uint32_t nid = 0;
+  Rec nrec = rec_of(nxt, nid);
   for (long long b0 = (long long)blockIdx.x * 256; b0 < total; b0 += gstride) {
     const DEntry e = nxt;
     const Rec rc = nrec;
+    const uint32_t rid = nid;
     nxt = nxt2;
     nxt2 = fetch(b0 + 2 * gstride + threadIdx.x);
-    nrec = rec_of(nxt);
+    nrec = rec_of(nxt, nid);
     const bool act = e.rec != kHole;
     const int64_t pid = o.id_base + (int64_t)e.pidx;
     if ((MODE == kCountSmem || MODE == kCountGlobal) && kcnt) {
-      if (act) pip_count_delta<KIND, 4>(cvg, e.x, e.y, e.rec, rc, kcnt, [&](int q, int d) {
+      if (act) pip_count_delta<KIND, 4>(cvg, e.x, e.y, rid, rc, kcnt, [&](int q, int d) {
         if (sh) atomicAdd(&dh[q], (unsigned int)d);
         else atomicAdd(o.counts + q, (unsigned long long)(long long)d);
       });
@@ -1585,7 +1600,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.defer = dbuf;
     p.defer_xy = PIPE ? (uint32_t)options().defer_xy : 0u;
     p.rec_cnt = rec_cnt;
-    p.multi_base = (uint32_t)c->num_runs;
+    p.multi_base = (uint32_t)c->multi_unit;
     p.kcnt = kcnt;
     p.l2_frac = (float)options().l2_frac_pct * 0.01f;
     p.defer_cap = (uint32_t)per;

@@ -38,13 +38,17 @@ struct RunRec {
 };
 constexpr int kMaskPolys = 64;     // records with more distinct polygons use the slow path
 
-// The probe's record (16 B): the build's RunRec packed for one dependent fetch.  `blob` is the
-// record's data in 16-byte units from CanvasDev::blob:
+// Packed records: one contiguous blob per record in CanvasDev::blob (16-byte units), located by
+// its header's unit offset u, which is what the fine canvas holds for a boundary / multi-owner
+// pixel (v = -2 - u).  Layout at u:
+//   header (16 B): RecHdr {term, ecnt, pinfo, id}
 //   int32 polys[pcnt]                      (padded to 16 B)
 //   primitives[ecnt]: short4 (ax,ay,bx,by) relative to the pixel's lower-left corner when every
 //                     coordinate fits in int16 (kRecShort), else int4 absolute
 //   masks[ecnt]:      uint8 when pcnt <= 8 (kRecByte), else uint64 (toggle mask / local index)
-// Multi-owner records have no blob (ecnt = pcnt = 0).
+// Multi-owner records (no edges) are a header only, after every boundary record, one unit each.
+// `Rec` is the decoded header with `blob` = the data's unit offset (u + 1); the canvas keeps a
+// Rec array indexed by record id (= RecHdr::id) for the per-record counter expansion.
 struct Rec {
   uint32_t blob;
   int32_t term;
@@ -92,6 +96,7 @@ struct spade_canvas {
   bool empty = true;          // no polygon vertices: everything is outside
   int64_t num_runs = 0, num_records = 0, num_run_edges = 0, num_set_entries = 0;
   int64_t num_set_ranges = 0, cfine_elems = 0, coarse_elems = 0;   // array sizes (checksum)
+  int64_t multi_unit = 0;     // blob offset of the first multi-owner record header
   double mixed_tile_frac = 0.0;
   // owned device allocations
   int32_t* fine = nullptr;
