@@ -66,6 +66,11 @@ typedef struct {
 /* flags: keep the dense W x H fine canvas as the probe's second level even when the compact
  * mixed-tile layout applies (for tests / comparisons; results are identical). */
 #define SPADE_CANVAS_DENSE 1
+/* flags: no 16-bit copy of a dense second level (the probe then gathers the int32 canvas).  By
+ * default a dense second level over fewer than 65534 polygons is probed through a uint16 copy
+ * (owner id / empty / "record": half the gather footprint; records are looked up in the int32
+ * canvas by the exact-test stage).  Results are identical either way. */
+#define SPADE_CANVAS_NO_FINE16 2
 
 /* Build the discrete canvas + boundary index for a polygon set (P:113-123 canvas creation,
  * Sec. 4.2; P:146 and P:268 boundary index, Sec. 4.3 / 5.5).

@@ -599,6 +599,14 @@ __global__ void k_compact(const int32_t* __restrict__ fine, int W, int H, int b,
   }
 }
 
+// 16-bit copy of the dense canvas (spade_internal.cuh kF16*)
+__global__ void k_fine16(const int32_t* __restrict__ fine, int64_t WH, uint16_t* __restrict__ f16) {
+  for (int64_t p = blockIdx.x * (int64_t)kBT + threadIdx.x; p < WH; p += (int64_t)gridDim.x * kBT) {
+    const int32_t v = fine[p];
+    f16[p] = v >= 0 ? (uint16_t)v : v == kEmpty ? kF16Empty : kF16Record;
+  }
+}
+
 struct BigSize { __host__ __device__ int64_t operator()(int32_t v) const { return v >= 2 ? v : 0; } };
 struct BigFlag { __host__ __device__ int32_t operator()(int32_t v) const { return v >= 2 ? 1 : 0; } };
 
@@ -1034,6 +1042,11 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
       return fail(set_error(SPADE_ERR_OOM, "build: compact canvas"));
     LAUNCH(k_compact, NT << (2 * b), c->fine, g.W, g.H, b, Wc, tval, mscan, NT, owner_lim, c->cfine);
   }
+  const bool f16 = !compact && P < (int32_t)kF16Empty && !(prm && (prm->flags & SPADE_CANVAS_NO_FINE16));
+  if (f16) {
+    if (cudaMalloc(&c->fine16, sizeof(uint16_t) * WH) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: fine16"));
+    LAUNCH(k_fine16, WH, c->fine, WH, c->fine16);
+  }
   TRYF(cudaStreamSynchronize(st), "sync compact");
 #undef TRYF
 #undef ALLOC
@@ -1055,7 +1068,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   d.compact = compact ? 1 : 0;
   d.mix_min = compact ? kTileMixedCompact : kTileMixed;
   d.cfine = c->cfine;
-  d.fine = c->fine; d.coarse = c->coarse; d.recs = c->recs; d.blob = c->blob;
+  d.fine = c->fine; d.fine16 = c->fine16; d.f16 = f16 ? 1 : 0; d.coarse = c->coarse; d.recs = c->recs; d.blob = c->blob;
   d.sets = c->sets; d.set_rng = c->set_rng;
   if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
   if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));
@@ -1086,7 +1099,7 @@ int canvas_checksum(const spade_canvas* c, uint64_t* out, cudaStream_t st) {
   uint64_t h = mix64(0x5ADEull ^ (uint64_t)c->d.num_polys ^ ((uint64_t)c->d.kind << 40));
   if (!c->empty) {
     const CanvasDev& d = c->d;
-    const int64_t hdr[] = {d.minx, d.miny, d.extw, d.exth, d.s, d.W, d.H, d.b, d.Wc, d.Hc, d.compact, d.mix_min,
+    const int64_t hdr[] = {d.minx, d.miny, d.extw, d.exth, d.s, d.W, d.H, d.b, d.Wc, d.Hc, d.compact, d.mix_min, d.f16,
                            c->num_runs, c->num_records, c->num_run_edges, c->num_set_entries, c->num_set_ranges,
                            c->multi_unit};
     for (int64_t v : hdr) h = mix64(h ^ (uint64_t)v);
@@ -1095,7 +1108,8 @@ int canvas_checksum(const spade_canvas* c, uint64_t* out, cudaStream_t st) {
     if (e != cudaSuccess) return check_cuda(e, "spade_canvas_checksum");
     e = cudaMemsetAsync(acc, 0, sizeof(unsigned long long), st);
     struct A { const void* p; int64_t words; };
-    const A arrs[] = {{c->fine, (int64_t)d.W * d.H}, {c->cfine, c->cfine_elems}, {c->coarse, (c->coarse_elems + 1) / 2},
+    const A arrs[] = {{c->fine, (int64_t)d.W * d.H}, {c->fine16, c->fine16 ? ((int64_t)d.W * d.H + 1) / 2 : 0},
+                      {c->cfine, c->cfine_elems}, {c->coarse, (c->coarse_elems + 1) / 2},
                       {c->recs, c->num_records * (int64_t)(sizeof(Rec) / 4)}, {c->blob, c->blob_bytes / 4},
                       {c->sets, c->num_set_entries}, {c->set_rng, 2 * c->num_set_ranges}};
     uint64_t salt = 1;

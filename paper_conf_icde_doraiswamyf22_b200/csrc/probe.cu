@@ -78,6 +78,17 @@ __device__ __forceinline__ uint32_t ld_fine(const int32_t* p, uint64_t pol) {
   return r;
 }
 
+__device__ __forceinline__ uint32_t ld_fine16(const uint16_t* p, uint64_t pol) {
+  uint32_t r;
+  asm volatile("ld.global.nc.L2::cache_hint.u16 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
+// class of a 16-bit fine code (spade_internal.cuh kF16*): owner + 1, 0 = none, or ~0 = a record
+// (boundary / multi-owner pixel; the record itself is found through the int32 canvas)
+__device__ __forceinline__ uint32_t class16(uint32_t code) {
+  return code < kF16Empty ? code + 1u : code == kF16Empty ? 0u : 0xffffffffu;
+}
+
 // 4-byte asynchronous copy global -> shared (LDGSTS): the gathered value lands in shared memory,
 // so the number of gathers in flight is not bounded by registers
 __device__ __forceinline__ void cp_async4(uint32_t saddr, const void* g, uint64_t pol) {
@@ -96,6 +107,14 @@ __device__ __forceinline__ uint32_t nctaid_x() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%nctaid.x;" : "=r"(r));
   return r;
+}
+
+// The record (header blob unit) of point (x, y) on a boundary / multi-owner pixel, from the
+// int32 canvas (the fine16 layout's records; rare in-probe paths of any layout).
+__device__ __forceinline__ uint32_t rec_of_point(const CanvasDev* __restrict__ cvg, int x, int y) {
+  const CanvasDev& cv = *cvg;
+  const uint32_t fx = ((uint32_t)x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)y - (uint32_t)cv.miny) >> cv.s;
+  return (uint32_t)(-2 - __ldg(cv.fine + ((size_t)fy * (uint32_t)cv.W + fx)));
 }
 
 struct U4 {
@@ -161,9 +180,10 @@ struct Params {
 // per-record counts are spread over the owner sets after the probe (k_multi_expand) — the
 // paper's aggregation plan for points: partial aggregates per canvas location, then combined
 // per polygon.  One global atomic per such point instead of one per (point, polygon).
-template <int MODE, class C>
+template <int MODE, int LAYOUT = 0, class C>
 __device__ __forceinline__ void count_multi_owner(const Params& prm, C& c) {
-  if (!(MODE == kCountSmem || MODE == kCountGlobal) || prm.rec_cnt == nullptr) return;
+  // (fine16: a record's id is not in the 16-bit code; the exact-test stage counts them)
+  if (!(MODE == kCountSmem || MODE == kCountGlobal) || LAYOUT == 2 || prm.rec_cnt == nullptr) return;
   if ((int)(c[0] | c[1] | c[2] | c[3]) >= 0) return;
 #pragma unroll
   for (int q = 0; q < kNPT; ++q)
@@ -616,7 +636,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
   const uint32_t Hc = (uint32_t)cv.Hc, Wc1 = Wc + 1u;
   const uint32_t b = (uint32_t)cv.b, bm = (1u << cv.b) - 1u, mixmin = cv.mix_min;
-  const int32_t* __restrict__ finep = COMPACT ? cv.cfine : cv.fine;
+  const int32_t* __restrict__ finep = COMPACT == 1 ? cv.cfine : cv.fine;
+  const uint16_t* __restrict__ f16p = cv.fine16;
   auto load_batch = [&](Vec4& v, uint32_t base) {
     const uint32_t idx = base + tid;
     if (base + chunk <= nvec) v = ld_stream(vp + idx);       // CTA-uniform: full batch
@@ -687,15 +708,15 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
         const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
         const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
-        const uint32_t fidx = COMPACT ? ((((f[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
-        f[q] = classify_fine((int32_t)ld_fine(finep + fidx, pol));
+        const uint32_t fidx = COMPACT == 1 ? ((((f[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
+        f[q] = COMPACT == 2 ? class16(ld_fine16(f16p + fidx, pol)) : classify_fine((int32_t)ld_fine(finep + fidx, pol));
       }
     }
     return f;
   };
   // phase C of one batch: the sinks.  getxy(q): coordinates of point q of this thread.
   auto process = [&](uint32_t base, U4 c, auto getxy) {
-    count_multi_owner<MODE>(prm, c);
+    count_multi_owner<MODE, COMPACT>(prm, c);
     const uint32_t orc = c[0] | c[1] | c[2] | c[3];
     if (QUEUE) {
       // phase C1 (COUNT): boundary points -> warp queue (one smem atomic per lane that has any),
@@ -749,7 +770,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
             dreg[d] = DEntry{p.x, p.y, ~c[q], pidx};
           } else {
             if (d < prm.defer_cap) dreg[d] = DEntry{0, 0, kHole, 0u};
-            rare_emit_point<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, p.x, p.y, ~c[q], prm.o.id_base + pidx);
+            rare_emit_point<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, p.x, p.y,
+                                        COMPACT == 2 ? rec_of_point(prm.cvg, p.x, p.y) : ~c[q], prm.o.id_base + pidx);
           }
           ++d;
         }
@@ -821,12 +843,12 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
           const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
           const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
           const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
-          const uint32_t fidx = COMPACT ? ((((c[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
-          c[q] = classify_fine((int32_t)ld_fine(finep + fidx, pol));
+          const uint32_t fidx = COMPACT == 1 ? ((((c[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
+          c[q] = COMPACT == 2 ? class16(ld_fine16(f16p + fidx, pol)) : classify_fine((int32_t)ld_fine(finep + fidx, pol));
         }
       }
       // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
-      count_multi_owner<MODE>(prm, c);
+      count_multi_owner<MODE, COMPACT>(prm, c);
       const uint32_t orc = c[0] | c[1] | c[2] | c[3];
       if (!QUEUE) {
         // phase C1 (COUNT, deferred): boundary points -> this CTA's deferral region (one smem
@@ -849,7 +871,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
                 dr[d] = DEntry{x, y, ~c[q], 0u};
               } else {
                 if (d < prm.defer_cap) dr[d] = DEntry{0, 0, kHole, 0u};
-                emit_point_inl<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, x, y, ~c[q], 0);
+                emit_point_inl<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, x, y,
+                                           COMPACT == 2 ? rec_of_point(prm.cvg, x, y) : ~c[q], 0);
               }
               ++d;
             }
@@ -999,7 +1022,9 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
   const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
   const uint32_t Hc = (uint32_t)cv.Hc, Wc1 = Wc + 1u;
   const uint32_t b = (uint32_t)cv.b, bm = (1u << cv.b) - 1u, mixmin = cv.mix_min;
-  const int32_t* __restrict__ finep = COMPACT ? cv.cfine : cv.fine;
+  const int32_t* __restrict__ finep = COMPACT == 1 ? cv.cfine : cv.fine;
+  const uint16_t* __restrict__ f16p = cv.fine16;
+  uint32_t halves = 0;                             // fine16: which half of the gathered word, per (batch % D, q)
   const uint32_t first = blockIdx.x * T, stride = nctaid_x() * T;
   const uint32_t nb = first < nvec ? (nvec - first + stride - 1) / stride : 0u;   // batches of this CTA
   const uint32_t ring_s = (uint32_t)__cvta_generic_to_shared(ring) + 4u * tid;
@@ -1028,8 +1053,18 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
         const uint32_t sa = slot + q * (T * 4);
         if (c >= mixmin) {
           const uint32_t fx = ux >> s, fy = uy >> s;
-          const uint32_t fidx = COMPACT ? ((((c & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
-          cp_async4(sa, finep + fidx, pol);
+          const uint32_t fidx = COMPACT == 1 ? ((((c & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
+          if (COMPACT == 2) {
+            // cp.async moves >= 4 bytes: the aligned word holding the code, half noted
+            const uint32_t hb = (it % D) * NPT + q;
+            halves = (halves & ~(1u << hb)) | ((fidx & 1u) << hb);
+            cp_async4(sa, f16p + (fidx & ~1u), pol);
+          } else {
+            cp_async4(sa, finep + fidx, pol);
+          }
+        } else if (COMPACT == 2) {
+          const uint32_t code = c == 0u ? (uint32_t)kF16Empty : c - 1u;    // uniform tile: both halves
+          asm volatile("st.shared.b32 [%0], %1;" ::"r"(sa), "r"(code | (code << 16)) : "memory");
         } else {
           asm volatile("st.shared.b32 [%0], %1;" ::"r"(sa), "r"(c - 1u) : "memory");   // pixel value: owner / -1
         }
@@ -1046,9 +1081,10 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
       for (int q = 0; q < NPT; ++q) {
         uint32_t v;
         asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(slot + q * (T * 4)) : "memory");
-        c[q] = v + 1u;                               // 0 none | owner + 1 | >= 2^31 record ~c
+        if (COMPACT == 2) c[q] = class16((v >> (((halves >> ((j % D) * NPT + q)) & 1u) * 16)) & 0xffffu);
+        else c[q] = v + 1u;                          // 0 none | owner + 1 | >= 2^31 record ~c
       }
-      count_multi_owner<MODE>(prm, c);
+      count_multi_owner<MODE, COMPACT>(prm, c);
       const uint32_t orc = c[0] | c[1] | c[2] | c[3];
       if ((int)orc < 0) {
         uint32_t bnd = 0;
@@ -1070,7 +1106,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
             } else {
               if (d < prm.defer_cap) dr[d] = DEntry{0, 0, kHole, 0u};
               const int2 p = __ldg(prm.xy + pbase + q);
-              emit_point_inl<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, p.x, p.y, ~c[q], 0);
+              emit_point_inl<MODE, KIND>(prm.cvg, myhist, prm.hcopies, prm.o, p.x, p.y,
+                                         COMPACT == 2 ? rec_of_point(prm.cvg, p.x, p.y) : ~c[q], 0);
             }
             ++d;
           }
@@ -1108,7 +1145,7 @@ template <int MODE, int KIND, int G>
 __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                             uint32_t cap, const unsigned int* __restrict__ fill, int nreg,
                                                             unsigned long long* __restrict__ counts, int smem_hist,
-                                                            const int2* __restrict__ pxy) {
+                                                            const int2* __restrict__ pxy, int pix) {
   constexpr int T = 1024, GPB = T / G;
   __shared__ long long s_pre[1025];              // exclusive prefix of the region fills
   extern __shared__ unsigned int dh[];
@@ -1139,6 +1176,7 @@ __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __r
     nxt = fetch(b0 + gstride + grp);             // the group's next point in flight meanwhile
     const bool act = e.rec != kHole;
     if (act && pxy) { const int2 q = __ldg(pxy + e.pidx); e.x = q.x; e.y = q.y; }   // entry without coordinates
+    if (act && pix) e.rec = rec_of_point(cvg, e.x, e.y);                         // fine16 canvas
     Rec r{0u, kEmpty, 0, 0u};
     if (act) r = load_rec(cvg, e.rec);
     bool big;
@@ -1177,7 +1215,8 @@ __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __r
 template <int MODE, int KIND>
 __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                   uint32_t cap, const unsigned int* __restrict__ fill, int nreg, Out o,
-                                                  int smem_hist, const int2* __restrict__ pxy, unsigned int* __restrict__ kcnt) {
+                                                  int smem_hist, const int2* __restrict__ pxy, unsigned int* __restrict__ kcnt,
+                                                  int pix) {
   using BS = cub::BlockScan<int, 256>;
   __shared__ typename BS::TempStorage tmp;
   __shared__ unsigned long long s_gb;
@@ -1210,6 +1249,7 @@ __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict
   auto rec_of = [&](DEntry& d, uint32_t& id) {
     if (d.rec == kHole) return Rec{0u, kEmpty, 0, 0u};
     if (pxy) { const int2 q = __ldg(pxy + d.pidx); d.x = q.x; d.y = q.y; }
+    if (pix) d.rec = rec_of_point(cvg, d.x, d.y);   // fine16 canvas: the record from the int32 level
     return load_rec(cvg, d.rec, &id);
   };
   DEntry nxt = fetch((long long)blockIdx.x * 256 + threadIdx.x);
@@ -1623,13 +1663,13 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
         auto kd = G >= 16 ? k_deferred_count<MODE, KIND, 16> : G >= 8 ? k_deferred_count<MODE, KIND, 8> : k_deferred_count<MODE, KIND, 4>;
         cudaFuncSetAttribute(kd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(hsm, 1));
         kd<<<sms, 1024, hsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o.counts, hs,
-                                   PIPE && !p.defer_xy ? p.xy : nullptr);
+                                   PIPE && !p.defer_xy ? p.xy : nullptr, COMPACT == 2 ? 1 : 0);
         launched = true;
       }
       if (!launched) {
         if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
         k_deferred<MODE, KIND><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh,
-                                                           PIPE && !p.defer_xy ? p.xy : nullptr, kcnt);
+                                                           PIPE && !p.defer_xy ? p.xy : nullptr, kcnt, COMPACT == 2 ? 1 : 0);
       }
       count_launch();
       e = cudaGetLastError();
@@ -1662,8 +1702,12 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
 
 template <int MODE, int QUEUE = 0, int PIPE = 0>
 int launch_layout(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
-  if (c->d.kind == kDisks)
+  // second level: 2 = dense uint16 (fine16), 1 = compact int32, 0 = dense int32
+  if (c->d.kind == kDisks) {
+    if (c->d.f16) return launch<MODE, 2, QUEUE, kDisks, PIPE>(c, xy, n, p, extra, st);
     return c->d.compact ? launch<MODE, 1, QUEUE, kDisks, PIPE>(c, xy, n, p, extra, st) : launch<MODE, 0, QUEUE, kDisks, PIPE>(c, xy, n, p, extra, st);
+  }
+  if (c->d.f16) return launch<MODE, 2, QUEUE, kPolygons, PIPE>(c, xy, n, p, extra, st);
   return c->d.compact ? launch<MODE, 1, QUEUE, kPolygons, PIPE>(c, xy, n, p, extra, st)
                       : launch<MODE, 0, QUEUE, kPolygons, PIPE>(c, xy, n, p, extra, st);
 }

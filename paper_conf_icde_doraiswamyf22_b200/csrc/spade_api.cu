@@ -120,7 +120,7 @@ void spade_canvas_free(spade_canvas* c) {
   if (!c) return;
   DeviceGuard dg(c->device);
   cudaDeviceSynchronize();
-  cudaFree(c->fine); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->recs); cudaFree(c->blob);
+  cudaFree(c->fine); cudaFree(c->fine16); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->recs); cudaFree(c->blob);
   cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->d_dev);
   delete c;
 }

@@ -20,6 +20,9 @@ constexpr int32_t kMultiMark = INT32_MIN;     // transient during the fill only
 // Compact layout (mix_min = 0x8000, needs P < 32767 and < 32768 mixed tiles): entry 0x8000|m and
 // the tile's pixels are the m-th block of 2^b x 2^b int32 in cfine (only mixed tiles stored).
 constexpr uint16_t kTileEmpty = 0, kTileMixed = 0xFFFF, kTileMixedCompact = 0x8000;
+// 16-bit copy of a dense fine canvas (P < 65534): code = owner id (< 0xFFFE), kF16Empty, or
+// kF16Record (boundary / multi-owner pixel: the record is found through the int32 canvas).
+constexpr uint16_t kF16Empty = 0xFFFE, kF16Record = 0xFFFF;
 
 // Boundary-index record as the build derives it (build intermediate; packed into Rec below).
 // For a boundary pixel: the distinct polygons whose edges touch the
@@ -79,6 +82,8 @@ struct CanvasDev {            // passed by value to kernels
   int32_t compact;            // 1: compact fine layout (cfine), 0: dense (fine)
   uint32_t mix_min;           // tile entries >= mix_min are mixed
   const int32_t* fine;        // dense W x H canvas (always present)
+  const uint16_t* fine16;     // 16-bit copy of it (f16 layout only; see kF16Record)
+  int32_t f16;                // 1: the probe's second level is fine16 (dense layout, P < 65534)
   const int32_t* cfine;       // compact mixed-tile blocks (compact layout only)
   const uint16_t* coarse;
   const Rec* recs;            // records: boundary pixels, then multi-owner pixels
@@ -100,6 +105,7 @@ struct spade_canvas {
   double mixed_tile_frac = 0.0;
   // owned device allocations
   int32_t* fine = nullptr;
+  uint16_t* fine16 = nullptr;
   int32_t* cfine = nullptr;
   uint16_t* coarse = nullptr;
   spade::Rec* recs = nullptr;
