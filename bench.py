@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu/clocks)")
     ap.add_argument("--dense", action="store_true", help="force the dense fine-canvas layout (A/B runs)")
     ap.add_argument("--max-dim", type=int, default=None, help="override the workload's canvas max_dim")
+    ap.add_argument("--opt", action="append", default=[], metavar="NAME=VALUE",
+                    help="spade_set_option before the run (A/B of probe paths; results never depend on it)")
     return ap.parse_args()
 
 
@@ -316,6 +318,9 @@ def main():
     if ws > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     sp.load()
+    for o in a.opt:
+        k, v = o.split("=")
+        sp.set_option(k, int(v))
     w = workload(a.workload, a.points_per_gpu)
     n = w.n_points
     is_dist = hasattr(w, "disks")
@@ -432,6 +437,7 @@ def main():
                 "parallelism": f"dp{ws} (points sharded, canvas replicated)",
                 "l2": "inputs (8 B/point, >= 8 GB per GPU) exceed the 126 MB L2; no flush needed",
                 "canvas": info, "canvas_build_s": build_s,
+                **({"options": a.opt} if a.opt else {}),
             },
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,

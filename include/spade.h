@@ -253,6 +253,8 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  merging K per point
  *   "host_chunk"   2^25 (default): points per staging chunk of the host-resident calls
  *                  (256 .. 2^28)
+ *   "fine16"       1 (default) / 0: probe canvases that have a 16-bit second level
+ *                  (SPADE_CANVAS_NO_FINE16 not set) through it, or through the int32 level
  *   "max_launch_points"  2^31 - 64 (default, the maximum): points per probe sub-launch; a call
  *                  with more points runs several sub-launches (each < 2^31 points: 32-bit point
  *                  offsets and per-record counters; the counters are spread over the owner sets

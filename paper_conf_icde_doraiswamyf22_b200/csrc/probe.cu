@@ -26,6 +26,7 @@
 #include <vector>
 #include <cstdio>
 #include <atomic>
+#include <type_traits>
 #include <cub/block/block_scan.cuh>
 #include <cub/block/block_radix_sort.cuh>
 #include <cub/block/block_reduce.cuh>
@@ -263,19 +264,21 @@ template <int KIND, int U, class PT, class MT>
 __device__ __forceinline__ uint64_t hit_mask(const PT* __restrict__ seg, const MT* __restrict__ msk, int ne, int X, int px, int py) {
   uint64_t m = 0;
   if (U > 1) {
+    // byte masks held in 32-bit registers (the deferred kernel runs at its register limit)
+    using MV = typename std::conditional<sizeof(MT) == 1, uint32_t, uint64_t>::type;
     for (int e0 = 0; e0 < ne; e0 += U) {
       int4 g[U];
-      uint64_t mk[U];
+      MV mk[U];
 #pragma unroll
       for (int k = 0; k < U; ++k) {
         const int e = e0 + k < ne ? e0 + k : ne - 1;     // clamped: in bounds, tested once
         g[k] = ld_prim(seg + e);
-        mk[k] = ld_mask(msk + e);
+        mk[k] = (MV)ld_mask(msk + e);
       }
 #pragma unroll
       for (int k = 0; k < U; ++k) {
         if (e0 + k >= ne) break;
-        if (prim_hit<KIND>(g[k], X, px, py)) m ^= mk[k];
+        if (prim_hit<KIND>(g[k], X, px, py)) m ^= (uint64_t)mk[k];
       }
     }
   } else {
@@ -1141,11 +1144,11 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
 // COUNT's second kernel, cooperative: the deferred boundary points of every CTA region, flattened;
 // each group of G lanes tests one point (group_mask), its first lane merges the result and counts
 // it (shared-memory histogram when the P bins fit, else warp-aggregated global atomics).
-template <int MODE, int KIND, int G>
+template <int MODE, int KIND, int G, int PIX>
 __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                             uint32_t cap, const unsigned int* __restrict__ fill, int nreg,
                                                             unsigned long long* __restrict__ counts, int smem_hist,
-                                                            const int2* __restrict__ pxy, int pix) {
+                                                            const int2* __restrict__ pxy) {
   constexpr int T = 1024, GPB = T / G;
   __shared__ long long s_pre[1025];              // exclusive prefix of the region fills
   extern __shared__ unsigned int dh[];
@@ -1176,7 +1179,7 @@ __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __r
     nxt = fetch(b0 + gstride + grp);             // the group's next point in flight meanwhile
     const bool act = e.rec != kHole;
     if (act && pxy) { const int2 q = __ldg(pxy + e.pidx); e.x = q.x; e.y = q.y; }   // entry without coordinates
-    if (act && pix) e.rec = rec_of_point(cvg, e.x, e.y);                         // fine16 canvas
+    if (act && PIX) e.rec = rec_of_point(cvg, e.x, e.y);                         // fine16 canvas
     Rec r{0u, kEmpty, 0, 0u};
     if (act) r = load_rec(cvg, e.rec);
     bool big;
@@ -1212,11 +1215,10 @@ __global__ void __launch_bounds__(1024, 1) k_deferred_count(const CanvasDev* __r
 // many blocks (one point per thread), exact test over the pixel's edges (pip_eval).  COUNT:
 // shared-memory histogram (or global atomics); SELECT/PAIRS: per-block count pass, block scan,
 // one global atomic, write pass.
-template <int MODE, int KIND>
+template <int MODE, int KIND, int PIX, int KAGG>
 __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict__ cvg, const DEntry* __restrict__ defer,
                                                   uint32_t cap, const unsigned int* __restrict__ fill, int nreg, Out o,
-                                                  int smem_hist, const int2* __restrict__ pxy, unsigned int* __restrict__ kcnt,
-                                                  int pix) {
+                                                  int smem_hist, const int2* __restrict__ pxy, unsigned int* __restrict__ kcnt) {
   using BS = cub::BlockScan<int, 256>;
   __shared__ typename BS::TempStorage tmp;
   __shared__ unsigned long long s_gb;
@@ -1249,8 +1251,8 @@ __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict
   auto rec_of = [&](DEntry& d, uint32_t& id) {
     if (d.rec == kHole) return Rec{0u, kEmpty, 0, 0u};
     if (pxy) { const int2 q = __ldg(pxy + d.pidx); d.x = q.x; d.y = q.y; }
-    if (pix) d.rec = rec_of_point(cvg, d.x, d.y);   // fine16 canvas: the record from the int32 level
-    return load_rec(cvg, d.rec, &id);
+    if (PIX) d.rec = rec_of_point(cvg, d.x, d.y);   // fine16 canvas: the record from the int32 level
+    return load_rec(cvg, d.rec, KAGG ? &id : nullptr);
   };
   DEntry nxt = fetch((long long)blockIdx.x * 256 + threadIdx.x);
   DEntry nxt2 = fetch((long long)blockIdx.x * 256 + gstride + threadIdx.x);
@@ -1265,7 +1267,7 @@ __global__ void __launch_bounds__(256, 4) k_deferred(const CanvasDev* __restrict
     nrec = rec_of(nxt, nid);
     const bool act = e.rec != kHole;
     const int64_t pid = o.id_base + (int64_t)e.pidx;
-    if ((MODE == kCountSmem || MODE == kCountGlobal) && kcnt) {
+    if ((MODE == kCountSmem || MODE == kCountGlobal) && KAGG) {
       if (act) pip_count_delta<KIND, 4>(cvg, e.x, e.y, rid, rc, kcnt, [&](int q, int d) {
         if (sh) atomicAdd(&dh[q], (unsigned int)d);
         else atomicAdd(o.counts + q, (unsigned long long)(long long)d);
@@ -1660,16 +1662,19 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
         const int G = coop > 0 ? coop : (epr > 10.0 ? 16 : epr > 4.0 ? 8 : 4);
         const int hs = (size_t)P * 4 <= 200 * 1024 ? 1 : 0;
         const size_t hsm = hs ? (size_t)P * 4 : 0;
-        auto kd = G >= 16 ? k_deferred_count<MODE, KIND, 16> : G >= 8 ? k_deferred_count<MODE, KIND, 8> : k_deferred_count<MODE, KIND, 4>;
+        constexpr int PX = COMPACT == 2;
+        auto kd = G >= 16 ? k_deferred_count<MODE, KIND, 16, PX> : G >= 8 ? k_deferred_count<MODE, KIND, 8, PX> : k_deferred_count<MODE, KIND, 4, PX>;
         cudaFuncSetAttribute(kd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(hsm, 1));
         kd<<<sms, 1024, hsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o.counts, hs,
-                                   PIPE && !p.defer_xy ? p.xy : nullptr, COMPACT == 2 ? 1 : 0);
+                                   PIPE && !p.defer_xy ? p.xy : nullptr);
         launched = true;
       }
       if (!launched) {
-        if (dsm > 48 * 1024) cudaFuncSetAttribute(k_deferred<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
-        k_deferred<MODE, KIND><<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh,
-                                                           PIPE && !p.defer_xy ? p.xy : nullptr, kcnt, COMPACT == 2 ? 1 : 0);
+        constexpr int PX = COMPACT == 2;
+        auto kd = kcnt ? k_deferred<MODE, KIND, PX, (MODE == kCountSmem || MODE == kCountGlobal)> : k_deferred<MODE, KIND, PX, 0>;
+        if (dsm > 48 * 1024) cudaFuncSetAttribute(kd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
+        kd<<<sms * 8, 256, dsm, st>>>(c->d_dev, dbuf, p.defer_cap, dfill, grid, p.o, sh,
+                                      PIPE && !p.defer_xy ? p.xy : nullptr, kcnt);
       }
       count_launch();
       e = cudaGetLastError();
@@ -1703,11 +1708,12 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
 template <int MODE, int QUEUE = 0, int PIPE = 0>
 int launch_layout(const spade_canvas* c, const int2* xy, int64_t n, const Params& p, size_t extra, cudaStream_t st) {
   // second level: 2 = dense uint16 (fine16), 1 = compact int32, 0 = dense int32
+  const bool f16 = c->d.f16 && options().fine16;
   if (c->d.kind == kDisks) {
-    if (c->d.f16) return launch<MODE, 2, QUEUE, kDisks, PIPE>(c, xy, n, p, extra, st);
+    if (f16) return launch<MODE, 2, QUEUE, kDisks, PIPE>(c, xy, n, p, extra, st);
     return c->d.compact ? launch<MODE, 1, QUEUE, kDisks, PIPE>(c, xy, n, p, extra, st) : launch<MODE, 0, QUEUE, kDisks, PIPE>(c, xy, n, p, extra, st);
   }
-  if (c->d.f16) return launch<MODE, 2, QUEUE, kPolygons, PIPE>(c, xy, n, p, extra, st);
+  if (f16) return launch<MODE, 2, QUEUE, kPolygons, PIPE>(c, xy, n, p, extra, st);
   return c->d.compact ? launch<MODE, 1, QUEUE, kPolygons, PIPE>(c, xy, n, p, extra, st)
                       : launch<MODE, 0, QUEUE, kPolygons, PIPE>(c, xy, n, p, extra, st);
 }

@@ -95,7 +95,7 @@ Options& options() {
   static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
                    env_int("SPADE_CACHE_SLOTS", 4096), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
                    env_int("SPADE_PIPE", -1), env_int("SPADE_DEFER_XY", 0), env_int("SPADE_L2_FRAC_PCT", 100), env_int("SPADE_MULTI_AGG", 1), env_int("SPADE_K_AGG", -1),
-                   (int64_t)1 << 25, (1ll << 31) - 64, 4096};
+                   (int64_t)1 << 25, (1ll << 31) - 64, 4096, env_int("SPADE_FINE16", 1)};
   return o;
 }
 }  // namespace spade
@@ -510,6 +510,7 @@ int spade_set_option(const char* name, int64_t value) {
   else if (n == "host_chunk" && value >= 256 && value <= ((int64_t)1 << 28)) o.host_chunk = value;
   else if (n == "max_launch_points" && value >= 256 && value <= (1ll << 31) - 64) o.max_launch_points = value;
   else if (n == "defer_budget_mb" && value >= 64 && value <= (1ll << 20)) o.defer_budget_mb = value;
+  else if (n == "fine16" && bit) o.fine16 = (int)value;
   else if (n == "coop" && (value == -1 || value == 0 || value == 4 || value == 8 || value == 16)) o.coop = (int)value;
   else return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: bad option %s = %lld", name, (long long)value);
   return SPADE_OK;

@@ -146,6 +146,7 @@ struct Options {
   int64_t host_chunk;         // points per staging chunk of the host-resident calls
   int64_t max_launch_points;  // points per probe sub-launch (< 2^31; smaller values: tests)
   int64_t defer_budget_mb;    // deferral scratch per sub-launch (16 B per reserved entry)
+  int fine16;                 // probe fine16 canvases through their 16-bit level (1) or the int32 one (0)
 };
 
 // Makes the canvas's device current for the duration of an entry point (restored after).
