@@ -820,6 +820,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   if (MODE == kCountSmem || MODE == kCountGlobal) {
     // COUNT (in-loop exact tests: the C3 configuration; or deferred: C5): written out without the
     // lambdas, which cost these register-bound variants a spill of the loop state
+    const uint32_t hist_s = (uint32_t)__cvta_generic_to_shared(myhist), hstride_b = 4u * prm.hcopies;
     Vec4 nxt;
     if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
     // (the stride is re-read from the special register each batch: kept live, it spilled)
@@ -915,7 +916,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
       if (MODE == kCountSmem) {
         // phase C2: direct hits (branch-free: non-hits and boundary points go to the trash bin P)
 #pragma unroll
-        for (int q = 0; q < NPT; ++q) atomicAdd(&myhist[min(c[q] - 1u, P) * prm.hcopies], 1u);
+        for (int q = 0; q < NPT; ++q)       // one IMAD per address: bin * (4 * copies) + this lane's copy
+          asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(min(c[q] - 1u, P) * hstride_b + hist_s) : "memory");
       } else {
         // phase C2, too many polygons for a shared-memory histogram: the count cache
 #pragma unroll
