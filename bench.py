@@ -328,18 +328,29 @@ def main():
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
 
-    # canvas build (timed separately; not part of a step); kNN builds no canvas (knn.cu)
+    # canvas build (timed separately; not part of a step); kNN builds no canvas (knn.cu).  Built
+    # twice: the first build also pays the CUDA module load of the build kernels ("cold"), the
+    # second is the steady-state cost; per-stage device times (CUDA events) of the second.
+    def build_canvas():
+        if w.op == "knn":
+            return None
+        if is_dist:
+            return sp.Canvas.disks(w.disks["center_xy"], w.disks["r2"], max_dim=a.max_dim or w.max_dim, dense=a.dense)
+        return sp.Canvas(w.polys, max_dim=a.max_dim or w.max_dim, dense=a.dense)
+
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    if w.op == "knn":
-        cv = None
-    elif is_dist:
-        cv = sp.Canvas.disks(w.disks["center_xy"], w.disks["r2"], max_dim=a.max_dim or w.max_dim, dense=a.dense)
-    else:
-        cv = sp.Canvas(w.polys, max_dim=a.max_dim or w.max_dim, dense=a.dense)
+    cv = build_canvas()
+    torch.cuda.synchronize()
+    build_cold_s = time.perf_counter() - t0
+    if cv is not None:
+        cv.close()
+    t0 = time.perf_counter()
+    cv = build_canvas()
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
     info = cv.info() if cv is not None else {}
+    build_stages = cv.build_times() if cv is not None else {}
 
     # this rank's shard: global indices [rank*n, (rank+1)*n), generated in place on the device
     xy = torch.empty((n, 2), dtype=torch.int32, device=dev)
@@ -393,6 +404,14 @@ def main():
     clocks = sampler.stop() if not a.profile else None
     t_ms = e0.elapsed_time(e1)
     kern_ms = [s.elapsed_time(t) for s, t in kev]
+    # per-stage breakdown of one more (untimed) step: CUDA events between the library's stages
+    stage_ms = None
+    if op in ("count", "select", "pairs"):
+        sp.set_option("stage_events", 1)
+        step()
+        torch.cuda.synchronize()
+        stage_ms = sp.last_call_stages()
+        sp.set_option("stage_events", 0)
     t_max = t_ms
     if ws > 1:
         tt = torch.tensor([t_ms], dtype=torch.float64, device=dev)
@@ -436,7 +455,8 @@ def main():
                    else {"polygons": P, "vertices": int(len(w.polys["ring_xy"]))}),
                 "parallelism": f"dp{ws} (points sharded, canvas replicated)",
                 "l2": "inputs (8 B/point, >= 8 GB per GPU) exceed the 126 MB L2; no flush needed",
-                "canvas": info, "canvas_build_s": build_s,
+                "canvas": info, "canvas_build_s": build_s, "canvas_build_cold_s": build_cold_s,
+                "canvas_build_stage_ms": build_stages,
                 **({"options": a.opt} if a.opt else {}),
             },
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -448,6 +468,7 @@ def main():
                          "kernel_ms": kavg, "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
                          "traffic_source": traffic_src},
             "gpu_launches": int(l1 - l0),
+            "stages_ms": stage_ms,
             "check": check,
         }
         if clocks:

@@ -120,6 +120,16 @@ SPADE_API int spade_canvas_info(const spade_canvas* c, int32_t* W, int32_t* H, i
                       int32_t* Wc, int32_t* Hc, int32_t* log2_tile,
                       int64_t* num_runs, int64_t* num_run_edges, double* mixed_tile_frac);
 
+/* Build profile (the paper's "polygon processing" cost): device time of each stage of
+ * this canvas's build, from CUDA events recorded on the build stream at the stage boundaries
+ * (each stage is also an NVTX range "spade_build:<name>").  Writes min(cap, stages) values (ms)
+ * and returns the number of stages (< 0: error); spade_canvas_build_stage_name(i) names stage i
+ * (NULL past the last).  Stages: K-B0 edges + extent, K-B1 fragments + events, K-B2 boundary
+ * pixels + pixel-local edge lists, K-B3 corner owner sets, K-B4/B6 K sets + packed records,
+ * K-B5 coarse tiles + compact / 16-bit levels.  An empty canvas has 0 stages. */
+SPADE_API int spade_canvas_build_times(const spade_canvas* c, float* ms, int32_t cap);
+SPADE_API const char* spade_canvas_build_stage_name(int32_t i);
+
 /* 64-bit checksum of everything the probe reads from the canvas (geometry, fine / compact /
  * coarse levels, records, primitive blobs, owner sets), written to *out (HOST).  Equal polygon
  * arrays give equal checksums on any device (the build is deterministic); ranks that replicate a
@@ -255,6 +265,9 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  (256 .. 2^28)
  *   "fine16"       1 (default) / 0: probe canvases that have a 16-bit second level
  *                  (SPADE_CANVAS_NO_FINE16 not set) through it, or through the int32 level
+ *   "stage_events" 0 (default) / 1: record CUDA events between the stages of every COUNT / SELECT /
+ *                  PAIRS call on its stream (synchronises once per sub-launch to read them; see
+ *                  spade_last_call_stages)
  *   "max_launch_points"  2^31 - 64 (default, the maximum): points per probe sub-launch; a call
  *                  with more points runs several sub-launches (each < 2^31 points: 32-bit point
  *                  offsets and per-record counters; the counters are spread over the owner sets
@@ -266,6 +279,13 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  spade_select / spade_join_pairs is <= this budget + ~0.2 GB of output
  *                  overflow and compaction tables, whatever n is (64 .. 2^20). */
 SPADE_API int spade_set_option(const char* name, int64_t value);
+
+/* Per-stage device time (ms) of this thread's last spade_join_count / spade_select /
+ * spade_join_pairs call, recorded when option "stage_events" is 1 (zeros otherwise), summed over
+ * its sub-launches: [0] probe kernel (stream, classify, in-loop exact tests, direct sinks),
+ * [1] deferred exact tests, [2] output compaction (SELECT / PAIRS), [3] per-record counter
+ * expansion (COUNT over overlapping polygons).  Writes min(cap, 4) values; returns 4. */
+SPADE_API int spade_last_call_stages(float* ms, int32_t cap);
 
 /* Number of kernels this library has launched in this process (for the bench's gpu_launches). */
 SPADE_API int64_t spade_launch_count(void);

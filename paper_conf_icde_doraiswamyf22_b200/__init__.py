@@ -67,6 +67,10 @@ def load(path: str | None = None):
     lib.spade_canvas_free.restype = None
     lib.spade_canvas_info.argtypes = [P] + [ctypes.POINTER(i32)] * 6 + [ctypes.POINTER(i64)] * 2 + [ctypes.POINTER(ctypes.c_double)]
     lib.spade_canvas_info.restype = ctypes.c_int
+    lib.spade_canvas_build_times.argtypes = [P, ctypes.POINTER(ctypes.c_float), i32]
+    lib.spade_canvas_build_times.restype = ctypes.c_int
+    lib.spade_canvas_build_stage_name.argtypes = [i32]
+    lib.spade_canvas_build_stage_name.restype = ctypes.c_char_p
     lib.spade_canvas_checksum.argtypes = [P, ctypes.POINTER(ctypes.c_uint64), P]
     lib.spade_canvas_checksum.restype = ctypes.c_int
     lib.spade_join_count.argtypes = [P, P, i64, P, P]
@@ -93,6 +97,8 @@ def load(path: str | None = None):
     lib.spade_knn.restype = ctypes.c_int
     lib.spade_set_option.argtypes = [ctypes.c_char_p, i64]
     lib.spade_set_option.restype = ctypes.c_int
+    lib.spade_last_call_stages.argtypes = [ctypes.POINTER(ctypes.c_float), i32]
+    lib.spade_last_call_stages.restype = ctypes.c_int
     lib.spade_launch_count.argtypes = []
     lib.spade_launch_count.restype = i64
     lib.spade_status_string.argtypes = [ctypes.c_int]
@@ -104,9 +110,9 @@ def load(path: str | None = None):
 
 
 EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canvas_free", "spade_canvas_info",
-                    "spade_canvas_checksum", "spade_join_count",
+                    "spade_canvas_checksum", "spade_canvas_build_times", "spade_canvas_build_stage_name", "spade_join_count",
                     "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_select_host", "spade_join_pairs_host", "spade_knn_histogram",
-                    "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_set_option", "spade_launch_count",
+                    "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_set_option", "spade_launch_count", "spade_last_call_stages",
                     "spade_status_string", "spade_last_error"]
 
 
@@ -186,6 +192,17 @@ def set_option(name: str, value: int) -> None:
     _check(load().spade_set_option(name.encode(), int(value)), f"set_option({name})")
 
 
+PROBE_STAGES = ["probe", "deferred exact tests", "output compaction", "counter expansion"]
+
+
+def last_call_stages() -> dict:
+    """Per-stage device ms of this thread's last COUNT / SELECT / PAIRS call (needs
+    set_option("stage_events", 1) before the call; spade_last_call_stages)."""
+    ms = (ctypes.c_float * 4)()
+    load().spade_last_call_stages(ms, 4)
+    return {k: float(v) for k, v in zip(PROBE_STAGES, ms)}
+
+
 def launch_count() -> int:
     return int(load().spade_launch_count())
 
@@ -250,6 +267,14 @@ class Canvas:
         W, H, s, Wc, Hc, b = (x.value for x in i32)
         return {"W": W, "H": H, "log2_pixel": s, "Wc": Wc, "Hc": Hc, "log2_tile": b,
                 "num_records": i64[0].value, "num_run_edges": i64[1].value, "mixed_tile_frac": d.value}
+
+    def build_times(self) -> dict:
+        """Device time (ms) of each build stage (spade_canvas_build_times; CUDA events)."""
+        ms = (ctypes.c_float * 8)()
+        n = self._lib.spade_canvas_build_times(self._h, ms, 8)
+        if n < 0:
+            _check(n, "spade_canvas_build_times")
+        return {self._lib.spade_canvas_build_stage_name(i).decode(): float(ms[i]) for i in range(n)}
 
     def close(self):
         if getattr(self, "_h", None):

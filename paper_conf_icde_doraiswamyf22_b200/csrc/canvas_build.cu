@@ -17,13 +17,51 @@
 //          cu(X, py) ^ cr(X, py) ^ cr(px, py))
 // where cr / cu are the half-open rightward / upward ray tests (perturbation reading of C1).
 #include <cub/cub.cuh>
+#include <nvtx3/nvToolsExt.h>
 #include <vector>
 #include <algorithm>
 #include "spade_internal.cuh"
 
 namespace spade {
 
+const char* const kBuildStageNames[kBuildStages] = {
+    "edges+extent (K-B0)",        "fragments+events (K-B1)",  "boundary pixels+local edges (K-B2)",
+    "corner owner sets (K-B3)",   "K sets+records (K-B4/B6)", "coarse tiles+compact+fine16 (K-B5)"};
+
 namespace {
+
+// CUDA events at the stage boundaries of one build (read after the build's final sync) and an
+// NVTX range per stage
+struct StageTimer {
+  cudaEvent_t ev[kBuildStages + 1] = {};
+  int n = 0;
+  cudaStream_t st;
+  explicit StageTimer(cudaStream_t s) : st(s) {}
+  void mark() {                                   // end of the previous stage / start of the next
+    if (n > kBuildStages) return;
+    if (n > 0) nvtxRangePop();
+    if (cudaEventCreate(&ev[n]) == cudaSuccess) cudaEventRecord(ev[n], st);
+    if (n < kBuildStages) {
+      char name[96];
+      snprintf(name, sizeof(name), "spade_build:%s", kBuildStageNames[n]);
+      nvtxRangePushA(name);
+    }
+    ++n;
+  }
+  void read(float* out, int* count) {             // after a sync of st
+    *count = 0;
+    for (int i = 0; i + 1 < n; ++i) {
+      float ms = 0.f;
+      if (ev[i] && ev[i + 1] && cudaEventElapsedTime(&ms, ev[i], ev[i + 1]) == cudaSuccess) out[i] = ms;
+      *count = i + 1;
+    }
+  }
+  ~StageTimer() {
+    if (n > 0 && n <= kBuildStages) nvtxRangePop();
+    for (cudaEvent_t e : ev)
+      if (e) cudaEventDestroy(e);
+  }
+};
 
 struct Geo {
   int64_t minx, miny;
@@ -125,38 +163,70 @@ __global__ void k_count(const int4* __restrict__ seg, int64_t E, Geo g, int64_t*
 
 struct Frag { int32_t j, ilo, ihi, e; };
 
+// Warp-cooperative loops: every lane owns one task (an edge, a fragment, an event pair) of n_i
+// items; tasks of at most kLongTask items are run by their own lane, longer ones by the whole
+// warp in turn (lanes split the items), so one long edge / fill span does not serialise its warp
+// (the fine-resolution canvases of small polygon sets: C1 at 1-unit pixels).
+constexpr int64_t kLongTask = 16;
+__device__ __forceinline__ int64_t shfl64(int64_t v, int src) {
+  return (int64_t)(((uint64_t)(uint32_t)__shfl_sync(0xffffffffu, (int)(v >> 32), src) << 32) |
+                   (uint32_t)__shfl_sync(0xffffffffu, (int)(uint32_t)v, src));
+}
+__device__ __forceinline__ int4 shfl4(int4 v, int src) {
+  return make_int4(__shfl_sync(0xffffffffu, v.x, src), __shfl_sync(0xffffffffu, v.y, src),
+                   __shfl_sync(0xffffffffu, v.z, src), __shfl_sync(0xffffffffu, v.w, src));
+}
+
+// one fragment of edge k at row j (closed pixels [ilo, ihi] it touches)
+__device__ __forceinline__ void emit_frag(int4 e, int32_t k, const Geo& g, int64_t j, int64_t o, Frag* frags, int64_t* frag_w) {
+  int ilo, ihi;
+  frag_cols(e, g, j, ilo, ihi);
+  frags[o] = Frag{(int32_t)j, ilo, ihi, k};
+  frag_w[o] = ihi >= ilo ? ihi - ilo + 1 : 0;
+}
 // event key: row | polygon | k,  k = 2c + (x* strictly inside column c ? 1 : 0), c = column of x*,
 // so that  x* > X_i  <=>  k > 2i  for every column i.
+__device__ __forceinline__ uint64_t event_key(int4 e, uint64_t pk, const Geo& g, int64_t j, int pbits, int kbits) {
+  const int64_t dx = (int64_t)e.z - e.x, dy = (int64_t)e.w - e.y;
+  const int64_t Y0 = g.miny + j * g.S;
+  const int64_t t = dx * (Y0 - e.y);
+  const int64_t xf = e.x + floor_div(t, dy);                  // floor of the crossing x*
+  const int64_t c = floor_div(xf - g.minx, g.S);              // pixel column holding x*
+  const bool exact = (t % dy == 0) && ((xf - g.minx) % g.S == 0);
+  const uint64_t kk = 2 * (uint64_t)c + (exact ? 0 : 1);
+  return ((uint64_t)j << (pbits + kbits)) | (pk << kbits) | kk;
+}
+
 __global__ void k_emit(const int4* __restrict__ seg, const int32_t* __restrict__ poly, int64_t E, Geo g,
                        const int64_t* __restrict__ frag_off, const int64_t* __restrict__ ev_off,
                        Frag* __restrict__ frags, int64_t* __restrict__ frag_w, uint64_t* __restrict__ ev_keys,
                        int pbits, int kbits) {
-  for (int64_t k = blockIdx.x * (int64_t)kBT + threadIdx.x; k < E; k += (int64_t)gridDim.x * kBT) {
-    int4 e = seg[k];
-    int64_t a, b;
-    if (!degenerate(e)) {
-      frag_rows(e, g, a, b);
-      int64_t o = frag_off[k];
-      for (int64_t j = a; j <= b; ++j, ++o) {
-        int ilo, ihi;
-        frag_cols(e, g, j, ilo, ihi);
-        frags[o] = Frag{(int32_t)j, ilo, ihi, (int32_t)k};
-        frag_w[o] = ihi >= ilo ? ihi - ilo + 1 : 0;
-      }
+  const int lane = threadIdx.x & 31;
+  for (int64_t kb = blockIdx.x * (int64_t)kBT + (threadIdx.x & ~31); kb < E; kb += (int64_t)gridDim.x * kBT) {
+    const int64_t k = kb + lane;
+    const bool act = k < E;
+    const int4 e = act ? seg[k] : make_int4(0, 0, 0, 0);
+    int64_t fa = 0, fb = -1, ea = 0, eb = -1, fo = 0, eo = 0;
+    uint64_t pk = 0;
+    if (act && !degenerate(e)) { frag_rows(e, g, fa, fb); fo = frag_off[k]; }
+    if (act && e.y != e.w) { event_rows(e, g, ea, eb); eo = ev_off[k]; pk = (uint64_t)poly[k]; }
+    const int64_t nf = fb >= fa ? fb - fa + 1 : 0, ne = eb >= ea ? eb - ea + 1 : 0;
+    if (nf <= kLongTask)
+      for (int64_t j = fa; j <= fb; ++j) emit_frag(e, (int32_t)k, g, j, fo + (j - fa), frags, frag_w);
+    if (ne <= kLongTask)
+      for (int64_t j = ea; j <= eb; ++j) ev_keys[eo + (j - ea)] = event_key(e, pk, g, j, pbits, kbits);
+    for (unsigned m = __ballot_sync(0xffffffffu, nf > kLongTask); m; m &= m - 1) {
+      const int src = __ffs(m) - 1;
+      const int4 es = shfl4(e, src);
+      const int64_t a = shfl64(fa, src), b = shfl64(fb, src), o = shfl64(fo, src);
+      for (int64_t j = a + lane; j <= b; j += 32) emit_frag(es, (int32_t)(kb + src), g, j, o + (j - a), frags, frag_w);
     }
-    if (e.y == e.w) continue;
-    event_rows(e, g, a, b);
-    int64_t o = ev_off[k];
-    int64_t dx = (int64_t)e.z - e.x, dy = (int64_t)e.w - e.y;
-    uint64_t pk = (uint64_t)poly[k];
-    for (int64_t j = a; j <= b; ++j, ++o) {
-      int64_t Y0 = g.miny + j * g.S;
-      int64_t t = dx * (Y0 - e.y);
-      int64_t xf = e.x + floor_div(t, dy);                  // floor of the crossing x*
-      int64_t c = floor_div(xf - g.minx, g.S);              // pixel column holding x*
-      bool exact = (t % dy == 0) && ((xf - g.minx) % g.S == 0);
-      uint64_t kk = 2 * (uint64_t)c + (exact ? 0 : 1);
-      ev_keys[o] = ((uint64_t)j << (pbits + kbits)) | (pk << kbits) | kk;
+    for (unsigned m = __ballot_sync(0xffffffffu, ne > kLongTask); m; m &= m - 1) {
+      const int src = __ffs(m) - 1;
+      const int4 es = shfl4(e, src);
+      const int64_t a = shfl64(ea, src), b = shfl64(eb, src), o = shfl64(eo, src);
+      const uint64_t pks = (uint64_t)shfl64((int64_t)pk, src);
+      for (int64_t j = a + lane; j <= b; j += 32) ev_keys[o + (j - a)] = event_key(es, pks, g, j, pbits, kbits);
     }
   }
 }
@@ -270,10 +340,20 @@ __global__ void k_demit(const int4* __restrict__ seg, int64_t E, Geo g, const in
 }
 
 __global__ void k_mark(const Frag* __restrict__ frags, int64_t F, int W, int32_t* __restrict__ bflag) {
-  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < F; t += (int64_t)gridDim.x * kBT) {
-    Frag f = frags[t];
+  const int lane = threadIdx.x & 31;
+  for (int64_t tb = blockIdx.x * (int64_t)kBT + (threadIdx.x & ~31); tb < F; tb += (int64_t)gridDim.x * kBT) {
+    const int64_t t = tb + lane;
+    const Frag f = t < F ? frags[t] : Frag{0, 1, 0, 0};
+    const int n = f.ihi - f.ilo + 1;
     int32_t* row = bflag + (int64_t)f.j * W;
-    for (int i = f.ilo; i <= f.ihi; ++i) row[i] = 1;
+    if (n <= kLongTask)
+      for (int i = f.ilo; i <= f.ihi; ++i) row[i] = 1;
+    for (unsigned m = __ballot_sync(0xffffffffu, n > kLongTask); m; m &= m - 1) {
+      const int src = __ffs(m) - 1;
+      const int j = __shfl_sync(0xffffffffu, f.j, src), lo = __shfl_sync(0xffffffffu, f.ilo, src),
+                hi = __shfl_sync(0xffffffffu, f.ihi, src);
+      for (int i = lo + lane; i <= hi; i += 32) bflag[(int64_t)j * W + i] = 1;
+    }
   }
 }
 
@@ -285,18 +365,33 @@ __global__ void k_bids(const int32_t* __restrict__ bflag, const int32_t* __restr
 }
 
 // one (boundary pixel, edge) entry per pixel of every fragment
+__device__ __forceinline__ void local_entry(const int32_t* __restrict__ bscan, int64_t p, int64_t o, uint32_t pk, int32_t e,
+                                            uint64_t* __restrict__ keys, int32_t* __restrict__ vals, int32_t* __restrict__ cnt) {
+  const int32_t bid = bscan[p] - 1;
+  keys[o] = ((uint64_t)(uint32_t)bid << 32) | pk;
+  vals[o] = e;
+  atomicAdd(&cnt[bid], 1);
+}
 __global__ void k_local(const Frag* __restrict__ frags, int64_t F, int W, const int64_t* __restrict__ lw_off,
                         const int32_t* __restrict__ poly, const int32_t* __restrict__ bscan,
                         uint64_t* __restrict__ keys, int32_t* __restrict__ vals, int32_t* __restrict__ cnt) {
-  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < F; t += (int64_t)gridDim.x * kBT) {
-    Frag f = frags[t];
-    int64_t o = lw_off[t];
-    uint32_t pk = (uint32_t)poly[f.e];
-    for (int i = f.ilo; i <= f.ihi; ++i, ++o) {
-      int32_t bid = bscan[(int64_t)f.j * W + i] - 1;
-      keys[o] = ((uint64_t)(uint32_t)bid << 32) | pk;
-      vals[o] = f.e;
-      atomicAdd(&cnt[bid], 1);
+  const int lane = threadIdx.x & 31;
+  for (int64_t tb = blockIdx.x * (int64_t)kBT + (threadIdx.x & ~31); tb < F; tb += (int64_t)gridDim.x * kBT) {
+    const int64_t t = tb + lane;
+    const bool act = t < F;
+    const Frag f = act ? frags[t] : Frag{0, 1, 0, 0};
+    const int64_t o = act ? lw_off[t] : 0;
+    const uint32_t pk = act ? (uint32_t)poly[f.e] : 0u;
+    const int n = f.ihi - f.ilo + 1;
+    if (n <= kLongTask)
+      for (int i = f.ilo; i <= f.ihi; ++i) local_entry(bscan, (int64_t)f.j * W + i, o + (i - f.ilo), pk, f.e, keys, vals, cnt);
+    for (unsigned m = __ballot_sync(0xffffffffu, n > kLongTask); m; m &= m - 1) {
+      const int src = __ffs(m) - 1;
+      const int j = __shfl_sync(0xffffffffu, f.j, src), lo = __shfl_sync(0xffffffffu, f.ilo, src),
+                hi = __shfl_sync(0xffffffffu, f.ihi, src), es = __shfl_sync(0xffffffffu, f.e, src);
+      const int64_t os = shfl64(o, src);
+      const uint32_t pks = (uint32_t)__shfl_sync(0xffffffffu, (int)pk, src);
+      for (int i = lo + lane; i <= hi; i += 32) local_entry(bscan, (int64_t)j * W + i, os + (i - lo), pks, es, keys, vals, cnt);
     }
   }
 }
@@ -406,28 +501,49 @@ __global__ void k_merge(const uint64_t* __restrict__ key2, const int32_t* __rest
 // K-B3: sorted events of one (row, polygon) come in consecutive pairs (a closed ring crosses a
 // horizontal line an even number of times).  Polygon P contains the lower-left corner of pixel
 // i iff 2i lies in [k_a, k_b) for a pair, i.e. i in [ceil(k_a/2), ceil(k_b/2) - 1].
+__device__ __forceinline__ void fill_pixel(int32_t* __restrict__ corner, int64_t j, int W, int i, int32_t p,
+                                           unsigned long long* __restrict__ multi, unsigned long long* __restrict__ nmulti,
+                                           int64_t multi_cap) {
+  int32_t* row = corner + j * W;
+  const int old = atomicCAS(&row[i], kEmpty, p);
+  if (old == kEmpty) return;
+  const int prev = atomicExch(&row[i], kMultiMark);
+  const unsigned long long q = atomicAdd(nmulti, prev >= 0 ? 2ull : 1ull);
+  const uint64_t px = (uint64_t)(j * W + i);
+  if ((int64_t)q < multi_cap) multi[q] = (px << 32) | (uint32_t)p;
+  if (prev >= 0 && (int64_t)q + 1 < multi_cap) multi[q + 1] = (px << 32) | (uint32_t)prev;
+}
 __global__ void k_fill(const uint64_t* __restrict__ ev, int64_t NE, int W, int pbits, int kbits,
                        int32_t* __restrict__ corner, unsigned long long* __restrict__ multi,
                        unsigned long long* __restrict__ nmulti, int64_t multi_cap, int* __restrict__ bad) {
   const uint64_t kmask = (1ull << kbits) - 1, pmask = (1ull << pbits) - 1;
   const int64_t NP = NE / 2;
+  const int lane = threadIdx.x & 31;
   if (blockIdx.x == 0 && threadIdx.x == 0 && (NE & 1)) atomicOr(bad, 2);
-  for (int64_t t = blockIdx.x * (int64_t)kBT + threadIdx.x; t < NP; t += (int64_t)gridDim.x * kBT) {
-    uint64_t k0 = ev[2 * t], k1 = ev[2 * t + 1];
-    if ((k0 >> kbits) != (k1 >> kbits)) { atomicOr(bad, 2); continue; }
-    int64_t j = (int64_t)(k0 >> (kbits + pbits));
-    int32_t p = (int32_t)((k0 >> kbits) & pmask);
-    int64_t ka = (int64_t)(k0 & kmask), kb = (int64_t)(k1 & kmask);
-    int i0 = (int)((ka + 1) >> 1), i1 = (int)((kb + 1) >> 1);   // [ceil(ka/2), ceil(kb/2))
-    int32_t* row = corner + j * W;
-    for (int i = i0; i < i1; ++i) {
-      int old = atomicCAS(&row[i], kEmpty, p);
-      if (old == kEmpty) continue;
-      int prev = atomicExch(&row[i], kMultiMark);
-      unsigned long long q = atomicAdd(nmulti, prev >= 0 ? 2ull : 1ull);
-      const uint64_t px = (uint64_t)(j * W + i);
-      if ((int64_t)q < multi_cap) multi[q] = (px << 32) | (uint32_t)p;
-      if (prev >= 0 && (int64_t)q + 1 < multi_cap) multi[q + 1] = (px << 32) | (uint32_t)prev;
+  for (int64_t tb = blockIdx.x * (int64_t)kBT + (threadIdx.x & ~31); tb < NP; tb += (int64_t)gridDim.x * kBT) {
+    const int64_t t = tb + lane;
+    int64_t j = 0;
+    int32_t p = 0;
+    int i0 = 0, i1 = 0;
+    if (t < NP) {
+      const uint64_t k0 = ev[2 * t], k1 = ev[2 * t + 1];
+      if ((k0 >> kbits) != (k1 >> kbits)) {
+        atomicOr(bad, 2);
+      } else {
+        j = (int64_t)(k0 >> (kbits + pbits));
+        p = (int32_t)((k0 >> kbits) & pmask);
+        const int64_t ka = (int64_t)(k0 & kmask), kb = (int64_t)(k1 & kmask);
+        i0 = (int)((ka + 1) >> 1); i1 = (int)((kb + 1) >> 1);    // [ceil(ka/2), ceil(kb/2))
+      }
+    }
+    if (i1 - i0 <= kLongTask)
+      for (int i = i0; i < i1; ++i) fill_pixel(corner, j, W, i, p, multi, nmulti, multi_cap);
+    for (unsigned m = __ballot_sync(0xffffffffu, i1 - i0 > kLongTask); m; m &= m - 1) {
+      const int src = __ffs(m) - 1;
+      const int64_t js = shfl64(j, src);
+      const int32_t ps = __shfl_sync(0xffffffffu, p, src);
+      const int a = __shfl_sync(0xffffffffu, i0, src), b = __shfl_sync(0xffffffffu, i1, src);
+      for (int i = a + lane; i < b; i += 32) fill_pixel(corner, js, W, i, ps, multi, nmulti, multi_cap);
     }
   }
 }
@@ -773,6 +889,8 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
 #define ALLOC(ptr, n, what) TRYF(tmp.alloc(&ptr, (size_t)(n)), what)
 #define LAUNCH(kern, n, ...) do { kern<<<grid_for(n), kBT, 0, st>>>(__VA_ARGS__); count_launch(); TRYF(cudaGetLastError(), #kern); } while (0)
 
+  StageTimer stages(st);
+  stages.mark();                                   // K-B0
   DevBufs tmp;
   int4* seg; int32_t* epoly; int* ext; int* bad;
   ALLOC(seg, V, "edges"); ALLOC(epoly, V, "edges"); ALLOC(ext, 4, "ext"); ALLOC(bad, 1, "flag");
@@ -819,6 +937,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   const int64_t WH = (int64_t)g.W * g.H;
 
   // --- K-B1 counts, scans, emit ---
+  stages.mark();
   int64_t *nfrag, *nev, *frag_off, *ev_off;
   ALLOC(nfrag, V, "counts"); ALLOC(nev, V, "counts"); ALLOC(frag_off, V + 1, "counts"); ALLOC(ev_off, V + 1, "counts");
   if (kind == kPolygons) LAUNCH(k_count, V, seg, V, g, nfrag, nev);
@@ -843,6 +962,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   else LAUNCH(k_demit, V, seg, V, g, frag_off, ev_off, frags, frag_w, ev, pbits, kbits);
 
   // --- K-B2 boundary pixels, ids, pixel-local edge lists ---
+  stages.mark();
   int32_t *bflag, *bscan;
   ALLOC(bflag, WH, "boundary flags"); ALLOC(bscan, WH, "boundary ids");
   TRYF(cudaMemsetAsync(bflag, 0, sizeof(int32_t) * WH, st), "memset");
@@ -915,6 +1035,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   tmp.release(ph); tmp.release(pg); tmp.release(li); tmp.release(tix); tmp.release(tix2); tmp.release(key2s);
 
   // --- K-B3 corner owner sets ---
+  stages.mark();
   uint64_t* ev2;
   ALLOC(ev2, NE, "events");
   if (NE > 0)
@@ -960,6 +1081,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   tmp.release(multi);
 
   // --- K-B4 K sets of boundary pixels, records, final canvas ---
+  stages.mark();
   int32_t *ksize, *kidx; int64_t* koff;
   ALLOC(ksize, NB, "K sizes"); ALLOC(kidx, NB, "K sizes"); ALLOC(koff, NB + 1, "K offsets");
   int64_t KT = 0; int64_t NK = 0;
@@ -1020,6 +1142,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, boff, c->fine);
 
   // --- K-B5 coarse tiles (+ compact fine layout) ---
+  stages.mark();
   const int64_t NT = (int64_t)Wc * Hc;
   int32_t *tval, *tmix, *mscan;
   ALLOC(tval, NT, "tiles"); ALLOC(tmix, NT, "tiles"); ALLOC(mscan, NT, "tiles");
@@ -1047,7 +1170,9 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
     if (cudaMalloc(&c->fine16, sizeof(uint16_t) * WH) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: fine16"));
     LAUNCH(k_fine16, WH, c->fine, WH, c->fine16);
   }
+  stages.mark();                                   // end of K-B5
   TRYF(cudaStreamSynchronize(st), "sync compact");
+  stages.read(c->stage_ms, &c->num_stages);
 #undef TRYF
 #undef ALLOC
 #undef LAUNCH

@@ -1508,6 +1508,30 @@ __global__ void __launch_bounds__(256) k_multi_expand(const CanvasDev* __restric
   }
 }
 
+// Optional per-stage CUDA events of the last probe call (spade_set_option "stage_events"; read
+// with spade_last_call_stages): probe kernel, deferred exact tests, output compaction, per-record
+// counter expansion, summed over the call's sub-launches.
+struct StageEvents {
+  static constexpr int kN = kProbeStages;
+  cudaEvent_t ev[kN + 1] = {};
+  float acc[kN] = {};
+  bool on = false;
+  cudaStream_t st = nullptr;
+  void begin(cudaStream_t s) {
+    on = options().stage_events != 0;
+    if (!on) return;
+    st = s;
+    for (int i = 0; i <= kN; ++i) if (!ev[i]) cudaEventCreate(&ev[i]);
+  }
+  void rec(int i) { if (on) cudaEventRecord(ev[i], st); }
+  void add() {                                    // after rec(0..kN) of one sub-launch: accumulate
+    if (!on) return;
+    cudaEventSynchronize(ev[kN]);
+    for (int i = 0; i < kN; ++i) { float ms = 0.f; cudaEventElapsedTime(&ms, ev[i], ev[i + 1]); acc[i] += ms; }
+  }
+};
+thread_local StageEvents g_stages;
+
 // Stream-ordered device scratch freed on every exit path (errors included).
 struct ScratchGuard {
   void* p = nullptr;
@@ -1526,6 +1550,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
   const int sms = device_sm_count();
   keep_pool_memory();
+  g_stages.begin(st);
   // COUNT over a canvas with multi-owner pixels: per-record counters (count_multi_owner)
   constexpr bool kCnt = MODE == kCountSmem || MODE == kCountGlobal;
   const uint32_t num_multi = kCnt && options().multi_agg ? (uint32_t)(c->num_records - c->num_runs) : 0u;
@@ -1649,9 +1674,11 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.l2_frac = (float)options().l2_frac_pct * 0.01f;
     p.defer_cap = (uint32_t)per;
     p.defer_fill = dfill;
+    g_stages.rec(0);
     kern<<<grid, kT, smem, st>>>(p);
     count_launch();
     e = cudaGetLastError();
+    g_stages.rec(1);
     if (e == cudaSuccess && !QUEUE) {
       const int P = c->d.num_polys;
       const int sh = ((MODE == kCountSmem || MODE == kCountGlobal) && (size_t)P * 4 <= 96 * 1024) ? 1 : 0;
@@ -1691,6 +1718,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
                 tot, (long long)m, 100.0 * tot / m, mx, (long long)per, (long long)c->num_runs, (long long)c->num_run_edges);
       }
     }
+    g_stages.rec(2);
     if (kOut && e == cudaSuccess) {
       k_fixup<<<1, kFixT, 0, st>>>(p.o.holes, grid * kNW, p.o.total, p.o.cap, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
       count_launch();
@@ -1700,9 +1728,12 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       count_launch();
       e = cudaGetLastError();
     }
+    g_stages.rec(3);
     if (e != cudaSuccess) return check_cuda(e, "probe launch");
     const int rc = expand(off + m < n);
     if (rc != SPADE_OK) return rc;
+    g_stages.rec(4);
+    g_stages.add();
   }
   return SPADE_OK;
 }
@@ -1736,7 +1767,15 @@ bool use_queue(const spade_canvas* c, int mode) {
 
 }  // namespace
 
+int last_call_stages(float* ms, int cap) {
+  int n = 0;
+  for (; n < kProbeStages && n < cap; ++n) ms[n] = g_stages.acc[n];
+  return kProbeStages;
+}
+void reset_call_stages() { for (float& a : g_stages.acc) a = 0.f; }
+
 int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts, cudaStream_t st) {
+  reset_call_stages();
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.counts = (unsigned long long*)counts;
@@ -1801,6 +1840,7 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
 
 int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* out, int64_t cap,
                   unsigned long long* d_total, cudaStream_t st) {
+  reset_call_stages();
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = out; p.o.cap = cap; p.o.total = d_total;
@@ -1810,6 +1850,7 @@ int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t b
 
 int launch_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* opt, int32_t* opl,
                  int64_t cap, unsigned long long* d_total, cudaStream_t st) {
+  reset_call_stages();
   if (c->empty || n == 0) return SPADE_OK;
   Params p = base_params(c);
   p.o.id_base = base; p.o.out_ids = opt; p.o.out_poly = opl; p.o.cap = cap; p.o.total = d_total;

@@ -9,9 +9,16 @@
 #include <atomic>
 #include <algorithm>
 #include <vector>
+#include <nvtx3/nvToolsExt.h>
 #include "spade_internal.cuh"
 
 namespace spade {
+
+// NVTX range for the duration of one entry point (visible in nsys / ncu --nvtx)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 int build_canvas(const int32_t*, const int64_t*, const int64_t*, int32_t, const spade_canvas_params*, cudaStream_t,
                  spade_canvas**);
@@ -95,7 +102,8 @@ Options& options() {
   static Options o{env_int("SPADE_DEFER", 0), env_int("SPADE_COUNT_GLOBAL", 0), env_int("SPADE_GLOBAL_QUEUE", 0),
                    env_int("SPADE_CACHE_SLOTS", 4096), env_int("SPADE_COOP", 0), env_int("SPADE_DEBUG_DEFER", 0),
                    env_int("SPADE_PIPE", -1), env_int("SPADE_DEFER_XY", 0), env_int("SPADE_L2_FRAC_PCT", 100), env_int("SPADE_MULTI_AGG", 1), env_int("SPADE_K_AGG", -1),
-                   (int64_t)1 << 25, (1ll << 31) - 64, 4096, env_int("SPADE_FINE16", 1)};
+                   (int64_t)1 << 25, (1ll << 31) - 64, 4096, env_int("SPADE_FINE16", 1),
+                   env_int("SPADE_STAGE_EVENTS", 0)};
   return o;
 }
 }  // namespace spade
@@ -106,6 +114,7 @@ int spade_build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const in
                        int32_t num_polys, const spade_canvas_params* prm, spade_stream_t stream, spade_canvas** out) {
   if (!out) return set_error(SPADE_ERR_INVALID_ARG, "spade_build_canvas: out is NULL");
   *out = nullptr;
+  NvtxRange nv("spade_build_canvas");
   return build_canvas(ring_xy, ring_off, poly_ring_off, num_polys, prm, (cudaStream_t)stream, out);
 }
 
@@ -113,6 +122,7 @@ int spade_build_disk_canvas(const int32_t* center_xy, const int64_t* r2, int32_t
                             const spade_canvas_params* prm, spade_stream_t stream, spade_canvas** out) {
   if (!out) return set_error(SPADE_ERR_INVALID_ARG, "spade_build_disk_canvas: out is NULL");
   *out = nullptr;
+  NvtxRange nv("spade_build_disk_canvas");
   return build_disk_canvas(center_xy, r2, num_disks, prm, (cudaStream_t)stream, out);
 }
 
@@ -140,6 +150,16 @@ int spade_canvas_info(const spade_canvas* c, int32_t* W, int32_t* H, int32_t* lo
   return SPADE_OK;
 }
 
+int spade_canvas_build_times(const spade_canvas* c, float* ms, int32_t cap) {
+  if (!c || (cap > 0 && !ms) || cap < 0) return set_error(SPADE_ERR_INVALID_ARG, "spade_canvas_build_times: bad arguments");
+  for (int i = 0; i < c->num_stages && i < cap; ++i) ms[i] = c->stage_ms[i];
+  return c->num_stages;
+}
+
+const char* spade_canvas_build_stage_name(int32_t i) {
+  return i >= 0 && i < kBuildStages ? kBuildStageNames[i] : nullptr;
+}
+
 int spade_canvas_checksum(const spade_canvas* c, uint64_t* out, spade_stream_t stream) {
   if (!c || !out) return set_error(SPADE_ERR_INVALID_ARG, "spade_canvas_checksum: NULL argument");
   DeviceGuard dg(c->device);
@@ -151,6 +171,7 @@ int spade_join_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_
   if (rc) return rc;
   if (c->d.num_polys > 0 && !counts) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_count: counts is NULL");
   DeviceGuard dg(c->device);
+  NvtxRange nv("spade_join_count");
   return launch_count(c, xy, n, counts, (cudaStream_t)stream);
 }
 
@@ -160,6 +181,7 @@ int spade_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t po
   if (rc) return rc;
   if (capacity > 0 && !out_ids) return set_error(SPADE_ERR_INVALID_ARG, "spade_select: out_ids is NULL");
   DeviceGuard dg(c->device);
+  NvtxRange nv("spade_select");
   return run_with_capacity(capacity, n_out, (cudaStream_t)stream, "spade_select", [&](unsigned long long* t) {
     return launch_select(c, xy, n, point_id_base, out_ids, capacity, t, (cudaStream_t)stream);
   });
@@ -172,6 +194,7 @@ int spade_join_pairs(const spade_canvas* c, const int32_t* xy, int64_t n, int64_
   if (capacity > 0 && (!out_point_ids || !out_poly_ids))
     return set_error(SPADE_ERR_INVALID_ARG, "spade_join_pairs: output arrays are NULL");
   DeviceGuard dg(c->device);
+  NvtxRange nv("spade_join_pairs");
   return run_with_capacity(capacity, n_out, (cudaStream_t)stream, "spade_join_pairs", [&](unsigned long long* t) {
     return launch_pairs(c, xy, n, point_id_base, out_point_ids, out_poly_ids, capacity, t, (cudaStream_t)stream);
   });
@@ -188,6 +211,7 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
   if (P > 0 && !counts_host) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_count_host: counts_host is NULL");
   if (n == 0 || P == 0) return SPADE_OK;
   DeviceGuard dg(c->device);
+  NvtxRange nv("spade_join_count_host");
   cudaStream_t st = (cudaStream_t)stream;
   const int64_t kChunk = options().host_chunk;  // default 32 Mi points = 256 MiB per staging buffer
   const int64_t chunk = std::min(kChunk, n);
@@ -260,6 +284,7 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
 static int map_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, int64_t base, int64_t* out_ids,
                     int32_t* out_polys, int64_t capacity, int64_t* n_out, cudaStream_t st, const char* fn) {
   DeviceGuard dg(c->device);
+  NvtxRange nv(fn);
   const bool pairs = out_polys != nullptr || std::string(fn) == "spade_join_pairs_host";
   const int64_t chunk = std::min(options().host_chunk, n);
   int32_t* stage[2] = {nullptr, nullptr};
@@ -489,6 +514,11 @@ int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int32_t qx, i
 
 int64_t spade_launch_count(void) { return g_launches.load(); }
 
+int spade_last_call_stages(float* ms, int32_t cap) {
+  if (cap < 0 || (cap > 0 && !ms)) return set_error(SPADE_ERR_INVALID_ARG, "spade_last_call_stages: bad arguments");
+  return spade::last_call_stages(ms, cap);
+}
+
 
 int spade_set_option(const char* name, int64_t value) {
   using spade::set_error;
@@ -511,6 +541,7 @@ int spade_set_option(const char* name, int64_t value) {
   else if (n == "max_launch_points" && value >= 256 && value <= (1ll << 31) - 64) o.max_launch_points = value;
   else if (n == "defer_budget_mb" && value >= 64 && value <= (1ll << 20)) o.defer_budget_mb = value;
   else if (n == "fine16" && bit) o.fine16 = (int)value;
+  else if (n == "stage_events" && bit) o.stage_events = (int)value;
   else if (n == "coop" && (value == -1 || value == 0 || value == 4 || value == 8 || value == 16)) o.coop = (int)value;
   else return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: bad option %s = %lld", name, (long long)value);
   return SPADE_OK;

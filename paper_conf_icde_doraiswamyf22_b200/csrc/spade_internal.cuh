@@ -102,6 +102,8 @@ struct spade_canvas {
   int64_t num_runs = 0, num_records = 0, num_run_edges = 0, num_set_entries = 0;
   int64_t num_set_ranges = 0, cfine_elems = 0, coarse_elems = 0;   // array sizes (checksum)
   int64_t multi_unit = 0;     // blob offset of the first multi-owner record header
+  float stage_ms[8] = {};     // build stage times (CUDA events on the build stream; spade_canvas_build_times)
+  int num_stages = 0;
   double mixed_tile_frac = 0.0;
   // owned device allocations
   int32_t* fine = nullptr;
@@ -117,6 +119,10 @@ struct spade_canvas {
 };
 
 namespace spade {
+
+// Canvas build stages (timed with CUDA events, NVTX ranges "spade_build:<name>")
+constexpr int kBuildStages = 6;
+extern const char* const kBuildStageNames[kBuildStages];
 
 // Fine pixel index of pixel (fx, fy) whose coarse tile entry is the mixed value t.
 __host__ __device__ __forceinline__ const int32_t* fine_ptr(const CanvasDev& cv, uint32_t t, uint32_t fx, uint32_t fy) {
@@ -147,7 +153,10 @@ struct Options {
   int64_t max_launch_points;  // points per probe sub-launch (< 2^31; smaller values: tests)
   int64_t defer_budget_mb;    // deferral scratch per sub-launch (16 B per reserved entry)
   int fine16;                 // probe fine16 canvases through their 16-bit level (1) or the int32 one (0)
+  int stage_events;           // record per-stage CUDA events in every probe call (spade_last_call_stages)
 };
+constexpr int kProbeStages = 4;   // probe, deferred exact tests, output compaction, counter expansion
+int last_call_stages(float* ms, int cap);
 
 // Makes the canvas's device current for the duration of an entry point (restored after).
 struct DeviceGuard {

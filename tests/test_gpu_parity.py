@@ -322,3 +322,36 @@ def test_exact_capacity_and_compaction(spade, op):
         np.testing.assert_array_equal(b, opl)
     else:
         np.testing.assert_array_equal(np.sort(pt[:M].cpu().numpy()), oids)
+
+
+def test_build_profile_and_call_stages(spade):
+    """spade_canvas_build_times: one device time per build stage (CUDA events), bounded by the
+    build's wall time; spade_last_call_stages: per-stage times of the last call when the
+    stage_events option is on, zeros when off; results unchanged either way."""
+    import time
+    import torch
+    w = configs.c4(1)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    cv = spade.Canvas(w.polys, max_dim=w.max_dim)
+    torch.cuda.synchronize()
+    wall_ms = 1e3 * (time.perf_counter() - t0)
+    bt = cv.build_times()
+    assert len(bt) == 6 and all(v >= 0 for v in bt.values())
+    assert 0 < sum(bt.values()) <= wall_ms * 1.05
+    xy_h = gen.points_host(w.points, w.point_seed, 0, 200_000)
+    xy = torch.as_tensor(xy_h).cuda()
+    spade.set_option("stage_events", 1)
+    try:
+        c1 = spade.join_count(cv, xy).cpu().numpy()
+        st = spade.last_call_stages()
+        pt, pl = spade.join_pairs(cv, xy)
+        st2 = spade.last_call_stages()
+    finally:
+        spade.set_option("stage_events", 0)
+    assert st["probe"] > 0 and st["output compaction"] == 0
+    assert st2["probe"] > 0 and st2["output compaction"] > 0
+    c0 = spade.join_count(cv, xy).cpu().numpy()
+    assert all(v == 0 for v in spade.last_call_stages().values())
+    np.testing.assert_array_equal(c0, c1)
+    np.testing.assert_array_equal(c0, oracle.join_count(xy_h, w.polys))
