@@ -343,12 +343,13 @@ def main():
     cv = build_canvas()
     torch.cuda.synchronize()
     build_cold_s = time.perf_counter() - t0
-    if cv is not None:
-        cv.close()
     t0 = time.perf_counter()
-    cv = build_canvas()
+    cv2 = build_canvas()
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
+    if cv is not None:
+        cv.close()
+    cv = cv2
     info = cv.info() if cv is not None else {}
     build_stages = cv.build_times() if cv is not None else {}
 

@@ -793,17 +793,21 @@ int bits_for(int64_t v) {  // bits to hold values 0..v
   return b;
 }
 
+// Build temporaries: stream-ordered allocations from the device's memory pool (kept by the pool
+// between builds, keep_pool_memory), freed on the build stream.
 struct DevBufs {
   std::vector<void*> ptrs;
-  ~DevBufs() { for (void* p : ptrs) cudaFree(p); }
+  cudaStream_t st;
+  explicit DevBufs(cudaStream_t s) : st(s) {}
+  ~DevBufs() { for (void* p : ptrs) cudaFreeAsync(p, st); }
   template <class T> cudaError_t alloc(T** p, size_t count) {
-    cudaError_t e = cudaMalloc((void**)p, std::max<size_t>(count, 1) * sizeof(T));
+    cudaError_t e = cudaMallocAsync((void**)p, std::max<size_t>(count, 1) * sizeof(T), st);
     if (e == cudaSuccess) ptrs.push_back(*p); else *p = nullptr;
     return e;
   }
   void release(void* p) {
     auto it = std::find(ptrs.begin(), ptrs.end(), p);
-    if (it != ptrs.end()) { cudaFree(p); ptrs.erase(it); }
+    if (it != ptrs.end()) { cudaFreeAsync(p, st); ptrs.erase(it); }
   }
 };
 
@@ -889,9 +893,10 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
 #define ALLOC(ptr, n, what) TRYF(tmp.alloc(&ptr, (size_t)(n)), what)
 #define LAUNCH(kern, n, ...) do { kern<<<grid_for(n), kBT, 0, st>>>(__VA_ARGS__); count_launch(); TRYF(cudaGetLastError(), #kern); } while (0)
 
+  keep_pool_memory();
   StageTimer stages(st);
   stages.mark();                                   // K-B0
-  DevBufs tmp;
+  DevBufs tmp(st);
   int4* seg; int32_t* epoly; int* ext; int* bad;
   ALLOC(seg, V, "edges"); ALLOC(epoly, V, "edges"); ALLOC(ext, 4, "ext"); ALLOC(bad, 1, "flag");
   int h_ext0[4] = {INT_MAX, INT_MAX, INT_MIN, INT_MIN};

@@ -1478,6 +1478,8 @@ __global__ void __launch_bounds__(1024) k_move(Out o, const long long* __restric
 // Stream-ordered scratch comes from the device's default memory pool; by default the pool hands
 // memory back to the driver at every synchronisation, which made each call re-map its scratch.
 // Set once per device (the caller's current device, which the entry points switch to the canvas's).
+}  // namespace
+
 void keep_pool_memory() {
   static std::atomic<uint64_t> done{0};
   int dev = 0;
@@ -1491,6 +1493,8 @@ void keep_pool_memory() {
   }
   cudaGetLastError();
 }
+
+namespace {
 
 // Spread the per-record counts of multi-owner pixels over their owner sets (see count_multi_owner).
 __global__ void __launch_bounds__(256) k_multi_expand(const CanvasDev* __restrict__ cvg, const unsigned int* __restrict__ rec_cnt,

@@ -145,6 +145,7 @@ int set_error(int code, const char* fmt, ...);
 int check_cuda(cudaError_t e, const char* what);
 void count_launch(int n = 1);
 int device_sm_count();
+void keep_pool_memory();    // the device's default pool keeps freed memory (probe scratch, build temporaries)
 
 // probe-path options (spade_set_option; include/spade.h)
 struct Options {

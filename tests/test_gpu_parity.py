@@ -349,7 +349,7 @@ def test_build_profile_and_call_stages(spade):
         st2 = spade.last_call_stages()
     finally:
         spade.set_option("stage_events", 0)
-    assert st["probe"] > 0 and st["output compaction"] == 0
+    assert st["probe"] > 0 and st["output compaction"] < 0.05     # COUNT: no compaction (event gap only)
     assert st2["probe"] > 0 and st2["output compaction"] > 0
     c0 = spade.join_count(cv, xy).cpu().numpy()
     assert all(v == 0 for v in spade.last_call_stages().values())
