@@ -26,7 +26,7 @@ def build(force: bool = False) -> str:
     """Compile spade_oracle.c (+ the R-tree CPU baseline, rtree_join.c) into liboracle.so
     (plain gcc, -O2, pthreads)."""
     srcs = [os.path.join(_HERE, "spade_oracle.c"), os.path.join(_HERE, "rtree_join.c"),
-            os.path.join(_HERE, "distance_oracle.c")]
+            os.path.join(_HERE, "distance_oracle.c"), os.path.join(_HERE, "polygon_join_oracle.c")]
     newest = max(os.path.getmtime(x) for x in srcs)
     if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < newest:
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-pthread", "-o", _LIB_PATH, *srcs])
@@ -58,6 +58,12 @@ def _load():
         lib.oracle_disk_join_pairs.restype = i64
         lib.oracle_disk_select.argtypes = [P, i64, i64, P, P, i32, P, i64, ctypes.c_int]
         lib.oracle_disk_select.restype = i64
+        lib.oracle_segments_intersect.argtypes = [i64] * 8
+        lib.oracle_segments_intersect.restype = ctypes.c_int
+        lib.oracle_polygons_intersect.argtypes = [P, P, P, i32, P, P, P, i32]
+        lib.oracle_polygons_intersect.restype = ctypes.c_int
+        lib.oracle_polygon_join.argtypes = [P, P, P, i32, P, P, P, i32, P, P, i64, ctypes.c_int]
+        lib.oracle_polygon_join.restype = i64
         lib.oracle_knn.argtypes = [P, i64, i64, i64, i64, i64, P, P]
         lib.oracle_knn.restype = i64
         _lib = lib
@@ -221,3 +227,38 @@ def knn(xy, q, k: int, point_id_base: int = 0):
     if got < 0:
         raise MemoryError("oracle_knn failed")
     return ids[:got], d2[:got]
+
+
+# ---- polygon x polygon join (polygon_join_oracle.c, reading C15) ----------------
+
+def segments_intersect(a, b, c, d) -> bool:
+    """Closed segments a-b and c-d share a point (textbook SEGMENTS-INTERSECT, exact)."""
+    return bool(_load().oracle_segments_intersect(int(a[0]), int(a[1]), int(b[0]), int(b[1]),
+                                                   int(c[0]), int(c[1]), int(d[0]), int(d[1])))
+
+
+def polygons_intersect(polys1, a: int, polys2, b: int) -> bool:
+    """Closed regions of polygon a of polys1 and polygon b of polys2 intersect (ST_INTERSECTS)."""
+    x1, r1, p1, _ = _polys(polys1)
+    x2, r2, p2, _ = _polys(polys2)
+    return bool(_load().oracle_polygons_intersect(_ptr(x1), _ptr(r1), _ptr(p1), int(a), _ptr(x2), _ptr(r2), _ptr(p2), int(b)))
+
+
+def polygon_join(polys1, polys2, nthreads: int | None = None):
+    """All (a, b) with polygon a of polys1 intersecting polygon b of polys2 (closed regions),
+    sorted by (a, b): two int32 arrays.  Brute force over every polygon pair and edge pair."""
+    lib = _load()
+    x1, r1, p1, n1 = _polys(polys1)
+    x2, r2, p2, n2 = _polys(polys2)
+    nt = nthreads or default_threads()
+    cap = 1024
+    while True:
+        a = np.empty(cap, np.int32)
+        b = np.empty(cap, np.int32)
+        tot = lib.oracle_polygon_join(_ptr(x1), _ptr(r1), _ptr(p1), n1, _ptr(x2), _ptr(r2), _ptr(p2), n2,
+                                      _ptr(a), _ptr(b), cap, nt)
+        if tot < 0:
+            raise MemoryError("oracle_polygon_join")
+        if tot <= cap:
+            return a[:tot], b[:tot]
+        cap = int(tot)

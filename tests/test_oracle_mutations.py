@@ -36,6 +36,20 @@ DIST_MUTANTS = {
                        "for (int64_t i = 0; i < k; ++i) {\n        out_ids[i] = a[i + (i + 1 < n)].id;"),
 }
 
+# polygon x polygon join oracle (oracle/polygon_join_oracle.c) against tests/test_polygon_join_oracle_pins.py
+PJ_MUTANTS = {
+    "collinear_straddle": ("if (d1 * d2 < 0 && d3 * d4 < 0) return 1;", "if (d1 * d2 <= 0 && d3 * d4 <= 0) return 1;"),
+    "no_collinear_touch": ("    return (rx >= (px < qx ? px : qx))", "    return 0 && (rx >= (px < qx ? px : qx))"),
+    "one_sided_containment": ("                                                        ring_vertex_inside(&t->A, a, &t->B, b));",
+                              "                                                        0);"),
+    "first_ring_vertex_only": ("for (int64_t r = Q->pro[q]; r < Q->pro[q + 1]; ++r) {",
+                               "for (int64_t r = Q->pro[q]; r < Q->pro[q] + 1 && r < Q->pro[q + 1]; ++r) {"),
+    "drop_closing_edge": ("        for (int64_t k = A->ro[r]; k < A->ro[r + 1]; ++k) {",
+                          "        for (int64_t k = A->ro[r]; k + 1 < A->ro[r + 1]; ++k) {"),
+    "swapped_orient_operand": ("__int128 v = (__int128)(qx - px) * (ry - py) - (__int128)(qy - py) * (rx - px);",
+                               "__int128 v = (__int128)(qx - px) * (ry - py) - (__int128)(qy - py) * (rx - qx);"),
+}
+
 
 def _run_mutant(tmp_path, name, src_name, old, new, pins):
     for d in ("oracle", "gen", "tests"):
@@ -58,3 +72,8 @@ def test_pins_kill_mutant(name, tmp_path):
 @pytest.mark.parametrize("name", sorted(DIST_MUTANTS))
 def test_distance_pins_kill_mutant(name, tmp_path):
     _run_mutant(tmp_path, name, "distance_oracle.c", *DIST_MUTANTS[name], "tests/test_distance_oracle_pins.py")
+
+
+@pytest.mark.parametrize("name", sorted(PJ_MUTANTS))
+def test_polygon_join_pins_kill_mutant(name, tmp_path):
+    _run_mutant(tmp_path, name, "polygon_join_oracle.c", *PJ_MUTANTS[name], "tests/test_polygon_join_oracle_pins.py")
