@@ -188,6 +188,24 @@ SPADE_API int spade_join_pairs_host(const spade_canvas* c, const int32_t* xy_hos
                                     int32_t* out_poly_ids_host, int64_t capacity, int64_t* n_out,
                                     spade_stream_t stream);
 
+/* Polygon x Polygon join (Sec. 5.2): all pairs (a, b), polygon a of D1 and polygon b of D2,
+ * whose CLOSED regions intersect (ST_INTERSECTS; touching boundaries count; DESIGN.md
+ * reading C15), sorted by (a, b), each pair once.  Both sets use spade_build_canvas's layout
+ * (device arrays; even-odd regions over all rings of a polygon) and must be VALID polygons:
+ * rings of >= 3 vertices, no zero-length edge, no segment used twice by one polygon (rings may
+ * touch at points; different polygons may share edges).  `prm` (may be NULL) sets the resolution
+ * of the common pixel grid both sets are rasterised on (max_dim over the union extent, or
+ * log2_pixel); results do not depend on it.  The join tests the local edge pairs of pixels that
+ * are boundary pixels of both canvases (exact closed-segment test) and probes every ring's first
+ * vertex against the other set's canvas (the point join).
+ *   out_a, out_b [capacity] int32 device (polygon ids in D1, D2);  n_out HOST: number of pairs.
+ * capacity < n_out -> SPADE_ERR_CAPACITY (the first `capacity` pairs in order are written).
+ * Vertices outside [-2^30, 2^30) -> SPADE_ERR_COORD_RANGE.  Synchronises `stream`. */
+SPADE_API int spade_join_polygons(const int32_t* ring_xy1, const int64_t* ring_off1, const int64_t* poly_ring_off1,
+                                  int32_t num_polys1, const int32_t* ring_xy2, const int64_t* ring_off2,
+                                  const int64_t* poly_ring_off2, int32_t num_polys2, const spade_canvas_params* prm,
+                                  int32_t* out_a, int32_t* out_b, int64_t capacity, int64_t* n_out, spade_stream_t stream);
+
 /* ---- kNN selection over points (Sec. 5.2), in the paper's three steps ------------
  * The circles of step 1 are concentric around the query q with squared radii
  *   r2_b = the largest squared distance of bucket b,  b = 0 .. SPADE_KNN_BINS-1, where

@@ -67,6 +67,9 @@ def load(path: str | None = None):
     lib.spade_canvas_free.restype = None
     lib.spade_canvas_info.argtypes = [P] + [ctypes.POINTER(i32)] * 6 + [ctypes.POINTER(i64)] * 2 + [ctypes.POINTER(ctypes.c_double)]
     lib.spade_canvas_info.restype = ctypes.c_int
+    lib.spade_join_polygons.argtypes = [P, P, P, i32, P, P, P, i32, ctypes.POINTER(CanvasParams), P, P, i64,
+                                         ctypes.POINTER(i64), P]
+    lib.spade_join_polygons.restype = ctypes.c_int
     lib.spade_canvas_build_times.argtypes = [P, ctypes.POINTER(ctypes.c_float), i32]
     lib.spade_canvas_build_times.restype = ctypes.c_int
     lib.spade_canvas_build_stage_name.argtypes = [i32]
@@ -110,7 +113,7 @@ def load(path: str | None = None):
 
 
 EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canvas_free", "spade_canvas_info",
-                    "spade_canvas_checksum", "spade_canvas_build_times", "spade_canvas_build_stage_name", "spade_join_count",
+                    "spade_canvas_checksum", "spade_canvas_build_times", "spade_canvas_build_stage_name", "spade_join_polygons", "spade_join_count",
                     "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_select_host", "spade_join_pairs_host", "spade_knn_histogram",
                     "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_set_option", "spade_launch_count", "spade_last_call_stages",
                     "spade_status_string", "spade_last_error"]
@@ -286,6 +289,33 @@ class Canvas:
             self.close()
         except Exception:
             pass
+
+
+def join_polygons(polys1, polys2, capacity: int | None = None, max_dim: int = 4096, log2_pixel: int = -1,
+                  stream=None):
+    """Polygon x Polygon join (spade_join_polygons): (a, b) int32 CUDA tensors of every
+    polygon a of polys1 and b of polys2 whose closed regions intersect, sorted by (a, b)."""
+    torch = _torch()
+    d = []
+    for polys in (polys1, polys2):
+        d.append((_dev(polys["ring_xy"], torch.int32, 2), _dev(polys["ring_off"], torch.int64),
+                  _dev(polys["poly_ring_off"], torch.int64)))
+    n1, n2 = int(d[0][2].numel()) - 1, int(d[1][2].numel()) - 1
+    cap = max(n1 + n2, 1024) if capacity is None else int(capacity)
+    prm = CanvasParams(log2_pixel, max_dim, 0)
+    for _ in range(2):
+        a = torch.empty(max(cap, 1), dtype=torch.int32, device="cuda")
+        b = torch.empty(max(cap, 1), dtype=torch.int32, device="cuda")
+        n_out = ctypes.c_int64()
+        args = [ctypes.c_void_p(t.data_ptr()) for t in d[0]] + [n1] + [ctypes.c_void_p(t.data_ptr()) for t in d[1]] + [n2]
+        rc = load().spade_join_polygons(*args, ctypes.byref(prm), ctypes.c_void_p(a.data_ptr()),
+                                        ctypes.c_void_p(b.data_ptr()), cap, ctypes.byref(n_out), _stream(stream))
+        if rc == SPADE_ERR_CAPACITY:
+            cap = n_out.value
+            continue
+        _check(rc, "spade_join_polygons")
+        return a[: n_out.value], b[: n_out.value]
+    raise SpadeError(SPADE_ERR_CAPACITY, "join_polygons: capacity retry failed")
 
 
 def canvas_checksum(canvas: Canvas, stream=None) -> int:

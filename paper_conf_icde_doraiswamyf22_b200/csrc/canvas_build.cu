@@ -834,9 +834,22 @@ cudaError_t cub_call(DevBufs& bufs, F f) {
 
 // One builder for both canvas kinds: the front end (K-B0/K-B1 for polygon edges, K-D0/K-D1 for
 // disks) produces primitives, boundary fragments and fill events; everything after is shared.
+int tile_log2_for(int64_t W0, int64_t H0, int32_t P) {
+  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (<= 160 KB),
+  // including one sentinel column and row of always-empty tiles (the probe clamps tile
+  // coordinates into them instead of testing the extent); tile side 2^b pixels, s + b <= 30.
+  // The probe's COUNT histogram ((P+1) uint32) shares the ~196 KB budget with the tiles.
+  const int64_t hist1 = ((int64_t)P + 1) * 4, kSoft = 196 * 1024;
+  const int64_t kMaxTiles = hist1 <= kSoft - 8192 ? std::min<int64_t>(81920, std::max<int64_t>(4096, (kSoft - hist1) / 2))
+                                                  : 81920;
+  int b = 0;
+  while ((((W0 + (1 << b) - 1) >> b) + 1) * (((H0 + (1 << b) - 1) >> b) + 1) > kMaxTiles) ++b;
+  return b;
+}
+
 static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off,
                      const int32_t* center_xy, const int64_t* r2, int32_t P, const spade_canvas_params* prm,
-                     cudaStream_t st, spade_canvas** out) {
+                     cudaStream_t st, spade_canvas** out, const GridSpec* grid = nullptr) {
   *out = nullptr;
   const char* fn = kind == kDisks ? "spade_build_disk_canvas" : "spade_build_canvas";
   if (P < 0 || (kind == kPolygons && P > 0 && (!ring_off || !poly_ring_off)) || (kind == kDisks && P > 0 && (!center_xy || !r2)))
@@ -913,8 +926,11 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   if (kind == kDisks && h_bad) return fail(set_error(SPADE_ERR_COORD_RANGE, "a disk reaches outside [-2^30, 2^30)"));
 
   // --- canvas geometry (reading C5) ---
+  if (grid && (h_ext[0] < grid->minx || h_ext[1] < grid->miny || h_ext[2] > grid->maxx || h_ext[3] > grid->maxy))
+    return fail(set_error(SPADE_ERR_INTERNAL, "%s: forced grid does not contain the extent", fn));
+  if (grid) { h_ext[0] = grid->minx; h_ext[1] = grid->miny; h_ext[2] = grid->maxx; h_ext[3] = grid->maxy; }
   int64_t ew = (int64_t)h_ext[2] - h_ext[0], eh = (int64_t)h_ext[3] - h_ext[1];
-  int s = forced_s;
+  int s = grid ? grid->s : forced_s;
   if (s < 0) {
     s = 0;
     while (std::max((ew >> s) + 1, (eh >> s) + 1) > max_dim) ++s;
@@ -923,15 +939,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   Geo g;
   g.minx = h_ext[0]; g.miny = h_ext[1]; g.s = s; g.S = 1ll << s;
   const int64_t W0 = (ew >> s) + 1, H0 = (eh >> s) + 1;
-  // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (<= 160 KB),
-  // including one sentinel column and row of always-empty tiles (the probe clamps tile
-  // coordinates into them instead of testing the extent); tile side 2^b pixels, s + b <= 30.
-  // The probe's COUNT histogram ((P+1) uint32) shares the ~196 KB budget with the tiles.
-  const int64_t hist1 = ((int64_t)P + 1) * 4, kSoft = 196 * 1024;
-  const int64_t kMaxTiles = hist1 <= kSoft - 8192 ? std::min<int64_t>(81920, std::max<int64_t>(4096, (kSoft - hist1) / 2))
-                                                  : 81920;
-  int b = 0;
-  while ((((W0 + (1 << b) - 1) >> b) + 1) * (((H0 + (1 << b) - 1) >> b) + 1) > kMaxTiles) ++b;
+  const int b = grid ? grid->b : tile_log2_for(W0, H0, P);
   if (s + b > 30) return fail(set_error(SPADE_ERR_INVALID_ARG, "canvas tiles too coarse (s=%d, b=%d)", s, b));
   const int Wc = (int)((W0 + (1 << b) - 1) >> b), Hc = (int)((H0 + (1 << b) - 1) >> b);
   // the canvas itself is padded to whole tiles: pixels beyond the extent are ordinary pixels
@@ -1260,6 +1268,12 @@ int canvas_checksum(const spade_canvas* c, uint64_t* out, cudaStream_t st) {
   }
   *out = h;
   return SPADE_OK;
+}
+
+int build_canvas_on_grid(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off, int32_t P,
+                         const GridSpec& grid, cudaStream_t st, spade_canvas** out) {
+  spade_canvas_params prm{grid.s, 0, SPADE_CANVAS_DENSE | SPADE_CANVAS_NO_FINE16};
+  return build_any(kPolygons, ring_xy, ring_off, poly_ring_off, nullptr, nullptr, P, &prm, st, out, &grid);
 }
 
 int build_canvas(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off, int32_t P,

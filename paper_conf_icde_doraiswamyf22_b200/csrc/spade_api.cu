@@ -24,6 +24,8 @@ int build_canvas(const int32_t*, const int64_t*, const int64_t*, int32_t, const 
                  spade_canvas**);
 int build_disk_canvas(const int32_t*, const int64_t*, int32_t, const spade_canvas_params*, cudaStream_t, spade_canvas**);
 int canvas_checksum(const spade_canvas*, uint64_t*, cudaStream_t);
+int join_polygons(const int32_t*, const int64_t*, const int64_t*, int32_t, const int32_t*, const int64_t*, const int64_t*,
+                  int32_t, const spade_canvas_params*, int32_t*, int32_t*, int64_t, int64_t*, cudaStream_t);
 
 namespace {
 thread_local char g_err[512] = "";
@@ -148,6 +150,16 @@ int spade_canvas_info(const spade_canvas* c, int32_t* W, int32_t* H, int32_t* lo
   if (num_run_edges) *num_run_edges = c->num_run_edges;
   if (mixed_tile_frac) *mixed_tile_frac = c->mixed_tile_frac;
   return SPADE_OK;
+}
+
+int spade_join_polygons(const int32_t* ring_xy1, const int64_t* ring_off1, const int64_t* poly_ring_off1, int32_t num_polys1,
+                        const int32_t* ring_xy2, const int64_t* ring_off2, const int64_t* poly_ring_off2, int32_t num_polys2,
+                        const spade_canvas_params* prm, int32_t* out_a, int32_t* out_b, int64_t capacity, int64_t* n_out,
+                        spade_stream_t stream) {
+  if (!n_out) return set_error(SPADE_ERR_INVALID_ARG, "spade_join_polygons: n_out is NULL");
+  NvtxRange nv("spade_join_polygons");
+  return join_polygons(ring_xy1, ring_off1, poly_ring_off1, num_polys1, ring_xy2, ring_off2, poly_ring_off2, num_polys2,
+                       prm, out_a, out_b, capacity, n_out, (cudaStream_t)stream);
 }
 
 int spade_canvas_build_times(const spade_canvas* c, float* ms, int32_t cap) {

@@ -170,6 +170,17 @@ struct DeviceGuard {
 };
 Options& options();
 
+// A forced canvas grid: the polygon x polygon join lays both polygon sets on one pixel grid
+// (the extent must contain the set's own; s = log2 pixel, b = log2 tile).
+struct GridSpec {
+  int32_t minx, miny, maxx, maxy;
+  int32_t s, b;
+};
+int build_canvas_on_grid(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off, int32_t P,
+                         const GridSpec& grid, cudaStream_t st, spade_canvas** out);
+// tile exponent the builder picks for a W0 x H0 pixel canvas over P polygons
+int tile_log2_for(int64_t W0, int64_t H0, int32_t P);
+
 // probe launchers (probe.cu)
 int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* counts, cudaStream_t st);
 int launch_select(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t base, int64_t* out,

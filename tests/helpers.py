@@ -48,3 +48,30 @@ def sorted_pairs(pt, pl):
     pt = np.asarray(pt, np.int64); pl = np.asarray(pl, np.int64)
     o = np.lexsort((pl, pt))
     return pt[o], pl[o]
+
+
+def valid_polyset(rng, n, lo, hi, scale=1):
+    """Valid polygons (simple rings, no zero-length edges): stars, rectangles, rectangles with a
+    rectangular hole, two-component rectangles."""
+    polys = []
+    for _ in range(n):
+        kind = rng.random()
+        cx, cy = rng.integers(lo + 6, hi - 5, 2)
+        if kind < 0.4:
+            r = pg.star(rng, int(rng.integers(3, 9)), cx, cy, rng.integers(3, 8), rng.integers(3, 8), rmin=0.5)
+            r = r[np.any(r != np.roll(r, 1, 0), axis=1)]
+            if len(r) < 3:
+                r = pg.rect(cx - 2, cy - 2, cx + 2, cy + 2)
+            polys.append([r])
+        else:
+            w, h = rng.integers(2, 8, 2)
+            outer = pg.rect(cx - w, cy - h, cx + w, cy + h)
+            if kind < 0.6 and w >= 4 and h >= 4:
+                polys.append([outer, pg.rect(cx - w + 2, cy - h + 2, cx + w - 2, cy + h - 2)])
+            elif kind < 0.8:
+                polys.append([outer, pg.rect(cx + w + 2, cy, cx + w + 4, cy + 3)])
+            else:
+                polys.append([outer])
+    out = pg.assemble(polys)
+    out["ring_xy"] = (np.asarray(out["ring_xy"], np.int64) * scale).astype(np.int32)
+    return out

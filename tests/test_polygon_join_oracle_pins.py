@@ -22,6 +22,7 @@ import pytest
 
 import oracle
 from gen import polygons as pg
+from tests.helpers import valid_polyset as _valid_polyset
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 CASES = json.load(open(os.path.join(ROOT, "tests", "golden", "polygon_join_cases.json")))["cases"]
@@ -74,33 +75,6 @@ def test_grid_vs_shifted_grid_closed_form():
     exp = {(j * k + i, j2 * k + i2) for j in range(m) for i in range(k) for j2 in range(m) for i2 in range(k)
            if i2 in (i - 1, i) and j2 in (j - 1, j)}
     assert set(zip(a.tolist(), b.tolist())) == exp
-
-
-def _valid_polyset(rng, n, lo, hi, scale=1):
-    """Valid polygons (simple rings, no zero-length edges): stars, rectangles, rectangles with a
-    rectangular hole, two-component rectangles."""
-    polys = []
-    for _ in range(n):
-        kind = rng.random()
-        cx, cy = rng.integers(lo + 6, hi - 5, 2)
-        if kind < 0.4:
-            r = pg.star(rng, int(rng.integers(3, 9)), cx, cy, rng.integers(3, 8), rng.integers(3, 8), rmin=0.5)
-            r = r[np.any(r != np.roll(r, 1, 0), axis=1)]
-            if len(r) < 3:
-                r = pg.rect(cx - 2, cy - 2, cx + 2, cy + 2)
-            polys.append([r])
-        else:
-            w, h = rng.integers(2, 8, 2)
-            outer = pg.rect(cx - w, cy - h, cx + w, cy + h)
-            if kind < 0.6 and w >= 4 and h >= 4:
-                polys.append([outer, pg.rect(cx - w + 2, cy - h + 2, cx + w - 2, cy + h - 2)])
-            elif kind < 0.8:
-                polys.append([outer, pg.rect(cx + w + 2, cy, cx + w + 4, cy + 3)])
-            else:
-                polys.append([outer])
-    out = pg.assemble(polys)
-    out["ring_xy"] = (np.asarray(out["ring_xy"], np.int64) * scale).astype(np.int32)
-    return out
 
 
 def _closed_member(xy, polys, p):
