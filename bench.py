@@ -35,10 +35,10 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5", "dj", "dj2", "knn", "ov"],
+    ap.add_argument("--workload", default="c3", choices=["c1", "c2", "c3", "c4", "c5", "dj", "dj2", "knn", "ov", "pp"],
                     help="c3 (default) = the metric's join+COUNT config; c2 select, c4 pairs, c5 40k polygons; "
                          "dj / dj2 distance joins (type 1 pairs / type 2 count), knn kNN selection, "
-                         "ov overlap-heavy polygon set (1,000 overlapping stars)")
+                         "ov overlap-heavy polygon set (1,000 overlapping stars), pp polygon x polygon join")
     ap.add_argument("--points-per-gpu", type=int, default=None, help="default: the config's size (1B; C2 100M)")
     ap.add_argument("--impl", default="spade", choices=["spade", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -68,11 +68,14 @@ METRICS = {
     "dist_pairs": "points/sec for the type 1 distance join emitting (point_id, disk_id) pairs",
     "dist_count": "points/sec for the type 2 distance join COUNT (per-disk counts)",
     "knn": "points/sec scanned by kNN selection (circle aggregation + distance select + sort)",
+    "polyjoin": "polygon pairs/sec decided by the polygon x polygon join (|D1| x |D2| per call)",
 }
 
 
 def workload(name, n_per_gpu):
     from gen import configs
+    if name in configs.POLYJOIN:
+        return configs.POLYJOIN[name]()
     if name in configs.DISTANCE:
         return configs.DISTANCE[name](n_per_gpu or 1_000_000_000)
     if name in ("c1", "c2"):
@@ -269,11 +272,57 @@ def parity_check(w, cv, sp, idx, oracle_counts=None, rate=None, pairs_seconds=5.
     return res
 
 
+def polyjoin_oracle_rate(w, target_s, offset=0):
+    """The polygon x polygon oracle (brute force over every polygon pair and edge pair) on the
+    first k polygons of D1 (rotated by `offset`) x all of D2, k sized to ~target_s."""
+    import oracle
+    n1, n2 = len(w.polys["poly_ring_off"]) - 1, len(w.polys2["poly_ring_off"]) - 1
+
+    def subset(k):
+        import numpy as np
+        pro = np.asarray(w.polys["poly_ring_off"])
+        ro = np.asarray(w.polys["ring_off"])
+        lo = offset % max(1, n1 - k)
+        r0, r1 = pro[lo], pro[lo + k]
+        v0, v1 = ro[r0], ro[r1]
+        return {"ring_xy": np.asarray(w.polys["ring_xy"])[v0:v1], "ring_off": ro[r0:r1 + 1] - v0,
+                "poly_ring_off": pro[lo:lo + k + 1] - r0}, lo
+    sub, _ = subset(4)
+    t0 = time.perf_counter()
+    oracle.polygon_join(sub, w.polys2)
+    dt = max(time.perf_counter() - t0, 1e-3)
+    k = int(max(4, min(n1, 4 * target_s / dt)))
+    sub, lo = subset(k)
+    t0 = time.perf_counter()
+    a, b = oracle.polygon_join(sub, w.polys2)
+    dt = time.perf_counter() - t0
+    return {"value": k * n2 / dt, "unit": "polygon pairs/s", "cores": oracle.default_threads(), "kind": "oracle",
+            "sample": f"D1 polygons [{lo}, {lo + k}) x all {n2} of D2, brute force over every polygon and edge pair "
+                      f"({dt:.1f} s)", "seconds": dt, "subset": sub, "lo": lo, "pairs": (a + lo, b)}
+
+
 def run_reference(a):
     ws, rank, _ = dist_env()
     if rank != 0:
         return
     w = workload(a.workload, a.points_per_gpu)
+    if w.op == "polyjoin":
+        per_step = max(1.0, 120.0 / max(1, a.steps + a.warmup))
+        rates, secs, res = [], 0.0, None
+        for k in range(a.steps):
+            res = polyjoin_oracle_rate(w, per_step, offset=97 * k)
+            rates.append(res["value"])
+            secs += res["seconds"]
+        value = statistics.median(rates)
+        print(json.dumps({"impl": "reference", "metric": METRICS["polyjoin"], "value": value, "unit": "polygon pairs/s",
+                          "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * secs / max(1, a.steps),
+                          "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+                          "data": "synthetic", "config": {"workload": w.name, "desc": w.desc},
+                          "cpu_baseline": {"value": value, "unit": "polygon pairs/s", "cores": res["cores"], "kind": "oracle",
+                                           "sample": res["sample"]},
+                          "e2e": {"value": value, "unit": "polygon pairs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}),
+              flush=True)
+        return
     per_step = max(1.0, 120.0 / max(1, a.steps + a.warmup))
     res = None
     for _ in range(a.warmup):
@@ -300,6 +349,96 @@ def run_reference(a):
     print(json.dumps(line), flush=True)
 
 
+def run_polyjoin(a, w, sp, ws, rank, local):
+    """Polygon x polygon join (spade_join_polygons): one step = one whole join call (both canvases
+    built on a common grid, contact tests, ring-vertex probes, sort + unique) over device-resident
+    polygon arrays; e2e = the same call from host (numpy) arrays, H2D inside the timing."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    dev = torch.device("cuda", local)
+    n1, n2 = len(w.polys["poly_ring_off"]) - 1, len(w.polys2["poly_ring_off"]) - 1
+    dA = {k: torch.as_tensor(np.ascontiguousarray(v)).to(dev) for k, v in w.polys.items()}
+    dB = {k: torch.as_tensor(np.ascontiguousarray(v)).to(dev) for k, v in w.polys2.items()}
+    stream = torch.cuda.current_stream()
+    res = [None]
+
+    def step():
+        res[0] = sp.join_polygons(dA, dB, max_dim=w.max_dim)
+    for _ in range(max(3, a.warmup)):
+        step()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    if not a.profile:
+        sampler.start()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    l0 = sp.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(a.steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    l1 = sp.launch_count()
+    clocks = sampler.stop() if not a.profile else None
+    t_ms = e0.elapsed_time(e1)
+    if ws > 1:
+        tt = torch.tensor([t_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_ms = tt.item()
+    ga, gb = (x.cpu().numpy().astype(np.int64) for x in res[0])
+    value = ws * n1 * n2 * a.steps / (t_ms / 1e3)
+    line = None
+    if rank == 0:
+        V = int(len(w.polys["ring_xy"]) + len(w.polys2["ring_xy"]))
+        ms = t_ms / a.steps
+        line = {"metric": METRICS["polyjoin"], "value": value, "unit": "polygon pairs/s", "n_gpus": ws, "steps": a.steps,
+                "warmup": max(3, a.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+                "config": {"workload": w.name, "desc": w.desc, "polygons": [n1, n2], "vertices": V, "max_dim": w.max_dim,
+                           "parallelism": f"dp{ws} (replicated join per rank)",
+                           "l2": "one whole join per step (two canvas builds, contact tests, probes, sort)"},
+                "roofline": {"bound": "latency", "achieved": 16.0 * V / (ms / 1e3) / 1e9, "peak": measured_peak()[0],
+                             "unit": "GB/s", "frac": 16.0 * V / (ms / 1e3) / 1e9 / measured_peak()[0], "traffic": None,
+                             "kernel": "spade_join_polygons (whole call: builds + k_pp_contacts + probes + sort)",
+                             "note": "algorithmic bytes = 16 B per input vertex (read by each of the two builds); "
+                                     "the call is a chain of small kernels and host syncs: latency-bound"},
+                "gpu_launches": int(l1 - l0), "check": {"pairs": int(len(ga))}}
+        if clocks:
+            line["clocks"] = clocks
+        if not a.no_e2e and not a.profile:
+            times = []
+            for _ in range(a.e2e_steps):
+                torch.cuda.synchronize()
+                s0 = time.perf_counter()
+                r = sp.join_polygons(w.polys, w.polys2, max_dim=w.max_dim)
+                r[0].cpu()
+                times.append(time.perf_counter() - s0)
+            line["e2e"] = {"value": n1 * n2 / statistics.median(times), "unit": "polygon pairs/s",
+                           "h2d_bytes_per_step": int(sum(np.asarray(v).nbytes for d in (w.polys, w.polys2) for v in d.values())),
+                           "d2h_bytes_per_step": int(8 * len(ga)), "api": "join_polygons from host numpy arrays",
+                           "timing": "host wall clock around the call"}
+        if not a.no_cpu_baseline and not a.profile and ws == 1:
+            cb = polyjoin_oracle_rate(w, a.cpu_seconds)
+            sub, lo, (oa, ob) = cb.pop("subset"), cb.pop("lo"), cb.pop("pairs")
+            cb.pop("seconds")
+            line["cpu_baseline"] = cb
+            if not a.no_parity:
+                sa, sb = (x.cpu().numpy().astype(np.int64) for x in sp.join_polygons(sub, w.polys2, max_dim=w.max_dim))
+                m = (ga >= lo) & (ga < lo + len(sub["poly_ring_off"]) - 1)
+                line["parity"] = {"sample": f"D1 polygons [{lo}, {lo + len(sub['poly_ring_off']) - 1}) x all of D2",
+                                  "checked": "sorted (a, b) pairs of the sample: oracle vs GPU on the sample, and vs "
+                                             "the full GPU join restricted to the sample",
+                                  "pairs": int(len(oa)),
+                                  "ok": bool(np.array_equal(sa + lo, oa) and np.array_equal(sb, ob) and
+                                             np.array_equal(ga[m], oa) and np.array_equal(gb[m], ob))}
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
 def main():
     a = parse()
     if a.impl == "reference":
@@ -322,6 +461,8 @@ def main():
         k, v = o.split("=")
         sp.set_option(k, int(v))
     w = workload(a.workload, a.points_per_gpu)
+    if w.op == "polyjoin":
+        return run_polyjoin(a, w, sp, ws, rank, local)
     n = w.n_points
     is_dist = hasattr(w, "disks")
     P = len(w.disks["r2"]) if is_dist else len(w.polys["poly_ring_off"]) - 1

@@ -176,3 +176,27 @@ def ov(n_points: int = 1_000_000_000, n_polys: int = 1000) -> Workload:
 ALL = {"c1": c1, "c2": c2, "c3": c3, "c4": c4, "c5": c5}
 OVERLAP = {"ov": ov}
 DISTANCE = {"dj": dj, "dj2": dj2, "knn": knn}
+
+
+# ---- polygon x polygon join ----------------------------
+@dataclass
+class PolyJoinWorkload:
+    name: str
+    op: str                    # "polyjoin"
+    polys: dict = field(repr=False)     # D1
+    polys2: dict = field(repr=False)    # D2
+    max_dim: int = 8192
+    desc: str = ""
+    n_points: int = 0          # (no point stream)
+
+
+def pp() -> PolyJoinWorkload:
+    """Census-tract-like tiling (C4's 2,200 polygons with island holes) joined with the
+    neighbourhood-like tiling (C3's 260 polygons): which tracts meet which neighbourhoods
+    (the Polygon x Polygon join of P:202 on Table 1-like data)."""
+    return PolyJoinWorkload("pp_census2200_x_neighborhoods260", "polyjoin", c4(1).polys, c3(1).polys, max_dim=8192,
+                            desc="polygon x polygon join: 2,200 census-tract-like polygons (holes) x 260 "
+                                 "neighbourhood-like polygons, closed-region ST_INTERSECTS")
+
+
+POLYJOIN = {"pp": pp}

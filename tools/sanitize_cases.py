@@ -97,6 +97,15 @@ def main():
     n_checks += 1
     cv = sp.Canvas(configs.c1().polys, max_dim=1024)
     sp.canvas_checksum(cv)
+    # polygon x polygon join
+    from tests.helpers import valid_polyset
+    rng = np.random.default_rng(3)
+    A, B = valid_polyset(rng, 12, 0, 60, scale=16), valid_polyset(rng, 9, 0, 60, scale=16)
+    for s_ in (-1, 4):
+        a, b = sp.join_polygons(A, B, log2_pixel=s_)
+        oa, ob = oracle.polygon_join(A, B)
+        assert np.array_equal(a.cpu().numpy(), oa) and np.array_equal(b.cpu().numpy(), ob)
+        n_checks += 1
     torch.cuda.synchronize()
     print(f"sanitize cases: {n_checks} checks ok, {sp.launch_count()} kernel launches", flush=True)
 
