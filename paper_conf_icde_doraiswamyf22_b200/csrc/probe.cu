@@ -142,14 +142,23 @@ struct Out {
   int64_t ovf_cap;
   longlong2* holes;           // [grid * kNW] (start, length) of each warp's unused chunk tail
   uint32_t chunk;             // slots per warp chunk
+  int32_t policy;             // output stores: 0 streaming (evict-first), 1 default write-back, 2 L2 evict_last
 };
 
 template <int MODE>
 __device__ __forceinline__ void put_result(const Out& o, int64_t pos, int64_t id, int poly) {
   if (pos < o.cap) {
-    // streaming stores (evict-first): the output must not push the canvas out of L2
-    __stcs((long long*)o.out_ids + pos, (long long)id);
-    if (MODE == kPairs) __stcs(o.out_poly + pos, poly);
+    // streaming stores (evict-first) by default: the output must not push the canvas out of L2
+    if (o.policy == 0) {
+      __stcs((long long*)o.out_ids + pos, (long long)id);
+      if (MODE == kPairs) __stcs(o.out_poly + pos, poly);
+    } else if (o.policy == 1) {
+      o.out_ids[pos] = id;
+      if (MODE == kPairs) o.out_poly[pos] = poly;
+    } else {
+      asm volatile("st.global.L2::evict_last.b64 [%0], %1;" ::"l"(o.out_ids + pos), "l"(id) : "memory");
+      if (MODE == kPairs) asm volatile("st.global.L2::evict_last.b32 [%0], %1;" ::"l"(o.out_poly + pos), "r"(poly) : "memory");
+    }
   } else if (pos - o.cap < o.ovf_cap) {
     o.ovf_ids[pos - o.cap] = id;
     if (MODE == kPairs) o.ovf_poly[pos - o.cap] = poly;
@@ -1665,6 +1674,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     FixMeta* fix_meta = (FixMeta*)(scratch + offs[8] + 8 * (size_t)(kMaxHoles + 1));
     if (kOut) {
       p.o.chunk = K;
+      p.o.policy = options().store_policy;
       p.o.ovf_ids = (int64_t*)(scratch + offs[2]);
       p.o.ovf_poly = MODE == kPairs ? (int32_t*)(scratch + offs[3]) : nullptr;
       p.o.ovf_cap = ovf;
