@@ -156,8 +156,10 @@ __device__ __forceinline__ void put_result(const Out& o, int64_t pos, int64_t id
       o.out_ids[pos] = id;
       if (MODE == kPairs) o.out_poly[pos] = poly;
     } else {
-      asm volatile("st.global.L2::evict_last.b64 [%0], %1;" ::"l"(o.out_ids + pos), "l"(id) : "memory");
-      if (MODE == kPairs) asm volatile("st.global.L2::evict_last.b32 [%0], %1;" ::"l"(o.out_poly + pos), "r"(poly) : "memory");
+      uint64_t pol;
+      asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+      asm volatile("st.global.L2::cache_hint.b64 [%0], %1, %2;" ::"l"(o.out_ids + pos), "l"(id), "l"(pol) : "memory");
+      if (MODE == kPairs) asm volatile("st.global.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(o.out_poly + pos), "r"(poly), "l"(pol) : "memory");
     }
   } else if (pos - o.cap < o.ovf_cap) {
     o.ovf_ids[pos - o.cap] = id;
