@@ -48,6 +48,7 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU oracle sample time")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu/clocks)")
     ap.add_argument("--dense", action="store_true", help="force the dense fine-canvas layout (A/B runs)")
+    ap.add_argument("--count", action="store_true", help="run COUNT on the workload's canvas and points (A/B of the sinks)")
     ap.add_argument("--max-dim", type=int, default=None, help="override the workload's canvas max_dim")
     ap.add_argument("--opt", action="append", default=[], metavar="NAME=VALUE",
                     help="spade_set_option before the run (A/B of probe paths; results never depend on it)")
@@ -463,6 +464,8 @@ def main():
     w = workload(a.workload, a.points_per_gpu)
     if w.op == "polyjoin":
         return run_polyjoin(a, w, sp, ws, rank, local)
+    if a.count and w.op in ("select", "pairs"):
+        w.op = "count"
     n = w.n_points
     is_dist = hasattr(w, "disks")
     P = len(w.disks["r2"]) if is_dist else len(w.polys["poly_ring_off"]) - 1
