@@ -19,7 +19,11 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__issue_active.avg.pct_of_peak_sustained_active", "smsp__thread_inst_executed_per_inst_executed.ratio",
         "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum",
         "lts__t_sectors_srcunit_tex_op_read.sum", "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum",
-        "sm__cycles_elapsed.avg.per_second", "launch__grid_size", "launch__block_size"]
+        "sm__cycles_elapsed.avg.per_second", "launch__grid_size", "launch__block_size",
+        "l1tex__t_sector_hit_rate.pct", "lts__t_sectors_srcunit_tex_op_read_lookup_miss.sum",
+        "smsp__sass_inst_executed_op_shared_ld.sum", "smsp__sass_inst_executed_op_shared_atom.sum",
+        "smsp__sass_inst_executed_op_global_ld.sum", "smsp__sass_inst_executed_op_global_st.sum",
+        "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active", "smsp__inst_executed_op_branch.sum"]
 
 
 def ncu(rep, *args):
@@ -31,6 +35,14 @@ def raw(rep):
     h, u, v = rows[0], rows[1], rows[2]
     out = {}
     for i, n in enumerate(h):
+        if n.startswith("smsp__pcsamp_warps_issue_stalled_") and not n.endswith("_not_issued"):
+            try:
+                val = float(v[i].replace(",", ""))
+            except ValueError:
+                continue
+            if val > 0:
+                out.setdefault("stall_samples_by_reason", {})[n.replace("smsp__pcsamp_warps_issue_stalled_", "")] = val
+            continue
         if n in KEYS:
             try:
                 out[n] = {"value": float(v[i].replace(",", "")), "unit": u[i]}
