@@ -283,8 +283,6 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  (256 .. 2^28)
  *   "fine16"       1 (default) / 0: probe canvases that have a 16-bit second level
  *                  (SPADE_CANVAS_NO_FINE16 not set) through it, or through the int32 level
- *   "store_policy" 0 (default): SELECT / PAIRS output stores streaming (evict-first); 1 default
- *                  write-back; 2 L2::evict_last
  *   "stage_events" 0 (default) / 1: record CUDA events between the stages of every COUNT / SELECT /
  *                  PAIRS call on its stream (synchronises once per sub-launch to read them; see
  *                  spade_last_call_stages)
