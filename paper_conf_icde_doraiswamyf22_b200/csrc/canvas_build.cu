@@ -650,6 +650,31 @@ __global__ void k_kset_rng(int64_t NB, const int32_t* __restrict__ ksize, const 
 
 // final encoding: boundary pixel -> -2 - (its record's header offset in the blob); multi-owner
 // corner (owner set g) -> -2 - (record NB + g's header offset)
+// per boundary record: which of its local polygons belong to its corner set K (the K-aggregated
+// COUNT's sign of a polygon of odd edge parity, without searching K per point)
+__global__ void k_kbits(int64_t NR, int64_t NB, const RunRec* __restrict__ runs, const int32_t* __restrict__ rec_polys,
+                        const int32_t* __restrict__ sets, const int2* __restrict__ set_rng, uint64_t* __restrict__ kbits) {
+  for (int64_t r = blockIdx.x * (int64_t)kBT + threadIdx.x; r < NR; r += (int64_t)gridDim.x * kBT) {
+    uint64_t m = 0;
+    if (r < NB) {
+      const RunRec x = runs[r];
+      if (x.poly_cnt <= kMaskPolys && x.term != kEmpty) {
+        int tb = 0, tn = 1;
+        if (x.term < -1) { const int2 g = set_rng[-2 - x.term]; tb = g.x; tn = g.y; }
+        for (int k = 0; k < x.poly_cnt; ++k) {
+          const int32_t P = rec_polys[x.poly_begin + k];
+          bool in = false;
+          if (x.term >= 0) in = P == x.term;
+          else { int lo = 0, hi = tn; while (lo < hi) { const int mid = (lo + hi) >> 1; if (sets[tb + mid] < P) lo = mid + 1; else hi = mid; }
+                 in = lo < tn && sets[tb + lo] == P; }
+          if (in) m |= 1ull << k;
+        }
+      }
+    }
+    kbits[r] = m;
+  }
+}
+
 __global__ void k_finalize(int64_t WH, const int32_t* __restrict__ bflag, const int32_t* __restrict__ bscan,
                            const int32_t* __restrict__ corner, int64_t NB, const int64_t* __restrict__ boff,
                            int32_t* __restrict__ fine) {
@@ -1152,6 +1177,8 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   c->multi_unit = multi_unit;
   TRYF(cudaMemsetAsync(c->blob, 0, 16 * std::max<int64_t>(units, 1), st), "memset blob");   // padding bytes defined
   LAUNCH(k_blob_pack, NR, NR, NB, runs, pix_of, g, run_seg, run_mask, rec_polys, boff, bflags, c->recs, c->blob);
+  if (cudaMalloc(&c->kbits, sizeof(uint64_t) * std::max<int64_t>(NR, 1)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: K bits"));
+  LAUNCH(k_kbits, NR, NR, NB, runs, rec_polys, c->sets, c->set_rng, c->kbits);
   LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, boff, c->fine);
 
   // --- K-B5 coarse tiles (+ compact fine layout) ---
@@ -1207,7 +1234,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   d.mix_min = compact ? kTileMixedCompact : kTileMixed;
   d.cfine = c->cfine;
   d.fine = c->fine; d.fine16 = c->fine16; d.f16 = f16 ? 1 : 0; d.coarse = c->coarse; d.recs = c->recs; d.blob = c->blob;
-  d.sets = c->sets; d.set_rng = c->set_rng;
+  d.sets = c->sets; d.set_rng = c->set_rng; d.kbits = c->kbits;
   if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
   if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));
   *out = c;
@@ -1249,7 +1276,8 @@ int canvas_checksum(const spade_canvas* c, uint64_t* out, cudaStream_t st) {
     const A arrs[] = {{c->fine, (int64_t)d.W * d.H}, {c->fine16, c->fine16 ? ((int64_t)d.W * d.H + 1) / 2 : 0},
                       {c->cfine, c->cfine_elems}, {c->coarse, (c->coarse_elems + 1) / 2},
                       {c->recs, c->num_records * (int64_t)(sizeof(Rec) / 4)}, {c->blob, c->blob_bytes / 4},
-                      {c->sets, c->num_set_entries}, {c->set_rng, 2 * c->num_set_ranges}};
+                      {c->sets, c->num_set_entries}, {c->set_rng, 2 * c->num_set_ranges},
+                      {c->kbits, 2 * c->num_records}};
     uint64_t salt = 1;
     for (const A& a : arrs) {
       if (e == cudaSuccess && a.p && a.words > 0) {

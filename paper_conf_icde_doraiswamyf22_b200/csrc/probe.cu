@@ -365,8 +365,10 @@ struct DeltaFin {
   const int32_t* sets;
   int32_t term;
   int tb, tn;
+  uint64_t kb;                                   // bit k: the record's k-th polygon is in K (<= 64 polygons)
   Emit& emit;
-  __device__ __forceinline__ DeltaFin(const CanvasDev* __restrict__ cv, int32_t t, Emit& e) : sets(cv->sets), term(t), tb(0), tn(0), emit(e) {
+  __device__ __forceinline__ DeltaFin(const CanvasDev* __restrict__ cv, int32_t t, uint64_t kbits, Emit& e)
+      : sets(cv->sets), term(t), tb(0), tn(0), kb(kbits), emit(e) {
     if (t < -1) { const int2 g = cv->set_rng[-2 - t]; tb = g.x; tn = g.y; }
   }
   __device__ __forceinline__ bool inK(int P) const {
@@ -377,14 +379,14 @@ struct DeltaFin {
   }
   __device__ __forceinline__ void operator()(int P, int par) { if (par) emit(P, inK(P) ? -1 : 1); }
   __device__ __forceinline__ void mask(uint64_t m, const int32_t* __restrict__ rp) {
-    while (m) { const int k = __ffsll((long long)m) - 1; m &= m - 1; (*this)(__ldg(rp + k), 1); }
+    while (m) { const int k = __ffsll((long long)m) - 1; m &= m - 1; emit(__ldg(rp + k), ((kb >> k) & 1) ? -1 : 1); }
   }
 };
 template <int KIND, int U = 1, class Emit>
 __device__ __forceinline__ void pip_count_delta(const CanvasDev* __restrict__ cv, int px, int py, uint32_t rec, const Rec r,
                                                 unsigned int* __restrict__ kcnt, Emit&& emit) {
   if (r.term != kEmpty) atomicAdd(kcnt + rec, 1u);
-  DeltaFin<Emit> fin(cv, r.term, emit);
+  DeltaFin<Emit> fin(cv, r.term, __ldg(cv->kbits + rec), emit);
   pip_edges_rec<KIND, U>(cv, px, py, r, fin);
 }
 

@@ -133,7 +133,7 @@ void spade_canvas_free(spade_canvas* c) {
   DeviceGuard dg(c->device);
   cudaDeviceSynchronize();
   cudaFree(c->fine); cudaFree(c->fine16); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->recs); cudaFree(c->blob);
-  cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->d_dev);
+  cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->kbits); cudaFree(c->d_dev);
   delete c;
 }
 

@@ -90,6 +90,7 @@ struct CanvasDev {            // passed by value to kernels
   const uint4* blob;          // packed record data (Rec::blob)
   const int32_t* sets;        // concatenated sorted owner sets
   const int2* set_rng;        // (begin, count)
+  const uint64_t* kbits;      // per record id: bit k = the record's k-th polygon is in its corner set K (<= 64 polygons)
   int32_t kind;               // kPolygons / kDisks
 };
 
@@ -115,6 +116,7 @@ struct spade_canvas {
   int64_t blob_bytes = 0;
   int32_t* sets = nullptr;
   int2* set_rng = nullptr;
+  uint64_t* kbits = nullptr;
   spade::CanvasDev* d_dev = nullptr;   // copy of d in device memory (out-of-line exact test)
 };
 
