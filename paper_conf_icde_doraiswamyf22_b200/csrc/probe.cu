@@ -1500,18 +1500,35 @@ void keep_pool_memory() {
 namespace {
 
 // Spread the per-record counts of multi-owner pixels over their owner sets (see count_multi_owner).
+// hist != 0: per-block shared-memory bins of all P polygons (P <= 12K), flushed with one global
+// atomic per nonzero bin (an owner-set entry is one shared-memory atomic, not one global one).
 __global__ void __launch_bounds__(256) k_multi_expand(const CanvasDev* __restrict__ cvg, const unsigned int* __restrict__ rec_cnt,
-                                                     uint32_t multi_base, uint32_t num_multi, unsigned long long* counts) {
+                                                     uint32_t multi_base, uint32_t num_multi, unsigned long long* counts,
+                                                     int hist) {
+  extern __shared__ unsigned long long eh[];
+  const int P = cvg->num_polys;
+  if (hist) {
+    for (int i = threadIdx.x; i < P; i += 256) eh[i] = 0ull;
+    __syncthreads();
+  }
   for (uint32_t i = blockIdx.x * 256 + threadIdx.x; i < num_multi; i += gridDim.x * 256) {
     const unsigned int k = rec_cnt[i];
     if (k == 0u) continue;
     const int32_t term = cvg->recs[multi_base + i].term;
     if (term >= 0) {
-      atomicAdd(counts + term, (unsigned long long)k);
+      if (hist) atomicAdd(&eh[term], (unsigned long long)k); else atomicAdd(counts + term, (unsigned long long)k);
     } else if (term != kEmpty) {
       const int2 g = cvg->set_rng[-2 - term];
-      for (int j = 0; j < g.y; ++j) atomicAdd(counts + cvg->sets[g.x + j], (unsigned long long)k);
+      for (int j = 0; j < g.y; ++j) {
+        const int q = cvg->sets[g.x + j];
+        if (hist) atomicAdd(&eh[q], (unsigned long long)k); else atomicAdd(counts + q, (unsigned long long)k);
+      }
     }
+  }
+  if (hist) {
+    __syncthreads();
+    for (int i = threadIdx.x; i < P; i += 256)
+      if (eh[i]) atomicAdd(counts + i, eh[i]);
   }
 }
 
@@ -1590,10 +1607,12 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
   }
   // The per-record counters are uint32: they are spread over the owner sets (and cleared) after
   // every sub-launch, each of which holds < 2^31 points, so no counter can wrap whatever n is.
+  if (kcnt || rec_cnt) cudaFuncSetAttribute(k_multi_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 12288);
   auto expand = [&](bool clear) -> int {
     if (kcnt) {
       const int g = (int)std::min<int64_t>((int64_t)sms * 8, (c->num_records + 255) / 256);
-      k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, kcnt, 0u, (uint32_t)c->num_records, base.o.counts);
+      const int eh = c->d.num_polys <= 12288;
+      k_multi_expand<<<g, 256, eh ? 8 * c->d.num_polys : 0, st>>>(c->d_dev, kcnt, 0u, (uint32_t)c->num_records, base.o.counts, eh);
       count_launch();
       cudaError_t e2 = cudaGetLastError();
       if (e2 == cudaSuccess && clear) e2 = cudaMemsetAsync(kcnt, 0, sizeof(unsigned int) * c->num_records, st);
@@ -1601,7 +1620,8 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     }
     if (rec_cnt) {
       const int g = (int)std::min<int64_t>((int64_t)sms * 8, ((int64_t)num_multi + 255) / 256);
-      k_multi_expand<<<g, 256, 0, st>>>(c->d_dev, rec_cnt, (uint32_t)c->num_runs, num_multi, base.o.counts);
+      const int eh = c->d.num_polys <= 12288;
+      k_multi_expand<<<g, 256, eh ? 8 * c->d.num_polys : 0, st>>>(c->d_dev, rec_cnt, (uint32_t)c->num_runs, num_multi, base.o.counts, eh);
       count_launch();
       cudaError_t e2 = cudaGetLastError();
       if (e2 == cudaSuccess && clear) e2 = cudaMemsetAsync(rec_cnt, 0, sizeof(unsigned int) * num_multi, st);
