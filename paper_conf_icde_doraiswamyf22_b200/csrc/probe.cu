@@ -517,61 +517,25 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
 
 // COUNT, in-loop variant: evaluate up to 32 queued boundary points (one per lane).  Out of line:
 // the streaming loop keeps a small register footprint.
-// COUNT, in-loop variant: evaluate up to 32 queued boundary points (one per lane).  Out of line:
-// the streaming loop keeps a small register footprint.  Records with more than kCoopEdges
-// primitives (overlapping polygon sets: tens of edges of piled-up polygons in one pixel) are
-// evaluated by the whole warp in turn -- lanes split the primitives (coalesced loads, one round
-// trip instead of one per primitive) and XOR-reduce the parity masks; the other points keep one
-// lane each.  Must be called by all 32 lanes.
-#ifndef SPADE_COOP_EDGES
-#define SPADE_COOP_EDGES 8
-#endif
-constexpr int kCoopEdges = SPADE_COOP_EDGES;
 template <int MODE, int KIND>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const QEntry* wq,
                                    int cnt, int lane, unsigned int* hist, uint32_t hstride, unsigned long long* counts,
                                    unsigned int* kcnt) {
-  QEntry e{0, 0};
-  Rec r{0u, kEmpty, 0, 0u};
-  uint32_t rid = 0;
-  const bool act = lane < cnt;
-  if (act) {
-    e = wq[lane];
+  if (lane < cnt) {
+    const QEntry e = wq[lane];
     const CanvasDev& cv = *cvg;
     const uint32_t fx = ((uint32_t)e.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)e.y - (uint32_t)cv.miny) >> cv.s;
     const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
     const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
-    r = load_rec(cvg, ~c, &rid);
-  }
-  auto delta = [&](int q, int d) {
-    if (MODE == kCountSmem) atomicAdd(&hist[(uint32_t)q * hstride], (unsigned int)d);
-    else atomicAdd(counts + q, (unsigned long long)(long long)d);
-  };
-  auto hit = [&](int q) { count_hit<MODE>(hist, hstride, counts, q); };
-  const bool coop = act && r.ecnt > kCoopEdges && (r.pinfo & kRecPcnt) <= (uint32_t)kMaskPolys;
-  if (act && !coop) {
-    if (kcnt) pip_count_delta<KIND>(cvg, e.x, e.y, rid, r, kcnt, delta);
-    else pip_eval_rec<KIND>(cvg, e.x, e.y, r, hit);
-  }
-  for (unsigned lm = __ballot_sync(0xffffffffu, coop); lm; lm &= lm - 1) {
-    const int src = __ffs(lm) - 1;
-    const int px = __shfl_sync(0xffffffffu, e.x, src), py = __shfl_sync(0xffffffffu, e.y, src);
-    const Rec rs{__shfl_sync(0xffffffffu, r.blob, src), __shfl_sync(0xffffffffu, r.term, src),
-                 __shfl_sync(0xffffffffu, r.ecnt, src), __shfl_sync(0xffffffffu, r.pinfo, src)};
-    bool big;
-    const uint64_t m = group_mask<KIND, 32>(cvg, true, px, py, rs, lane, big);
-    if (lane == src) {
-      const int32_t* rp = (const int32_t*)(cvg->blob + rs.blob);
-      if (kcnt) {
-        if (rs.term != kEmpty) atomicAdd(kcnt + rid, 1u);
-        DeltaFin<decltype(delta)> fin(cvg, rs.term, __ldg(cvg->kbits + rid), delta);
-        fin.mask(m, rp);
-      } else {
-        TermMerge<decltype(hit)> fin(cvg, rs.term, hit);
-        fin.mask(m, rp);
-        fin.rest();
-      }
-    }
+    uint32_t rid = 0;
+    const Rec r = load_rec(cvg, ~c, &rid);
+    if (kcnt)
+      pip_count_delta<KIND>(cvg, e.x, e.y, rid, r, kcnt, [&](int q, int d) {
+        if (MODE == kCountSmem) atomicAdd(&hist[(uint32_t)q * hstride], (unsigned int)d);
+        else atomicAdd(counts + q, (unsigned long long)(long long)d);
+      });
+    else
+      pip_eval_rec<KIND>(cvg, e.x, e.y, r, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
   }
 }
 
