@@ -580,6 +580,23 @@ def main():
 
     kavg = statistics.mean(kern_ms)
     peak, peak_src = measured_peak()
+    # a same-run streaming-READ reference over the same 8 B/point buffer (the copy peak of
+    # MEASURED_PEAKS.json counts read + write bytes; a read-only stream can exceed it): the best
+    # of 5 float32 sums over the points buffer (a lower bound of the read peak; the round-1
+    # microbenchmark tools/microbench/probe_mb.cu read 7,100 GB/s on this pool)
+    read_gbs = None
+    if op in ("count", "select", "pairs", "knn"):
+        rv = xy.view(torch.float32)
+        best = None
+        for _ in range(5):
+            r0, r1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            r0.record(stream)
+            rv.sum()
+            r1.record(stream)
+            torch.cuda.synchronize()
+            t = r0.elapsed_time(r1)
+            best = t if best is None else min(best, t)
+        read_gbs = rv.numel() * 4 / (best / 1e3) / 1e9
     # algorithmic bytes per launch: the int2 stream, plus the results written (select: 8 B id per
     # selected point; pairs: 8 B id + 4 B polygon id per pair); counts are 8*P bytes, negligible
     # kNN: two passes over the points (circle aggregation, distance selection)
@@ -606,6 +623,9 @@ def main():
             },
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
+                         "frac_of_read_peak": achieved / max(7100.0, read_gbs or 0.0),
+                         "read_peak": {"same_run_torch_sum_gbs": read_gbs, "microbenchmark_gbs": 7100.0,
+                                       "note": "frac_of_read_peak divides by the larger of the two"},
                          "kernel": {"knn": "k_knn_hist + k_knn_select + top-k sort (spade_knn; includes its host syncs)",
                                     "count": "k_probe<COUNT> (spade_join_count)",
                                     "select": "k_probe<SELECT> (spade_select; includes its n_out readback)",

@@ -857,7 +857,8 @@ cudaError_t cub_call(DevBufs& bufs, F f) {
 
 }  // namespace
 
-// One builder for both canvas kinds: the front end (K-B0/K-B1 for polygon edges, K-D0/K-D1 for
+// One builder for both canvas kinds (canvas arrays come from the device's stream-ordered pool,
+// so repeated builds -- e.g. the polygon join's two canvases per call -- reuse memory): the front end (K-B0/K-B1 for polygon edges, K-D0/K-D1 for
 // disks) produces primitives, boundary fragments and fill events; everything after is shared.
 int tile_log2_for(int64_t W0, int64_t H0, int32_t P) {
   // coarse tiles: the shared-memory level holds at most kMaxTiles uint16 entries (<= 160 KB),
@@ -1139,9 +1140,9 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
     NK = last_idx + (last_sz >= 2 ? 1 : 0);
   }
   // final set storage: [corner owner sets (M entries, NG ranges)] ++ [K sets with |K| >= 2]
-  if (cudaMalloc(&c->sets, sizeof(int32_t) * std::max<int64_t>(M + KT, 1)) != cudaSuccess ||
-      cudaMalloc(&c->set_rng, sizeof(int2) * std::max<int64_t>(NG + NK, 1)) != cudaSuccess ||
-      cudaMalloc(&c->fine, sizeof(int32_t) * WH) != cudaSuccess)
+  if (cudaMallocAsync((void**)&c->sets, sizeof(int32_t) * std::max<int64_t>(M + KT, 1), st) != cudaSuccess ||
+      cudaMallocAsync((void**)&c->set_rng, sizeof(int2) * std::max<int64_t>(NG + NK, 1), st) != cudaSuccess ||
+      cudaMallocAsync((void**)&c->fine, sizeof(int32_t) * WH, st) != cudaSuccess)
     return fail(set_error(SPADE_ERR_OOM, "build: records"));
   RunRec* runs;
   ALLOC(runs, NB + NG, "records");
@@ -1170,14 +1171,14 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   TRYF(cudaStreamSynchronize(st), "sync blobs");
   // fine values -2 - offset must stay >= INT32_MIN
   if (units >= (1ll << 31) - 2) return fail(set_error(SPADE_ERR_INVALID_ARG, "boundary index too large (%lld x 16 B)", (long long)units));
-  if (cudaMalloc(&c->recs, sizeof(Rec) * std::max<int64_t>(NR, 1)) != cudaSuccess ||
-      cudaMalloc(&c->blob, 16 * std::max<int64_t>(units, 1)) != cudaSuccess)
+  if (cudaMallocAsync((void**)&c->recs, sizeof(Rec) * std::max<int64_t>(NR, 1), st) != cudaSuccess ||
+      cudaMallocAsync((void**)&c->blob, 16 * std::max<int64_t>(units, 1), st) != cudaSuccess)
     return fail(set_error(SPADE_ERR_OOM, "build: packed records"));
   c->blob_bytes = 16 * units;
   c->multi_unit = multi_unit;
   TRYF(cudaMemsetAsync(c->blob, 0, 16 * std::max<int64_t>(units, 1), st), "memset blob");   // padding bytes defined
   LAUNCH(k_blob_pack, NR, NR, NB, runs, pix_of, g, run_seg, run_mask, rec_polys, boff, bflags, c->recs, c->blob);
-  if (cudaMalloc(&c->kbits, sizeof(uint64_t) * std::max<int64_t>(NR, 1)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: K bits"));
+  if (cudaMallocAsync((void**)&c->kbits, sizeof(uint64_t) * std::max<int64_t>(NR, 1), st) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: K bits"));
   LAUNCH(k_kbits, NR, NR, NB, runs, rec_polys, c->sets, c->set_rng, c->kbits);
   LAUNCH(k_finalize, WH, WH, bflag, bscan, corner, NB, boff, c->fine);
 
@@ -1196,18 +1197,18 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   const bool compact = P < (int32_t)kTileMixedCompact - 1 && h_mixed <= 32768 && !(prm && (prm->flags & SPADE_CANVAS_DENSE));
   const uint32_t owner_lim = compact ? kTileMixedCompact : kTileMixed;     // tile values v+1 below this are uniform
   const int64_t NT1 = (int64_t)(Wc + 1) * (Hc + 1);
-  if (cudaMalloc(&c->coarse, sizeof(uint16_t) * (NT1 + 16)) != cudaSuccess)
+  if (cudaMallocAsync((void**)&c->coarse, sizeof(uint16_t) * (NT1 + 16), st) != cudaSuccess)
     return fail(set_error(SPADE_ERR_OOM, "build: coarse"));
   TRYF(cudaMemsetAsync(c->coarse, 0, sizeof(uint16_t) * (NT1 + 16), st), "memset");
   LAUNCH(k_coarse_final, NT1, tval, mscan, Wc, Hc, compact ? 1 : 0, owner_lim, c->coarse);
   if (compact && h_mixed > 0) {
-    if (cudaMalloc(&c->cfine, sizeof(int32_t) * (h_mixed << (2 * b))) != cudaSuccess)
+    if (cudaMallocAsync((void**)&c->cfine, sizeof(int32_t) * (h_mixed << (2 * b)), st) != cudaSuccess)
       return fail(set_error(SPADE_ERR_OOM, "build: compact canvas"));
     LAUNCH(k_compact, NT << (2 * b), c->fine, g.W, g.H, b, Wc, tval, mscan, NT, owner_lim, c->cfine);
   }
   const bool f16 = !compact && P < (int32_t)kF16Empty && !(prm && (prm->flags & SPADE_CANVAS_NO_FINE16));
   if (f16) {
-    if (cudaMalloc(&c->fine16, sizeof(uint16_t) * WH) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: fine16"));
+    if (cudaMallocAsync((void**)&c->fine16, sizeof(uint16_t) * WH, st) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: fine16"));
     LAUNCH(k_fine16, WH, c->fine, WH, c->fine16);
   }
   stages.mark();                                   // end of K-B5

@@ -55,6 +55,29 @@ int device_sm_count() {
   return sms;
 }
 
+// Streams and events of the host-resident calls, created once per thread and device and reused
+// (a call used to create 2-3 streams and 4-8 events and cudaMalloc its staging buffers; those now
+// come from the stream-ordered pool).
+struct HostStreams {
+  bool ok = false;
+  cudaStream_t s[3] = {};
+  cudaEvent_t ev[8] = {};
+};
+static HostStreams* host_streams() {
+  static thread_local HostStreams hs[16];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  HostStreams& h = hs[dev & 15];
+  if (!h.ok) {
+    for (cudaStream_t& st : h.s)
+      if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) return nullptr;
+    for (cudaEvent_t& e : h.ev)
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+    h.ok = true;
+  }
+  return &h;
+}
+
 static int check_points(const spade_canvas* c, const int32_t* xy, int64_t n, const char* fn) {
   if (!c) return set_error(SPADE_ERR_INVALID_ARG, "%s: canvas is NULL", fn);
   if (n < 0) return set_error(SPADE_ERR_INVALID_ARG, "%s: negative n", fn);
@@ -132,8 +155,13 @@ void spade_canvas_free(spade_canvas* c) {
   if (!c) return;
   DeviceGuard dg(c->device);
   cudaDeviceSynchronize();
-  cudaFree(c->fine); cudaFree(c->fine16); cudaFree(c->cfine); cudaFree(c->coarse); cudaFree(c->recs); cudaFree(c->blob);
-  cudaFree(c->sets); cudaFree(c->set_rng); cudaFree(c->kbits); cudaFree(c->d_dev);
+  // pool allocations (spade_build_canvas) go back to the pool; the header was cudaMalloc'ed
+  for (void* p : {(void*)c->fine, (void*)c->fine16, (void*)c->cfine, (void*)c->coarse, (void*)c->recs, (void*)c->blob,
+                  (void*)c->sets, (void*)c->set_rng, (void*)c->kbits})
+    if (p) cudaFreeAsync(p, 0);
+  cudaFree(c->d_dev);
+  cudaStreamSynchronize(0);
+  cudaGetLastError();
   delete c;
 }
 
@@ -229,31 +257,23 @@ int spade_join_count_host(const spade_canvas* c, const int32_t* xy_host, int64_t
   const int64_t chunk = std::min(kChunk, n);
   int32_t* stage[2] = {nullptr, nullptr};
   int64_t* d_counts = nullptr;
-  cudaStream_t cs = nullptr, ks = nullptr;
-  cudaEvent_t copied[2] = {nullptr, nullptr}, consumed[2] = {nullptr, nullptr};
+  HostStreams* hs = host_streams();
+  if (!hs) return set_error(SPADE_ERR_CUDA, "spade_join_count_host: stream setup failed");
+  keep_pool_memory();
+  cudaStream_t cs = hs->s[0], ks = hs->s[1];
+  cudaEvent_t copied[2] = {hs->ev[0], hs->ev[1]}, consumed[2] = {hs->ev[2], hs->ev[3]};
   cudaError_t e = cudaSuccess;
   auto cleanup = [&]() {
-    if (ks) cudaStreamSynchronize(ks);
-    if (cs) cudaStreamSynchronize(cs);
-    for (int i = 0; i < 2; ++i) {
-      if (stage[i]) cudaFree(stage[i]);
-      if (copied[i]) cudaEventDestroy(copied[i]);
-      if (consumed[i]) cudaEventDestroy(consumed[i]);
-    }
-    if (d_counts) cudaFree(d_counts);
-    if (cs) cudaStreamDestroy(cs);
-    if (ks) cudaStreamDestroy(ks);
+    cudaStreamSynchronize(ks);
+    cudaStreamSynchronize(cs);
+    for (int i = 0; i < 2; ++i)
+      if (stage[i]) cudaFreeAsync(stage[i], st);
+    if (d_counts) cudaFreeAsync(d_counts, st);
   };
 #define HTRY(call, what) do { e = (call); if (e != cudaSuccess) { int r_ = check_cuda(e, what); cleanup(); return r_; } } while (0)
-  HTRY(cudaMalloc(&stage[0], chunk * 8), "staging");
-  HTRY(cudaMalloc(&stage[1], chunk * 8), "staging");
-  HTRY(cudaMalloc(&d_counts, sizeof(int64_t) * P), "counts");
-  HTRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking), "stream");
-  HTRY(cudaStreamCreateWithFlags(&ks, cudaStreamNonBlocking), "stream");
-  for (int i = 0; i < 2; ++i) {
-    HTRY(cudaEventCreateWithFlags(&copied[i], cudaEventDisableTiming), "event");
-    HTRY(cudaEventCreateWithFlags(&consumed[i], cudaEventDisableTiming), "event");
-  }
+  HTRY(cudaMallocAsync((void**)&stage[0], chunk * 8, st), "staging");
+  HTRY(cudaMallocAsync((void**)&stage[1], chunk * 8, st), "staging");
+  HTRY(cudaMallocAsync((void**)&d_counts, sizeof(int64_t) * P, st), "counts");
   // order after prior work on the caller's stream
   HTRY(cudaEventRecord(consumed[0], st), "event");
   HTRY(cudaStreamWaitEvent(cs, consumed[0], 0), "wait");
@@ -305,37 +325,32 @@ static int map_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, in
   int64_t cap_b[2] = {chunk, chunk};
   unsigned long long* d_tot = nullptr;   // [2] device result counters
   unsigned long long* h_tot = nullptr;   // [2] pinned copies
-  cudaStream_t cs = nullptr, ks = nullptr, ds = nullptr;
-  cudaEvent_t copied[2] = {}, consumed[2] = {}, probed[2] = {}, drained[2] = {};
+  HostStreams* hs = host_streams();
+  if (!hs) return set_error(SPADE_ERR_CUDA, "%s: stream setup failed", fn);
+  keep_pool_memory();
+  cudaStream_t cs = hs->s[0], ks = hs->s[1], ds = hs->s[2];
+  cudaEvent_t copied[2] = {hs->ev[0], hs->ev[1]}, consumed[2] = {hs->ev[2], hs->ev[3]},
+              probed[2] = {hs->ev[4], hs->ev[5]}, drained[2] = {hs->ev[6], hs->ev[7]};
   cudaError_t e = cudaSuccess;
   auto cleanup = [&]() {
-    for (cudaStream_t s : {ks, cs, ds})
-      if (s) cudaStreamSynchronize(s);
+    for (cudaStream_t s : {ks, cs, ds}) cudaStreamSynchronize(s);
     for (int i = 0; i < 2; ++i) {
-      cudaFree(stage[i]); cudaFree(d_ids[i]); cudaFree(d_polys[i]);
-      for (cudaEvent_t ev : {copied[i], consumed[i], probed[i], drained[i]})
-        if (ev) cudaEventDestroy(ev);
+      if (stage[i]) cudaFreeAsync(stage[i], st);
+      if (d_ids[i]) cudaFreeAsync(d_ids[i], st);
+      if (d_polys[i]) cudaFreeAsync(d_polys[i], st);
     }
-    cudaFree(d_tot);
+    if (d_tot) cudaFreeAsync(d_tot, st);
     if (h_tot) cudaFreeHost(h_tot);
-    for (cudaStream_t s : {ks, cs, ds})
-      if (s) cudaStreamDestroy(s);
   };
 #define MTRY(call, what) do { e = (call); if (e != cudaSuccess) { int r_ = check_cuda(e, what); cleanup(); return r_; } } while (0)
 #define MRC(expr) do { int r_ = (expr); if (r_ != SPADE_OK) { cleanup(); return r_; } } while (0)
   for (int i = 0; i < 2; ++i) {
-    MTRY(cudaMalloc(&stage[i], chunk * 8), "staging");
-    MTRY(cudaMalloc(&d_ids[i], chunk * 8), "result buffer");
-    if (pairs) MTRY(cudaMalloc(&d_polys[i], chunk * 4), "result buffer");
+    MTRY(cudaMallocAsync((void**)&stage[i], chunk * 8, st), "staging");
+    MTRY(cudaMallocAsync((void**)&d_ids[i], chunk * 8, st), "result buffer");
+    if (pairs) MTRY(cudaMallocAsync((void**)&d_polys[i], chunk * 4, st), "result buffer");
   }
-  MTRY(cudaMalloc(&d_tot, 2 * sizeof(unsigned long long)), "counter");
+  MTRY(cudaMallocAsync((void**)&d_tot, 2 * sizeof(unsigned long long), st), "counter");
   MTRY(cudaHostAlloc(&h_tot, 2 * sizeof(unsigned long long), cudaHostAllocDefault), "pinned counter");
-  MTRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking), "stream");
-  MTRY(cudaStreamCreateWithFlags(&ks, cudaStreamNonBlocking), "stream");
-  MTRY(cudaStreamCreateWithFlags(&ds, cudaStreamNonBlocking), "stream");
-  for (int i = 0; i < 2; ++i)
-    for (cudaEvent_t* ev : {&copied[i], &consumed[i], &probed[i], &drained[i]})
-      MTRY(cudaEventCreateWithFlags(ev, cudaEventDisableTiming), "event");
   MTRY(cudaEventRecord(consumed[0], st), "event");   // order after prior work on the caller's stream
   for (cudaStream_t s : {cs, ks, ds}) MTRY(cudaStreamWaitEvent(s, consumed[0], 0), "wait");
 
@@ -359,10 +374,11 @@ static int map_host(const spade_canvas* c, const int32_t* xy_host, int64_t n, in
       e2 = cudaStreamSynchronize(ds);
       if (e2 == cudaSuccess) e2 = cudaStreamSynchronize(ks);
       if (e2 != cudaSuccess) return check_cuda(e2, fn);
-      cudaFree(d_ids[b]); d_ids[b] = nullptr;
-      cudaFree(d_polys[b]); d_polys[b] = nullptr;
-      e2 = cudaMalloc(&d_ids[b], cnt * 8);
-      if (e2 == cudaSuccess && pairs) e2 = cudaMalloc(&d_polys[b], cnt * 4);
+      cudaFreeAsync(d_ids[b], ks); d_ids[b] = nullptr;
+      if (d_polys[b]) cudaFreeAsync(d_polys[b], ks);
+      d_polys[b] = nullptr;
+      e2 = cudaMallocAsync((void**)&d_ids[b], cnt * 8, ks);
+      if (e2 == cudaSuccess && pairs) e2 = cudaMallocAsync((void**)&d_polys[b], cnt * 4, ks);
       if (e2 != cudaSuccess) return check_cuda(e2, fn);
       cap_b[b] = cnt;
       int rc = probe(b, off, m);
