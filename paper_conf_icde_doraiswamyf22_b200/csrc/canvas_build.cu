@@ -1236,8 +1236,10 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   d.cfine = c->cfine;
   d.fine = c->fine; d.fine16 = c->fine16; d.f16 = f16 ? 1 : 0; d.coarse = c->coarse; d.recs = c->recs; d.blob = c->blob;
   d.sets = c->sets; d.set_rng = c->set_rng; d.kbits = c->kbits;
-  if (cudaMalloc(&c->d_dev, sizeof(CanvasDev)) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
-  if ((ce = cudaMemcpy(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice)) != cudaSuccess) return fail(check_cuda(ce, "canvas header"));
+  if (cudaMallocAsync((void**)&c->d_dev, sizeof(CanvasDev), st) != cudaSuccess) return fail(set_error(SPADE_ERR_OOM, "build: canvas header"));
+  if ((ce = cudaMemcpyAsync(c->d_dev, &d, sizeof(CanvasDev), cudaMemcpyHostToDevice, st)) != cudaSuccess ||
+      (ce = cudaStreamSynchronize(st)) != cudaSuccess)
+    return fail(check_cuda(ce, "canvas header"));
   *out = c;
   return SPADE_OK;
 }

@@ -155,11 +155,10 @@ void spade_canvas_free(spade_canvas* c) {
   if (!c) return;
   DeviceGuard dg(c->device);
   cudaDeviceSynchronize();
-  // pool allocations (spade_build_canvas) go back to the pool; the header was cudaMalloc'ed
+  // every canvas array comes from the stream-ordered pool (spade_build_canvas): back to the pool
   for (void* p : {(void*)c->fine, (void*)c->fine16, (void*)c->cfine, (void*)c->coarse, (void*)c->recs, (void*)c->blob,
-                  (void*)c->sets, (void*)c->set_rng, (void*)c->kbits})
+                  (void*)c->sets, (void*)c->set_rng, (void*)c->kbits, (void*)c->d_dev})
     if (p) cudaFreeAsync(p, 0);
-  cudaFree(c->d_dev);
   cudaStreamSynchronize(0);
   cudaGetLastError();
   delete c;
