@@ -808,13 +808,26 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
       if (wtot) {
         const Slots sl = reserve(wtot, (nvec - 1 - base) / (nctaid_x() * chunk));
         const unsigned lt = (1u << lane) - 1u;
-        uint32_t k0 = 0;
+        const int64_t id0 = prm.o.id_base + prm.head + 4 * (int64_t)(base + tid);
+        if (sl.room >= wtot && sl.b0 + (long long)wtot <= prm.o.cap) {
+          // fast path (warp-uniform): the batch fits the current chunk below the capacity
+          long long p0 = sl.b0;
 #pragma unroll
-        for (int q = 0; q < NPT; ++q) {
-          if ((hm[q] >> lane) & 1u)
-            put_result<MODE>(prm.o, sl.at(k0 + __popc(hm[q] & lt)),
-                             prm.o.id_base + prm.head + 4 * (int64_t)(base + tid) + q, (int)c[q] - 1);
-          k0 += __popc(hm[q]);
+          for (int q = 0; q < NPT; ++q) {
+            if ((hm[q] >> lane) & 1u) {
+              const long long pos = p0 + __popc(hm[q] & lt);
+              __stcs((long long*)prm.o.out_ids + pos, (long long)(id0 + q));
+              if (MODE == kPairs) __stcs(prm.o.out_poly + pos, (int)c[q] - 1);
+            }
+            p0 += __popc(hm[q]);
+          }
+        } else {
+          uint32_t k0 = 0;
+#pragma unroll
+          for (int q = 0; q < NPT; ++q) {
+            if ((hm[q] >> lane) & 1u) put_result<MODE>(prm.o, sl.at(k0 + __popc(hm[q] & lt)), id0 + q, (int)c[q] - 1);
+            k0 += __popc(hm[q]);
+          }
         }
       }
     }
