@@ -283,6 +283,11 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  (256 .. 2^28)
  *   "fine16"       1 (default) / 0: probe canvases that have a 16-bit second level
  *                  (SPADE_CANVAS_NO_FINE16 not set) through it, or through the int32 level
+ *   "tma"          0 (default) / 1: COUNT with in-loop exact tests streams the points by TMA bulk
+ *                  copies (cp.async.bulk + one mbarrier per warp, 1 KB per warp per batch staged
+ *                  in shared memory) instead of 256-bit loads (A/B; measured in profiles/r02)
+ *   "smem_pad_kb"  0 (default) .. 64: unused dynamic shared memory added to probe launches (to
+ *                  compare variants at an equal shared-memory footprint)
  *   "stage_events" 0 (default) / 1: record CUDA events between the stages of every COUNT / SELECT /
  *                  PAIRS call on its stream (synchronises once per sub-launch to read them; see
  *                  spade_last_call_stages)

@@ -99,6 +99,22 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
+// TMA (bulk async copy) helpers: one mbarrier per warp, 1-D bulk copies global -> shared
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t phase) {
+  asm volatile("{\n .reg .pred p;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n}"
+               ::"r"(bar), "r"(phase) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar, uint64_t pol) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+               ::"r"(dst), "l"(src), "r"(bytes), "r"(bar), "l"(pol) : "memory");
+}
+
 __device__ __forceinline__ uint32_t ctaid_x() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%ctaid.x;" : "=r"(r));
@@ -169,6 +185,7 @@ struct Params {
   float l2_frac;              // fraction of fine-canvas lines gathered with L2::evict_last
   unsigned int* rec_cnt;      // COUNT over overlapping polygons: points per multi-owner record, or null
   uint32_t multi_base;        // blob unit of the first multi-owner record header (records at or past it have no edges)
+  uint32_t tma_off;           // QUEUE == 2: byte offset of the TMA stream stages in dynamic shared memory
   unsigned int* kcnt;         // COUNT with K aggregation: points per boundary record, or null
   const int2* xy;
   int64_t n;
@@ -589,12 +606,15 @@ __host__ __device__ __forceinline__ size_t queue_bytes(int mode) {
 }
 __host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
 
+// QUEUE: 0 = boundary points deferred to k_deferred, 1 = in-loop warp queues, 2 = in-loop queues
+// and the point stream staged by TMA (COUNT only; the A/B variant of the "tma" option)
 template <int MODE, int COMPACT, int QUEUE, int KIND>
 __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
   const CanvasDev& cv = prm.cv;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int T = kT, NW = kNW, NPT = kNPT;
+  constexpr bool TMA = QUEUE == 2;
 
   const uint32_t tbytes = (uint32_t)tiles_bytes_for(cv.Wc, cv.Hc);
   uint16_t* tiles = (uint16_t*)smem;
@@ -617,6 +637,10 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   if (MODE == kCountGlobal)
     for (uint32_t i = tid; i < prm.cache_slots; i += T) { ctag[i] = 0xffffffffu; ccnt[i] = 0u; }
   if (tid == 0) s_dfill = 0;
+  // TMA stream stage: one 1-KB slice (the warp's 32 vectors of a batch) + one mbarrier per warp
+  const uint32_t tma_stage = (uint32_t)__cvta_generic_to_shared(smem) + prm.tma_off + (uint32_t)warp * 1024u;
+  const uint32_t tma_bar = (uint32_t)__cvta_generic_to_shared(smem) + prm.tma_off + (uint32_t)NW * 1024u + 8u * warp;
+  if (TMA && lane == 0) mbar_init(tma_bar, 1);
   __syncthreads();
   DEntry* const dreg = QUEUE ? nullptr : prm.defer + (size_t)blockIdx.x * prm.defer_cap;
   const uint64_t pol = policy_evict_last(prm.l2_frac);
@@ -838,12 +862,44 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     // lambdas, which cost these register-bound variants a spill of the loop state
     const uint32_t hist_s = (uint32_t)__cvta_generic_to_shared(myhist), hstride_b = 4u * prm.hcopies;
     Vec4 nxt;
-    if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
+    uint32_t tma_phase = 0;
+    uint64_t spol = 0;
+    if (TMA) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(spol));
+    // TMA: lane 0 starts the bulk copy of the warp's slice of the batch at `b0` into its stage
+    auto tma_issue = [&](uint32_t b0) {
+      const uint32_t w0 = b0 + (uint32_t)warp * 32u;
+      if (lane == 0 && w0 < nvec) {
+        const uint32_t bytes = min(32u, nvec - w0) * 32u;
+        mbar_expect_tx(tma_bar, bytes);
+        bulk_g2s(tma_stage, vp + w0, bytes, tma_bar, spol);
+      }
+    };
+    if (TMA) tma_issue(blockIdx.x * chunk);
+    else if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
     // (the stride is re-read from the special register each batch: kept live, it spilled)
     for (uint32_t base = blockIdx.x * chunk; base < nvec; base += nctaid_x() * chunk) {
-      const Vec4 v = nxt;
+      Vec4 v;
       const uint32_t stride = nctaid_x() * chunk;
-      if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight meanwhile
+      if (TMA) {
+        // wait for this warp's slice, read it from shared memory, start the next batch's copy
+        const uint32_t w0 = base + (uint32_t)warp * 32u;
+        v.a = make_int4(INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN); v.b = v.a;
+        if (w0 < nvec) {
+          mbar_wait(tma_bar, tma_phase);
+          tma_phase ^= 1u;
+          if (w0 + lane < nvec) {
+            const uint32_t a = tma_stage + 32u * lane;
+            asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(v.a.x), "=r"(v.a.y), "=r"(v.a.z), "=r"(v.a.w) : "r"(a) : "memory");
+            asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(v.b.x), "=r"(v.b.y), "=r"(v.b.z), "=r"(v.b.w) : "r"(a + 16u) : "memory");
+          }
+        }
+        __syncwarp();
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic reads before the async-proxy overwrite
+        tma_issue(base + stride);
+      } else {
+        v = nxt;
+        if (base + stride < nvec) load_batch(nxt, base + stride);   // next batch in flight meanwhile
+      }
       // phase A: coarse (shared memory) lookup, branch-free.  Offsets from the extent origin are
       // unsigned; points left of / below the origin wrap to huge values and, like points right of /
       // above the canvas, clamp into the always-empty sentinel column / row (exact because
@@ -1578,8 +1634,12 @@ struct ScratchGuard {
 
 template <int MODE, int COMPACT, int QUEUE, int KIND, int PIPE = 0>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
-  const size_t smem = PIPE ? tiles_bytes_for(c->d.Wc, c->d.Hc) + ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes()
-                           : tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? queue_bytes(MODE) : 0);
+  const size_t base_smem = PIPE ? tiles_bytes_for(c->d.Wc, c->d.Hc) + ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes()
+                                : tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? queue_bytes(MODE) : 0);
+  // TMA stages (1 KB per warp + mbarriers) after everything else, 128-B aligned; the smem_pad_kb
+  // option adds the same amount of unused shared memory to other variants (equal-footprint A/B)
+  const size_t tma_off = (base_smem + 127) & ~(size_t)127;
+  const size_t smem = QUEUE == 2 ? tma_off + (size_t)kNW * (1024 + 8) : base_smem + (size_t)options().smem_pad_kb * 1024;
   void (*kern)(const Params);
   if constexpr (PIPE != 0) kern = k_probe_pipe<MODE, COMPACT, KIND>;
   else kern = k_probe<MODE, COMPACT, QUEUE, KIND>;
@@ -1714,6 +1774,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
     p.l2_frac = (float)options().l2_frac_pct * 0.01f;
     p.defer_cap = (uint32_t)per;
     p.defer_fill = dfill;
+    p.tma_off = (uint32_t)tma_off;
     g_stages.rec(0);
     kern<<<grid, kT, smem, st>>>(p);
     count_launch();
@@ -1850,6 +1911,9 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {
     if (!force_defer && tiles + hc * one + queue <= kSmemSoft) {
       p.hcopies = hc;
+      // A/B option "tma": the same launch with the point stream staged by TMA (+33 KB of stages)
+      if (options().tma && tiles + hc * one + queue + 128 + (size_t)kNW * 1032 <= 227 * 1024)
+        return launch_layout<kCountSmem, 2>(c, (const int2*)xy, n, p, hc * one, st);
       return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hc * one, st);
     }
   }

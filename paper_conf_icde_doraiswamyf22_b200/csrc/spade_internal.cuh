@@ -157,6 +157,8 @@ struct Options {
   int64_t defer_budget_mb;    // deferral scratch per sub-launch (16 B per reserved entry)
   int fine16;                 // probe fine16 canvases through their 16-bit level (1) or the int32 one (0)
   int stage_events;           // record per-stage CUDA events in every probe call (spade_last_call_stages)
+  int tma;                    // COUNT with in-loop queues: point stream staged by TMA bulk copies (A/B)
+  int smem_pad_kb;            // unused dynamic shared memory added to probe launches (equal-footprint A/B)
 };
 constexpr int kProbeStages = 4;   // probe, deferred exact tests, output compaction, counter expansion
 int last_call_stages(float* ms, int cap);
