@@ -535,24 +535,42 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
 // COUNT, in-loop variant: evaluate up to 32 queued boundary points (one per lane).  Out of line:
 // the streaming loop keeps a small register footprint.
 template <int MODE, int KIND>
+__device__ __forceinline__ void drain_point(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, int x, int y,
+                                            unsigned int* hist, uint32_t hstride, unsigned long long* counts,
+                                            unsigned int* kcnt) {
+  const CanvasDev& cv = *cvg;
+  const uint32_t fx = ((uint32_t)x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)y - (uint32_t)cv.miny) >> cv.s;
+  const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
+  const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
+  uint32_t rid = 0;
+  const Rec r = load_rec(cvg, ~c, &rid);
+  if (kcnt)
+    pip_count_delta<KIND>(cvg, x, y, rid, r, kcnt, [&](int q, int d) {
+      if (MODE == kCountSmem) atomicAdd(&hist[(uint32_t)q * hstride], (unsigned int)d);
+      else atomicAdd(counts + q, (unsigned long long)(long long)d);
+    });
+  else
+    pip_eval_rec<KIND>(cvg, x, y, r, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
+}
+
+template <int MODE, int KIND>
 __device__ __noinline__ void drain(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const QEntry* wq,
                                    int cnt, int lane, unsigned int* hist, uint32_t hstride, unsigned long long* counts,
                                    unsigned int* kcnt) {
   if (lane < cnt) {
     const QEntry e = wq[lane];
-    const CanvasDev& cv = *cvg;
-    const uint32_t fx = ((uint32_t)e.x - (uint32_t)cv.minx) >> cv.s, fy = ((uint32_t)e.y - (uint32_t)cv.miny) >> cv.s;
-    const uint32_t t = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
-    const uint32_t c = classify_fine(__ldg(fine_ptr(cv, t, fx, fy)));
-    uint32_t rid = 0;
-    const Rec r = load_rec(cvg, ~c, &rid);
-    if (kcnt)
-      pip_count_delta<KIND>(cvg, e.x, e.y, rid, r, kcnt, [&](int q, int d) {
-        if (MODE == kCountSmem) atomicAdd(&hist[(uint32_t)q * hstride], (unsigned int)d);
-        else atomicAdd(counts + q, (unsigned long long)(long long)d);
-      });
-    else
-      pip_eval_rec<KIND>(cvg, e.x, e.y, r, [&](int q) { count_hit<MODE>(hist, hstride, counts, q); });
+    drain_point<MODE, KIND>(cvg, tiles, e.x, e.y, hist, hstride, counts, kcnt);
+  }
+}
+
+// COUNT drain over a queue of point indices (the TMA variant): the point is re-read (L2)
+template <int MODE, int KIND>
+__device__ __noinline__ void drain_idx(const CanvasDev* __restrict__ cvg, const uint16_t* tiles, const uint32_t* wqi,
+                                       const int2* __restrict__ xy, int cnt, int lane, unsigned int* hist, uint32_t hstride,
+                                       unsigned long long* counts, unsigned int* kcnt) {
+  if (lane < cnt) {
+    const int2 p = __ldg(xy + wqi[lane]);
+    drain_point<MODE, KIND>(cvg, tiles, p.x, p.y, hist, hstride, counts, kcnt);
   }
 }
 
@@ -601,8 +619,8 @@ __device__ __noinline__ void emit_multi(const CanvasDev* __restrict__ cvg, const
 //   COUNT   hcopies x (P + 1) uint32 bins (bin P = "no polygon" trash bin), copy = lane & (hc-1)
 //   QUEUE   (in-loop exact test) kNW x kQCap QEntry (COUNT: coordinates) or uint32 (SELECT/
 //           PAIRS: point index) per warp: boundary points
-__host__ __device__ __forceinline__ size_t queue_bytes(int mode) {
-  return (size_t)kNW * kQCap * (mode == kSelect || mode == kPairs ? sizeof(uint32_t) : sizeof(QEntry));
+__host__ __device__ __forceinline__ size_t queue_bytes(int mode, int queue = 1) {
+  return (size_t)kNW * kQCap * (mode == kSelect || mode == kPairs || queue == 2 ? sizeof(uint32_t) : sizeof(QEntry));
 }
 __host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
 
@@ -628,7 +646,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   __shared__ int s_qn[kNW];                     // QUEUE: per-warp queue fill
   QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : MODE == kCountGlobal ? prm.cache_slots * 8 : 0)) +
                warp * kQCap;
-  uint32_t* wqi = (uint32_t*)rest + warp * kQCap;                 // SELECT/PAIRS queue
+  uint32_t* wqi = (MODE == kCountSmem || MODE == kCountGlobal ? (uint32_t*)wq - warp * kQCap * 2 : (uint32_t*)rest) +
+                  warp * kQCap;                                   // SELECT/PAIRS queue, TMA COUNT queue
   if (QUEUE && lane == 0) s_qn[warp] = 0;
 
   for (uint32_t i = tid; i < tbytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
@@ -967,16 +986,21 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #pragma unroll
             for (int q = 0; q < NPT; ++q)
               if ((bnd >> q) & 1u) {
-                const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
-                const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
-                wq[pos++] = QEntry{x, y};
+                if (TMA) {                   // (TMA variant: 4-B point indices; the drain re-reads the point)
+                  wqi[pos++] = (uint32_t)prm.head + 4 * (base + tid) + q;
+                } else {
+                  const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
+                  const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
+                  wq[pos++] = QEntry{x, y};
+                }
               }
           }
           __syncwarp();
           int qn = s_qn[warp];
           if (qn >= 32) {
             do {
-              drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
+              if (TMA) drain_idx<MODE, KIND>(prm.cvg, tiles, wqi + qn - 32, prm.xy, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
+              else drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
               qn -= 32;
             } while (qn >= 32);
             __syncwarp();
@@ -1021,7 +1045,10 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   }
   if (QUEUE && (MODE == kCountSmem || MODE == kCountGlobal)) {
     __syncwarp();
-    if (s_qn[warp] > 0) drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
+    if (s_qn[warp] > 0) {
+      if (TMA) drain_idx<MODE, KIND>(prm.cvg, tiles, wqi, prm.xy, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
+      else drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
+    }
   }
   __syncthreads();
   if (!QUEUE && tid == 0) prm.defer_fill[blockIdx.x] = min(s_dfill, prm.defer_cap);
@@ -1635,7 +1662,7 @@ struct ScratchGuard {
 template <int MODE, int COMPACT, int QUEUE, int KIND, int PIPE = 0>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
   const size_t base_smem = PIPE ? tiles_bytes_for(c->d.Wc, c->d.Hc) + ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes()
-                                : tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? queue_bytes(MODE) : 0);
+                                : tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? queue_bytes(MODE, QUEUE) : 0);
   // TMA stages (1 KB per warp + mbarriers) after everything else, 128-B aligned; the smem_pad_kb
   // option adds the same amount of unused shared memory to other variants (equal-footprint A/B)
   const size_t tma_off = (base_smem + 127) & ~(size_t)127;
@@ -1912,8 +1939,14 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
     if (!force_defer && tiles + hc * one + queue <= kSmemSoft) {
       p.hcopies = hc;
       // A/B option "tma": the same launch with the point stream staged by TMA (+33 KB of stages)
-      if (options().tma && tiles + hc * one + queue + 128 + (size_t)kNW * 1032 <= 227 * 1024)
-        return launch_layout<kCountSmem, 2>(c, (const int2*)xy, n, p, hc * one, st);
+      if (options().tma) {
+        // the TMA variant (index queue + 33 KB of stages) with as many histogram copies as fit
+        for (uint32_t ht = hc; ht >= 1; ht >>= 1)
+          if (tiles + ht * one + queue_bytes(kCountSmem, 2) + 128 + (size_t)kNW * 1032 <= kSmemSoft + options().tma_slack_kb * 1024) {
+            p.hcopies = ht;
+            return launch_layout<kCountSmem, 2>(c, (const int2*)xy, n, p, ht * one, st);
+          }
+      }
       return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hc * one, st);
     }
   }

@@ -159,6 +159,7 @@ struct Options {
   int stage_events;           // record per-stage CUDA events in every probe call (spade_last_call_stages)
   int tma;                    // COUNT with in-loop queues: point stream staged by TMA bulk copies (A/B)
   int smem_pad_kb;            // unused dynamic shared memory added to probe launches (equal-footprint A/B)
+  int tma_slack_kb;           // "tma": shared memory the TMA variant may use above the 196 KB budget
 };
 constexpr int kProbeStages = 4;   // probe, deferred exact tests, output compaction, counter expansion
 int last_call_stages(float* ms, int cap);
