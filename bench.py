@@ -454,9 +454,16 @@ def main():
     ws, rank, local = dist_env()
     if ws != a.gpus and rank == 0:
         print(f"warning: --gpus {a.gpus} but WORLD_SIZE {ws}", file=sys.stderr)
+    # one process per GPU; SPADE_DIST_BACKEND=gloo lets several ranks share one GPU (a test of the
+    # multi-rank flow on a 1-GPU box: device = local rank modulo the device count)
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("SPADE_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     sp.load()
     for o in a.opt:
         k, v = o.split("=")
