@@ -41,9 +41,6 @@ enum Mode { kCountSmem = 0, kCountGlobal = 1, kSelect = 2, kPairs = 3 };
 constexpr int kT = 1024;           // threads per CTA (one CTA per SM)
 constexpr int kNW = kT / 32;
 constexpr int kNPT = 4;            // points per thread per batch (one 256-bit vector)
-#ifndef SPADE_PIPE_CLASSIFY
-#define SPADE_PIPE_CLASSIFY 1
-#endif
 // Shared memory above ~196 KB per CTA shrinks the L1 carve-out below ~60 KB and costs ~35%
 // (measured on B200); the histogram copies are chosen to stay under it.
 constexpr size_t kSmemSoft = 196 * 1024;
@@ -1023,29 +1020,6 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         for (int q = 0; q < NPT; ++q)
           if (c[q] != 0u && !(c[q] >> 31)) count_cached(ctag, ccnt, prm.cache_slots, prm.o.counts, c[q] - 1u);
       }
-    }
-  } else if (QUEUE && SPADE_PIPE_CLASSIFY) {
-    // SELECT/PAIRS with in-loop queues: the queues hold point indices, so a batch needs no
-    // coordinates after its classification -- classify batch k+1 (tile lookups, fine gathers in
-    // flight) before running batch k's sinks, so the gathers' L2 latency overlaps the sinks
-    Vec4 nxt;
-    U4 ccur;
-    if (first < nvec) {
-      load_batch(nxt, first);
-      const Vec4 v0 = nxt;
-      if (first + nctaid_x() * chunk < nvec) load_batch(nxt, first + nctaid_x() * chunk);
-      ccur = classify(v0);
-    }
-    for (uint32_t base = first; base < nvec; base += nctaid_x() * chunk) {
-      const uint32_t stride = nctaid_x() * chunk;
-      U4 cnext;
-      if (base + stride < nvec) {
-        const Vec4 v1 = nxt;
-        if (base + 2 * stride < nvec) load_batch(nxt, base + 2 * stride);
-        cnext = classify(v1);
-      }
-      process(base, ccur, [](int) { return make_int2(0, 0); });
-      ccur = cnext;
     }
   } else {
     // only the next batch of points is prefetched; there are no CTA barriers in the loop, the 32
