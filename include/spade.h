@@ -288,6 +288,8 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  in shared memory) instead of 256-bit loads (A/B; measured in profiles/r02)
  *   "smem_pad_kb"  0 (default) .. 64: unused dynamic shared memory added to probe launches (to
  *                  compare variants at an equal shared-memory footprint)
+ *   "pipe_notile"  1 (default) / 0: canvases whose coarse tiles are all mixed use the pipelined
+ *                  probe without the tile grid, with a full per-polygon histogram in its place
  *   "stage_events" 0 (default) / 1: record CUDA events between the stages of every COUNT / SELECT /
  *                  PAIRS call on its stream (synchronises once per sub-launch to read them; see
  *                  spade_last_call_stages)

@@ -525,7 +525,7 @@ __device__ __noinline__ void scalar_point(const CanvasDev* __restrict__ cvg, con
   const uint32_t ux = (uint32_t)x - (uint32_t)cv.minx, uy = (uint32_t)y - (uint32_t)cv.miny;
   if (ux > cv.extw || uy > cv.exth) return;
   const uint32_t fx = ux >> cv.s, fy = uy >> cv.s;
-  uint32_t c = tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)];
+  uint32_t c = tiles ? tiles[(fy >> cv.b) * (uint32_t)(cv.Wc + 1) + (fx >> cv.b)] : cv.mix_min;   // null: all mixed
   if (c >= cv.mix_min) c = classify_fine(*fine_ptr(cv, c, fx, fy));
   if (c == 0) return;
   if (c & 0x80000000u) rare_emit_point<MODE, KIND>(cvg, hist, hstride, o, x, y, ~c, pid);
@@ -1078,15 +1078,20 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #endif
 constexpr int kPipeD = SPADE_PIPE_D;
 constexpr size_t kPipeSmem = (size_t)SPADE_PIPE_SMEM_KB * 1024;
-__host__ __device__ __forceinline__ size_t pipe_ring_bytes() { return (size_t)kPipeD * kNPT * kT * 4; }
+__host__ __device__ __forceinline__ size_t pipe_ring_bytes(int d = kPipeD) { return (size_t)d * kNPT * kT * 4; }
+// VAR 2 of the pipelined probe: canvases whose coarse tiles are ALL mixed (C5's 40k polygons)
+// skip the tile grid (an extent test instead of the sentinel lookup) and use the shared memory it
+// and two ring stages free for a full per-polygon histogram (no count cache, no global atomics)
+constexpr int kPipeNoTileD = 2;
 
-template <int MODE, int COMPACT, int KIND>
+template <int MODE, int COMPACT, int KIND, int VAR = 1>
 __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
   const CanvasDev& cv = prm.cv;
   const int tid = threadIdx.x, lane = tid & 31;
-  constexpr int T = kT, NPT = kNPT, D = kPipeD;
-  const uint32_t tbytes = (uint32_t)tiles_bytes_for(cv.Wc, cv.Hc);
+  constexpr bool NOTILE = VAR == 2;
+  constexpr int T = kT, NPT = kNPT, D = NOTILE ? kPipeNoTileD : kPipeD;
+  const uint32_t tbytes = NOTILE ? 0u : (uint32_t)tiles_bytes_for(cv.Wc, cv.Hc);
   uint16_t* tiles = (uint16_t*)smem;
   unsigned char* rest = smem + tbytes;
   const uint32_t P = (uint32_t)cv.num_polys;
@@ -1112,16 +1117,17 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
     const int64_t ntail = prm.n - tail0;
     if (lane < prm.head) {
       const int2 p = prm.xy[lane];
-      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.hcopies, prm.o, p.x, p.y, prm.o.id_base + lane);
+      scalar_point<MODE, KIND>(prm.cvg, NOTILE ? nullptr : tiles, myhist, prm.hcopies, prm.o, p.x, p.y, prm.o.id_base + lane);
     } else if (lane >= 4 && lane - 4 < ntail) {
       const int64_t i = tail0 + (lane - 4);
       const int2 p = prm.xy[i];
-      scalar_point<MODE, KIND>(prm.cvg, tiles, myhist, prm.hcopies, prm.o, p.x, p.y, prm.o.id_base + i);
+      scalar_point<MODE, KIND>(prm.cvg, NOTILE ? nullptr : tiles, myhist, prm.hcopies, prm.o, p.x, p.y, prm.o.id_base + i);
     }
   }
 
   const Vec4* vp = (const Vec4*)(prm.xy + prm.head);
   const uint32_t nvec = (uint32_t)prm.nvec;
+  const uint32_t extw = cv.extw, exth = cv.exth;
   const uint32_t minx = (uint32_t)cv.minx, miny = (uint32_t)cv.miny;
   const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
   const uint32_t Hc = (uint32_t)cv.Hc, Wc1 = Wc + 1u;
@@ -1153,7 +1159,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
         const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
         const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
         const uint32_t ux = (uint32_t)x - minx, uy = (uint32_t)y - miny;
-        const uint32_t c = tiles[min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc)];
+        // (NOTILE: every tile is mixed; points outside the extent are empty)
+        const uint32_t c = NOTILE ? (ux > extw || uy > exth ? 0u : mixmin) : tiles[min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc)];
         const uint32_t sa = slot + q * (T * 4);
         if (c >= mixmin) {
           const uint32_t fx = ux >> s, fy = uy >> s;
@@ -1661,14 +1668,16 @@ struct ScratchGuard {
 
 template <int MODE, int COMPACT, int QUEUE, int KIND, int PIPE = 0>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
-  const size_t base_smem = PIPE ? tiles_bytes_for(c->d.Wc, c->d.Hc) + ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes()
+  const size_t base_smem = PIPE == 2 ? ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes(kPipeNoTileD)
+                         : PIPE ? tiles_bytes_for(c->d.Wc, c->d.Hc) + ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes()
                                 : tiles_bytes_for(c->d.Wc, c->d.Hc) + extra_smem + (QUEUE ? queue_bytes(MODE, QUEUE) : 0);
   // TMA stages (1 KB per warp + mbarriers) after everything else, 128-B aligned; the smem_pad_kb
   // option adds the same amount of unused shared memory to other variants (equal-footprint A/B)
   const size_t tma_off = (base_smem + 127) & ~(size_t)127;
   const size_t smem = QUEUE == 2 ? tma_off + (size_t)kNW * (1024 + 8) : base_smem + (size_t)options().smem_pad_kb * 1024;
   void (*kern)(const Params);
-  if constexpr (PIPE != 0) kern = k_probe_pipe<MODE, COMPACT, KIND>;
+  if constexpr (PIPE == 2) kern = k_probe_pipe<MODE, COMPACT, KIND, 2>;
+  else if constexpr (PIPE != 0) kern = k_probe_pipe<MODE, COMPACT, KIND, 1>;
   else kern = k_probe<MODE, COMPACT, QUEUE, KIND>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
@@ -1920,6 +1929,15 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   const int pipe_opt = options().pipe;
   const bool pipe_auto = c->mixed_tile_frac > 0.5 && tiles + 2 * one > kSmemSoft && tiles + one <= 227 * 1024;
   if (pipe_opt == 1 || (pipe_opt < 0 && pipe_auto && !force_defer && !force_global)) {
+    // every tile mixed and a dense second level: the tile-less variant with a full histogram
+    if (options().pipe_notile && c->mixed_tile_frac >= 0.999 && !c->d.compact && !force_global) {
+      const size_t ring2 = pipe_ring_bytes(kPipeNoTileD);
+      for (uint32_t hc = 8; hc >= 1; hc >>= 1)
+        if (((hc * one + 15) & ~(size_t)15) + ring2 <= kPipeSmem) {
+          p.hcopies = hc;
+          return launch_layout<kCountSmem, 0, 2>(c, (const int2*)xy, n, p, hc * one, st);
+        }
+    }
     const size_t ring = pipe_ring_bytes();
     for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {
       if (tiles + ((hc * one + 15) & ~(size_t)15) + ring <= kPipeSmem) {

@@ -160,6 +160,7 @@ struct Options {
   int tma;                    // COUNT with in-loop queues: point stream staged by TMA bulk copies (A/B)
   int smem_pad_kb;            // unused dynamic shared memory added to probe launches (equal-footprint A/B)
   int tma_slack_kb;           // "tma": shared memory the TMA variant may use above the 196 KB budget
+  int pipe_notile;            // all-mixed canvases: the tile-less pipelined probe with a full histogram
 };
 constexpr int kProbeStages = 4;   // probe, deferred exact tests, output compaction, counter expansion
 int last_call_stages(float* ms, int cap);

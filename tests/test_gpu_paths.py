@@ -17,7 +17,7 @@ from tests.helpers import lattice, random_polyset, sorted_pairs
 pytestmark = pytest.mark.gpu
 
 DEFAULTS = {"defer": 0, "count_global": 0, "global_queue": 0, "cache_slots": 4096, "coop": 0, "pipe": -1,
-            "defer_xy": 0, "multi_agg": 1, "k_agg": -1, "tma": 0, "fine16": 1}
+            "defer_xy": 0, "multi_agg": 1, "k_agg": -1, "tma": 0, "fine16": 1, "pipe_notile": 1}
 
 COUNT_PATHS = [
     {},
@@ -47,6 +47,7 @@ COUNT_PATHS = [
     {"k_agg": 1, "pipe": 1},
     {"k_agg": 1, "multi_agg": 0, "pipe": 1, "count_global": 1},
     {"tma": 1},
+    {"pipe": 1, "pipe_notile": 1},
     {"tma": 1, "k_agg": 1},
     {"fine16": 0, "pipe": 1},
 ]
