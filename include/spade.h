@@ -288,8 +288,14 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  in shared memory) instead of 256-bit loads (A/B; measured in profiles/r02)
  *   "smem_pad_kb"  0 (default) .. 64: unused dynamic shared memory added to probe launches (to
  *                  compare variants at an equal shared-memory footprint)
- *   "pipe_notile"  1 (default) / 0: canvases whose coarse tiles are all mixed use the pipelined
+ *   "pipe_notile"  0 (default) / 1: canvases whose coarse tiles are all mixed use the pipelined
  *                  probe without the tile grid, with a full per-polygon histogram in its place
+ *                  (measured slower on C5: 13.6 vs 11.2 ms; A/B only)
+ *   "hist_copies_max"  16 (default), 32, 8, 4, 2, 1: most copies of the COUNT shared-memory
+ *                  histogram (copy = lane mod copies; 32 = one bank per lane, no conflicts)
+ *   "idx_queue"    0 (default) / 1 / -1 (when it makes room for more histogram copies): COUNT
+ *                  in-loop queues hold 4-B point indices instead of 8-B points (A/B: C3 with
+ *                  32 copies and index queues 1.95 ms vs 1.73 ms with 16 copies and point queues)
  *   "stage_events" 0 (default) / 1: record CUDA events between the stages of every COUNT / SELECT /
  *                  PAIRS call on its stream (synchronises once per sub-launch to read them; see
  *                  spade_last_call_stages)

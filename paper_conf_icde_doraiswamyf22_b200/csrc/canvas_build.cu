@@ -1194,7 +1194,7 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   TRYF(cudaMemcpyAsync(&last_mix, tmix + NT - 1, 4, cudaMemcpyDeviceToHost, st), "mixed");
   TRYF(cudaStreamSynchronize(st), "sync coarse");
   const int64_t h_mixed = (int64_t)last_scan + last_mix;
-  const bool compact = P < (int32_t)kTileMixedCompact - 1 && h_mixed <= 32768 && !(prm && (prm->flags & SPADE_CANVAS_DENSE));
+  const bool compact = P < (int32_t)kTileMixedCompact - 1 && h_mixed <= 32768 && b <= 8 && !(prm && (prm->flags & SPADE_CANVAS_DENSE));
   const uint32_t owner_lim = compact ? kTileMixedCompact : kTileMixed;     // tile values v+1 below this are uniform
   const int64_t NT1 = (int64_t)(Wc + 1) * (Hc + 1);
   if (cudaMallocAsync((void**)&c->coarse, sizeof(uint16_t) * (NT1 + 16), st) != cudaSuccess)

@@ -38,7 +38,10 @@ namespace {
 
 enum Mode { kCountSmem = 0, kCountGlobal = 1, kSelect = 2, kPairs = 3 };
 
-constexpr int kT = 1024;           // threads per CTA (one CTA per SM)
+#ifndef SPADE_PROBE_T
+#define SPADE_PROBE_T 1024
+#endif
+constexpr int kT = SPADE_PROBE_T;  // threads per CTA (one CTA per SM)
 constexpr int kNW = kT / 32;
 constexpr int kNPT = 4;            // points per thread per batch (one 256-bit vector)
 // Shared memory above ~196 KB per CTA shrinks the L1 carve-out below ~60 KB and costs ~35%
@@ -187,6 +190,7 @@ struct Params {
   uint32_t multi_base;        // blob unit of the first multi-owner record header (records at or past it have no edges)
   uint32_t tma_off;           // QUEUE == 2: byte offset of the TMA stream stages in dynamic shared memory
   unsigned int* kcnt;         // COUNT with K aggregation: points per boundary record, or null
+  const int32_t* cfine_tile0;  // compact layout: cfine - (0x8000 << 2b), the block of tile entry 0x8000 (b <= 8)
   const int2* xy;
   int64_t n;
   int64_t head;               // points before the first 32-byte aligned one (0..3)
@@ -620,12 +624,13 @@ __device__ __noinline__ void emit_multi(const CanvasDev* __restrict__ cvg, const
 //   QUEUE   (in-loop exact test) kNW x kQCap QEntry (COUNT: coordinates) or uint32 (SELECT/
 //           PAIRS: point index) per warp: boundary points
 __host__ __device__ __forceinline__ size_t queue_bytes(int mode, int queue = 1) {
-  return (size_t)kNW * kQCap * (mode == kSelect || mode == kPairs || queue == 2 ? sizeof(uint32_t) : sizeof(QEntry));
+  return (size_t)kNW * kQCap * (mode == kSelect || mode == kPairs || queue >= 2 ? sizeof(uint32_t) : sizeof(QEntry));
 }
 __host__ __device__ __forceinline__ size_t tiles_bytes_for(int Wc, int Hc) { return (((size_t)(Wc + 1) * (Hc + 1)) * 2 + 15) & ~(size_t)15; }
 
 // QUEUE: 0 = boundary points deferred to k_deferred, 1 = in-loop warp queues, 2 = in-loop queues
-// and the point stream staged by TMA (COUNT only; the A/B variant of the "tma" option)
+// and the point stream staged by TMA (COUNT only; the A/B variant of the "tma" option), 3 = in-loop
+// queues of 4-B point indices (COUNT: frees shared memory for more histogram copies)
 template <int MODE, int COMPACT, int QUEUE, int KIND>
 __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params prm) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -633,6 +638,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int T = kT, NW = kNW, NPT = kNPT;
   constexpr bool TMA = QUEUE == 2;
+  constexpr bool IDXQ = QUEUE >= 2;             // COUNT queue of 4-B point indices (the drain re-reads the point)
 
   const uint32_t tbytes = (uint32_t)tiles_bytes_for(cv.Wc, cv.Hc);
   uint16_t* tiles = (uint16_t*)smem;
@@ -757,8 +763,13 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
         const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
         const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
-        const uint32_t fidx = COMPACT == 1 ? ((((f[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
-        f[q] = COMPACT == 2 ? class16(ld_fine16(f16p + fidx, pol)) : classify_fine((int32_t)ld_fine(finep + fidx, pol));
+        if (COMPACT == 1) {        // (see the COUNT loop: tile entry's flag bit folded into cfine_tile0)
+          const uint32_t fidx = (f[q] * (bm + 1u) + (fy & bm)) * (bm + 1u) + (fx & bm);
+          f[q] = classify_fine((int32_t)ld_fine(prm.cfine_tile0 + fidx, pol));
+        } else {
+          const uint32_t fidx = fy * W + fx;
+          f[q] = COMPACT == 2 ? class16(ld_fine16(f16p + fidx, pol)) : classify_fine((int32_t)ld_fine(finep + fidx, pol));
+        }
       }
     }
     return f;
@@ -896,6 +907,9 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
     if (TMA) tma_issue(blockIdx.x * chunk);
     else if (blockIdx.x * chunk < nvec) load_batch(nxt, blockIdx.x * chunk);
     // (the stride is re-read from the special register each batch: kept live, it spilled)
+#ifdef SPADE_COUNT_UNROLL2
+#pragma unroll 2
+#endif
     for (uint32_t base = blockIdx.x * chunk; base < nvec; base += nctaid_x() * chunk) {
       Vec4 v;
       const uint32_t stride = nctaid_x() * chunk;
@@ -931,15 +945,24 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
         const uint32_t ux = (uint32_t)x - minx, uy = (uint32_t)y - miny;
         c[q] = tiles[min(uy >> sb, Hc) * Wc1 + min(ux >> sb, Wc)];
       }
-      // phase B: fine pixels of mixed tiles; all gathers of the batch in flight together
+      // phase B: fine pixels of mixed tiles; all gathers of the batch in flight together.
+      // Compact layout: the pixel is ((t·B + ly)·B + lx) past cfine_tile0, the base of the block of
+      // tile entry t = 0x8000 | m (t's flag bit folded into the base pointer, B = 2^b): two IMADs
+      // instead of the shift/mask chain (this phase's instructions issue for every point of a warp
+      // in which any point needs a gather, i.e. nearly always).
 #pragma unroll
       for (int q = 0; q < NPT; ++q) {
         if (c[q] >= mixmin) {
           const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
           const int y = q == 0 ? v.a.y : q == 1 ? v.a.w : q == 2 ? v.b.y : v.b.w;
           const uint32_t fx = ((uint32_t)x - minx) >> s, fy = ((uint32_t)y - miny) >> s;
-          const uint32_t fidx = COMPACT == 1 ? ((((c[q] & 0x7fffu) << b) | (fy & bm)) << b) | (fx & bm) : fy * W + fx;
-          c[q] = COMPACT == 2 ? class16(ld_fine16(f16p + fidx, pol)) : classify_fine((int32_t)ld_fine(finep + fidx, pol));
+          if (COMPACT == 1) {
+            const uint32_t fidx = (c[q] * (bm + 1u) + (fy & bm)) * (bm + 1u) + (fx & bm);
+            c[q] = classify_fine((int32_t)ld_fine(prm.cfine_tile0 + fidx, pol));
+          } else {
+            const uint32_t fidx = fy * W + fx;
+            c[q] = COMPACT == 2 ? class16(ld_fine16(f16p + fidx, pol)) : classify_fine((int32_t)ld_fine(finep + fidx, pol));
+          }
         }
       }
       // now c = 0 (none) | owner + 1 | >= 2^31: boundary / multi-owner record ~c
@@ -986,7 +1009,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
 #pragma unroll
             for (int q = 0; q < NPT; ++q)
               if ((bnd >> q) & 1u) {
-                if (TMA) {                   // (TMA variant: 4-B point indices; the drain re-reads the point)
+                if (IDXQ) {                  // (index queue: 4-B point indices; the drain re-reads the point)
                   wqi[pos++] = (uint32_t)prm.head + 4 * (base + tid) + q;
                 } else {
                   const int x = q == 0 ? v.a.x : q == 1 ? v.a.z : q == 2 ? v.b.x : v.b.z;
@@ -999,7 +1022,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
           int qn = s_qn[warp];
           if (qn >= 32) {
             do {
-              if (TMA) drain_idx<MODE, KIND>(prm.cvg, tiles, wqi + qn - 32, prm.xy, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
+              if (IDXQ) drain_idx<MODE, KIND>(prm.cvg, tiles, wqi + qn - 32, prm.xy, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
               else drain<MODE, KIND>(prm.cvg, tiles, wq + qn - 32, 32, lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
               qn -= 32;
             } while (qn >= 32);
@@ -1046,7 +1069,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   if (QUEUE && (MODE == kCountSmem || MODE == kCountGlobal)) {
     __syncwarp();
     if (s_qn[warp] > 0) {
-      if (TMA) drain_idx<MODE, KIND>(prm.cvg, tiles, wqi, prm.xy, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
+      if (IDXQ) drain_idx<MODE, KIND>(prm.cvg, tiles, wqi, prm.xy, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
       else drain<MODE, KIND>(prm.cvg, tiles, wq, s_qn[warp], lane, myhist, prm.hcopies, prm.o.counts, prm.kcnt);
     }
   }
@@ -1893,6 +1916,8 @@ Params base_params(const spade_canvas* c) {
   p.cv = c->d;
   p.cvg = c->d_dev;
   p.hcopies = 1;
+  // (wraps below cfine: only ever offset back into it by a tile entry's 0x8000 << 2b)
+  if (c->d.compact) p.cfine_tile0 = (const int32_t*)((uintptr_t)c->d.cfine - ((uintptr_t)kTileMixedCompact << (2 * c->d.b)) * 4u);
   return p;
 }
 
@@ -1953,8 +1978,14 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
       return launch_layout<kCountGlobal, 0, 1>(c, (const int2*)xy, n, p, (size_t)slots * 8, st);
     }
   }
-  for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {
-    if (!force_defer && tiles + hc * one + queue <= kSmemSoft) {
+  // Histogram copies: copy = lane & (hc - 1) at bin·hc + copy, so with 32 copies every lane of
+  // a warp increments its own bank (the histogram atomics were the largest share of C3's
+  // shared-memory wavefronts: 124M of 240M, 88M of them bank conflicts, at 8 copies).  A queue of
+  // 4-B point indices (the drain re-reads its points) makes room for them beside big tile grids.
+  const uint32_t hmax = (uint32_t)options().hist_copies_max;
+  const int idxq = options().idx_queue;
+  for (uint32_t hc = hmax; hc >= 1 && !force_global; hc >>= 1) {
+    if (!force_defer && idxq != 1 && tiles + hc * one + queue <= kSmemSoft) {
       p.hcopies = hc;
       // A/B option "tma": the same launch with the point stream staged by TMA (+33 KB of stages)
       if (options().tma) {
@@ -1966,6 +1997,10 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
           }
       }
       return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hc * one, st);
+    }
+    if (!force_defer && idxq != 0 && tiles + hc * one + queue_bytes(kCountSmem, 3) <= kSmemSoft) {
+      p.hcopies = hc;
+      return launch_layout<kCountSmem, 3>(c, (const int2*)xy, n, p, hc * one, st);
     }
   }
   for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {

@@ -129,7 +129,8 @@ Options& options() {
                    env_int("SPADE_PIPE", -1), env_int("SPADE_DEFER_XY", 0), env_int("SPADE_L2_FRAC_PCT", 100), env_int("SPADE_MULTI_AGG", 1), env_int("SPADE_K_AGG", -1),
                    (int64_t)1 << 25, (1ll << 31) - 64, 4096, env_int("SPADE_FINE16", 1),
                    env_int("SPADE_STAGE_EVENTS", 0), env_int("SPADE_TMA", 0), env_int("SPADE_SMEM_PAD_KB", 0),
-                   env_int("SPADE_TMA_SLACK_KB", 0), env_int("SPADE_PIPE_NOTILE", 1)};
+                   env_int("SPADE_TMA_SLACK_KB", 0), env_int("SPADE_PIPE_NOTILE", 0),
+                   env_int("SPADE_HIST_COPIES_MAX", 16), env_int("SPADE_IDX_QUEUE", 0)};
   return o;
 }
 }  // namespace spade
@@ -574,6 +575,8 @@ int spade_set_option(const char* name, int64_t value) {
   else if (n == "smem_pad_kb" && value >= 0 && value <= 64) o.smem_pad_kb = (int)value;
   else if (n == "tma_slack_kb" && value >= 0 && value <= 31) o.tma_slack_kb = (int)value;
   else if (n == "pipe_notile" && bit) o.pipe_notile = (int)value;
+  else if (n == "hist_copies_max" && value >= 1 && value <= 32 && (value & (value - 1)) == 0) o.hist_copies_max = (int)value;
+  else if (n == "idx_queue" && (value == -1 || bit)) o.idx_queue = (int)value;
   else if (n == "coop" && (value == -1 || value == 0 || value == 4 || value == 8 || value == 16)) o.coop = (int)value;
   else return set_error(SPADE_ERR_INVALID_ARG, "spade_set_option: bad option %s = %lld", name, (long long)value);
   return SPADE_OK;

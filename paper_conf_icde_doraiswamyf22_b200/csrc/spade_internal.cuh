@@ -161,6 +161,8 @@ struct Options {
   int smem_pad_kb;            // unused dynamic shared memory added to probe launches (equal-footprint A/B)
   int tma_slack_kb;           // "tma": shared memory the TMA variant may use above the 196 KB budget
   int pipe_notile;            // all-mixed canvases: the tile-less pipelined probe with a full histogram
+  int hist_copies_max;        // COUNT shared-memory histogram copies, at most (power of 2, <= 32)
+  int idx_queue;              // COUNT in-loop queues of point indices: -1 auto, 0 never, 1 always
 };
 constexpr int kProbeStages = 4;   // probe, deferred exact tests, output compaction, counter expansion
 int last_call_stages(float* ms, int cap);

@@ -17,7 +17,8 @@ from tests.helpers import lattice, random_polyset, sorted_pairs
 pytestmark = pytest.mark.gpu
 
 DEFAULTS = {"defer": 0, "count_global": 0, "global_queue": 0, "cache_slots": 4096, "coop": 0, "pipe": -1,
-            "defer_xy": 0, "multi_agg": 1, "k_agg": -1, "tma": 0, "fine16": 1, "pipe_notile": 1}
+            "defer_xy": 0, "multi_agg": 1, "k_agg": -1, "tma": 0, "fine16": 1, "pipe_notile": 0,
+            "hist_copies_max": 16, "idx_queue": 0}
 
 COUNT_PATHS = [
     {},
@@ -50,6 +51,12 @@ COUNT_PATHS = [
     {"pipe": 1, "pipe_notile": 1},
     {"tma": 1, "k_agg": 1},
     {"fine16": 0, "pipe": 1},
+    {"idx_queue": 1},
+    {"idx_queue": -1, "hist_copies_max": 32},
+    {"idx_queue": 1, "k_agg": 1},
+    {"hist_copies_max": 8, "idx_queue": 0},
+    {"hist_copies_max": 1, "idx_queue": 1},
+    {"hist_copies_max": 16, "multi_agg": 0},
 ]
 
 
