@@ -5,6 +5,6 @@ set -e
 R=$(cd "$(dirname "$0")/.." && pwd); C=$R/paper_conf_icde_doraiswamyf22_b200/csrc
 OUT=$1; FLAGS=$2; T=$(mktemp -d)
 F="-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 --expt-relaxed-constexpr -Xcompiler -fPIC,-fvisibility=hidden"
-nvcc $F $FLAGS -I $R/include -dc -o $T/probe.o $C/probe.cu
+nvcc $F $FLAGS -I $R/include -dc -o $T/probe.o $C/probe.cu > $T/log 2>&1 || { cat $T/log; exit 1; }
 nvcc -gencode arch=compute_100a,code=sm_100a -shared -Xcompiler -fPIC -o $OUT $C/spade_api.o $C/canvas_build.o $T/probe.o $C/knn.o $C/polygon_join.o
 rm -rf $T
