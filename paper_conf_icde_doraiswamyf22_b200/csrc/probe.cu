@@ -207,7 +207,11 @@ template <int MODE, int LAYOUT = 0, class C>
 __device__ __forceinline__ void count_multi_owner(const Params& prm, C& c) {
   // (fine16: a record's id is not in the 16-bit code; the exact-test stage counts them)
   if (!(MODE == kCountSmem || MODE == kCountGlobal) || LAYOUT == 2 || prm.rec_cnt == nullptr) return;
-  if ((int)(c[0] | c[1] | c[2] | c[3]) >= 0) return;
+  // (one warp vote on the way in; measured: C3 1.72 -> 1.69 ms against a per-lane test, ov flat.
+  // Warp-aggregating the atomics with __match_any_sync was measured too: ov 29.1 -> 29.5-29.9 ms,
+  // the lanes of a warp rarely share a record; removing them altogether gives 24.6 ms)
+  const unsigned act = __activemask();
+  if (!__any_sync(act, (int)(c[0] | c[1] | c[2] | c[3]) < 0)) return;
 #pragma unroll
   for (int q = 0; q < kNPT; ++q)
     if ((c[q] >> 31) && ~c[q] >= prm.multi_base) {
