@@ -25,18 +25,30 @@ def build(force: bool = False, verbose: bool = False) -> str:
     deps = srcs + [os.path.abspath(__file__), os.path.join(CSRC, "spade_internal.cuh"), os.path.join(ROOT, "include", "spade.h")]
     if not force and not _stale(LIB, deps):
         return LIB
+    # Each translation unit is its own device module (no device link across them): CUDA's lazy
+    # loading then loads only the module of the kernels a call uses -- a first canvas build loads
+    # the builder's ~1 MB module, not the probe's ~16 MB (C5 cold build 2.0 s -> see DESIGN.md).
+    # probe.cu keeps separate compilation (-dc + its own device link: its register allocation
+    # was tuned that way).
     objs = []
     for s in srcs:
         o = os.path.join(CSRC, os.path.basename(s).replace(".cu", ".o"))
-        cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-dc", "-o", o, s]
+        rdc = os.path.basename(s) == "probe.cu"
+        cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-dc" if rdc else "-c", "-o", o, s]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"nvcc failed for {s}:\n{r.stdout}\n{r.stderr}")
         if verbose:
             print(r.stderr)
         objs.append(o)
-    cmd = ["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-Xcompiler", "-fPIC",
-           "-o", LIB, *objs]
+        if rdc:
+            dl = o.replace(".o", "_dlink.o")
+            cmd = ["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-Xcompiler", "-fPIC", "-dlink", "-o", dl, o]
+            r = subprocess.run(cmd, capture_output=True, text=True)
+            if r.returncode != 0:
+                raise RuntimeError(f"device link failed for {s}:\n{r.stdout}\n{r.stderr}")
+            objs.append(dl)
+    cmd = ["g++", "-shared", "-fPIC", "-o", LIB, *objs, "-L/usr/local/cuda/lib64", "-lcudadevrt", "-lcudart_static", "-lrt", "-lpthread", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
