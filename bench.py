@@ -49,6 +49,9 @@ def parse():
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu/clocks)")
     ap.add_argument("--dense", action="store_true", help="force the dense fine-canvas layout (A/B runs)")
     ap.add_argument("--count", action="store_true", help="run COUNT on the workload's canvas and points (A/B of the sinks)")
+    ap.add_argument("--layers", action="store_true",
+                    help="COUNT through the paper's layer index (spade_build_layered: one probe pass per layer of "
+                         "non-intersecting polygons) instead of the owner sets of one canvas (A/B, P:148 / P:270-274)")
     ap.add_argument("--max-dim", type=int, default=None, help="override the workload's canvas max_dim")
     ap.add_argument("--opt", action="append", default=[], metavar="NAME=VALUE",
                     help="spade_set_option before the run (A/B of probe paths; results never depend on it)")
@@ -503,6 +506,13 @@ def main():
     cv = cv2
     info = cv.info() if cv is not None else {}
     build_stages = cv.build_times() if cv is not None else {}
+    lc, layers_info = None, None
+    if a.layers and w.op == "count" and not is_dist:
+        t0 = time.perf_counter()
+        lc = sp.LayeredCanvas(w.polys, max_dim=a.max_dim or w.max_dim)
+        torch.cuda.synchronize()
+        layers_info = {"num_layers": lc.num_layers, "build_s": time.perf_counter() - t0,
+                       "plan": "layer index: one canvas and one probe pass per layer (spade_join_count_layered)"}
 
     # this rank's shard: global indices [rank*n, (rank+1)*n), generated in place on the device
     xy = torch.empty((n, 2), dtype=torch.int32, device=dev)
@@ -521,7 +531,10 @@ def main():
         if ev_k0 is not None:
             ev_k0.record(stream)
         if op == "count":
-            sp.join_count(cv, xy, counts)
+            if lc is not None:
+                sp.join_count_layered(lc, xy, counts)
+            else:
+                sp.join_count(cv, xy, counts)
         elif op == "knn":
             n_results[0] = sp.knn(xy, w.query, w.k, point_id_base=rank * n)[0].numel()
         elif op == "select":
@@ -584,6 +597,13 @@ def main():
         check = {"k_returned": n_results[0], "k": w.k, "note": "single-GPU kNN per rank (N>1: per-shard)"}
     else:
         check = {"selected": n_results[0], "selectivity": n_results[0] / n}
+    if lc is not None:
+        # the layered plan's counts (the last step's) against the owner-set canvas on the same shard
+        ref = torch.zeros(P, dtype=torch.int64, device=dev)
+        sp.join_count(cv, xy, ref)
+        if ws > 1:
+            dist.all_reduce(ref)
+        check["layers_equal_owner_sets"] = bool(torch.equal(ref, counts))
 
     kavg = statistics.mean(kern_ms)
     peak, peak_src = measured_peak()
@@ -610,7 +630,7 @@ def main():
     out_bytes = {"count": 0, "select": 8 * n_results[0], "pairs": 12 * n_results[0], "knn": n * 8}[op]
     alg_bytes = n * 8 + out_bytes
     achieved = alg_bytes / (kavg / 1e3) / 1e9
-    traffic, traffic_src = ncu_traffic(w.name)
+    traffic, traffic_src = ncu_traffic(w.name) if lc is None else (None, None)
 
     line = None
     if rank == 0:
@@ -624,6 +644,7 @@ def main():
                    else {"polygons": P, "vertices": int(len(w.polys["ring_xy"]))}),
                 "parallelism": f"dp{ws} (points sharded, canvas replicated)",
                 "l2": "inputs (8 B/point, >= 8 GB per GPU) exceed the 126 MB L2; no flush needed",
+                **({"layers": layers_info} if layers_info else {}),
                 "canvas": info, "canvas_build_s": build_s, "canvas_build_cold_s": build_cold_s,
                 "canvas_build_stage_ms": build_stages,
                 **({"options": a.opt} if a.opt else {}),

@@ -206,6 +206,36 @@ SPADE_API int spade_join_polygons(const int32_t* ring_xy1, const int64_t* ring_o
                                   const int64_t* poly_ring_off2, int32_t num_polys2, const spade_canvas_params* prm,
                                   int32_t* out_a, int32_t* out_b, int64_t capacity, int64_t* n_out, spade_stream_t stream);
 
+/* ---- Layer index ---------------------------------------------------
+ * The paper's plan for overlapping polygon sets: layers of mutually non-intersecting polygons, one
+ * canvas and one pass over the points per layer.  (spade_build_canvas handles overlaps exactly in
+ * ONE canvas with owner sets; this is the alternative plan, kept for comparison: DESIGN.md §6.)
+ *
+ * spade_layer_assign: greedy colouring (Welsh-Powell) of the conflict graph given as npairs HOST
+ *   pairs (pair_a[i], pair_b[i]) of polygon ids in [0, P) (self pairs and duplicates allowed):
+ *   layer_of [P] HOST output, layer of each polygon, such that no pair shares a layer;
+ *   num_layers HOST output.  Host-only (no device work).  Ids out of range -> INVALID_ARG.
+ * spade_build_layered: conflicts = the closed-intersection self-join of the set
+ *   (spade_join_polygons; touching polygons conflict too), layers by spade_layer_assign, then one
+ *   spade_build_canvas per layer over all P polygon slots (the other layers' polygons get no
+ *   rings), so every layer's COUNT uses global polygon ids.  Arguments as spade_build_canvas (device
+ *   arrays, which must be VALID polygons as for spade_join_polygons); `*out` owns the canvases
+ *   (spade_layered_free).  Synchronises `stream`.
+ * spade_join_count_layered: COUNT as spade_join_count, one probe pass per layer, ACCUMULATED into
+ *   the device counts [P] (the caller zeroes them).
+ * spade_layered_info: number of layers; layer_of [P] HOST (may be NULL).
+ * spade_layered_free: frees the layers (NULL: no-op). */
+typedef struct spade_layered spade_layered;
+SPADE_API int spade_layer_assign(const int32_t* pair_a, const int32_t* pair_b, int64_t npairs, int32_t num_polys,
+                                 int32_t* layer_of, int32_t* num_layers);
+SPADE_API int spade_build_layered(const int32_t* ring_xy, const int64_t* ring_off, const int64_t* poly_ring_off,
+                                  int32_t num_polys, const spade_canvas_params* prm, spade_stream_t stream,
+                                  spade_layered** out);
+SPADE_API int spade_join_count_layered(const spade_layered* layered, const int32_t* xy, int64_t n, int64_t* counts,
+                                       spade_stream_t stream);
+SPADE_API int spade_layered_info(const spade_layered* layered, int32_t* num_layers, int32_t* layer_of);
+SPADE_API void spade_layered_free(spade_layered* layered);
+
 /* ---- kNN selection over points (Sec. 5.2), in the paper's three steps ------------
  * The circles of step 1 are concentric around the query q with squared radii
  *   r2_b = the largest squared distance of bucket b,  b = 0 .. SPADE_KNN_BINS-1, where

@@ -98,6 +98,16 @@ def load(path: str | None = None):
     lib.spade_knn_topk.restype = ctypes.c_int
     lib.spade_knn.argtypes = [P, i64, i64, i32, i32, i64, P, P, ctypes.POINTER(i64), P]
     lib.spade_knn.restype = ctypes.c_int
+    lib.spade_layer_assign.argtypes = [P, P, i64, i32, P, ctypes.POINTER(i32)]
+    lib.spade_layer_assign.restype = ctypes.c_int
+    lib.spade_build_layered.argtypes = [P, P, P, i32, ctypes.POINTER(CanvasParams), P, ctypes.POINTER(P)]
+    lib.spade_build_layered.restype = ctypes.c_int
+    lib.spade_join_count_layered.argtypes = [P, P, i64, P, P]
+    lib.spade_join_count_layered.restype = ctypes.c_int
+    lib.spade_layered_info.argtypes = [P, ctypes.POINTER(i32), P]
+    lib.spade_layered_info.restype = ctypes.c_int
+    lib.spade_layered_free.argtypes = [P]
+    lib.spade_layered_free.restype = None
     lib.spade_set_option.argtypes = [ctypes.c_char_p, i64]
     lib.spade_set_option.restype = ctypes.c_int
     lib.spade_last_call_stages.argtypes = [ctypes.POINTER(ctypes.c_float), i32]
@@ -116,7 +126,8 @@ EXPORTED_SYMBOLS = ["spade_build_canvas", "spade_build_disk_canvas", "spade_canv
                     "spade_canvas_checksum", "spade_canvas_build_times", "spade_canvas_build_stage_name", "spade_join_polygons", "spade_join_count",
                     "spade_select", "spade_join_pairs", "spade_join_count_host", "spade_select_host", "spade_join_pairs_host", "spade_knn_histogram",
                     "spade_knn_radius", "spade_knn_select", "spade_knn_topk", "spade_knn", "spade_set_option", "spade_launch_count", "spade_last_call_stages",
-                    "spade_status_string", "spade_last_error"]
+                    "spade_status_string", "spade_last_error", "spade_layer_assign", "spade_build_layered",
+                    "spade_join_count_layered", "spade_layered_info", "spade_layered_free"]
 
 
 def _check(rc: int, what: str):
@@ -289,6 +300,89 @@ class Canvas:
             self.close()
         except Exception:
             pass
+
+
+class LayeredCanvas:
+    """The paper's layer index (spade_build_layered): the polygons split
+    into layers of mutually non-intersecting polygons (greedy colouring of the closed-intersection
+    self-join), one canvas and one probe pass per layer.  The alternative to the owner sets of a
+    single Canvas, kept for comparison; polygons must be valid (as for join_polygons)."""
+
+    def __init__(self, polys, log2_pixel: int = -1, max_dim: int = 4096, stream=None):
+        torch = _torch()
+        lib = load()
+        self.device = torch.device("cuda", torch.cuda.current_device())
+        ring_xy = _dev(polys["ring_xy"], torch.int32, 2)
+        ring_off = _dev(polys["ring_off"], torch.int64)
+        poly_ring_off = _dev(polys["poly_ring_off"], torch.int64)
+        self.num_polys = int(poly_ring_off.numel()) - 1
+        prm = CanvasParams(log2_pixel, max_dim, 0)
+        h = ctypes.c_void_p()
+        rc = lib.spade_build_layered(ctypes.c_void_p(ring_xy.data_ptr()), ctypes.c_void_p(ring_off.data_ptr()),
+                                     ctypes.c_void_p(poly_ring_off.data_ptr()), self.num_polys, ctypes.byref(prm),
+                                     _stream(stream), ctypes.byref(h))
+        _check(rc, "spade_build_layered")
+        self._h, self._lib = h, lib
+
+    @property
+    def handle(self):
+        return self._h
+
+    @property
+    def num_layers(self) -> int:
+        L = ctypes.c_int32()
+        _check(self._lib.spade_layered_info(self._h, ctypes.byref(L), None), "spade_layered_info")
+        return L.value
+
+    def layer_of(self):
+        """numpy int32[P]: the layer of every polygon."""
+        import numpy as np
+        out = np.empty(self.num_polys, dtype=np.int32)
+        L = ctypes.c_int32()
+        _check(self._lib.spade_layered_info(self._h, ctypes.byref(L), out.ctypes.data_as(ctypes.c_void_p)),
+               "spade_layered_info")
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.spade_layered_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def join_count_layered(layered: LayeredCanvas, xy, counts=None, stream=None):
+    """Per-polygon COUNT over a layered canvas (spade_join_count_layered: one pass per layer);
+    accumulates into `counts` if given."""
+    torch = _torch()
+    xy, n = _points(xy, layered.device)
+    if counts is None:
+        counts = torch.zeros(layered.num_polys, dtype=torch.int64, device=layered.device)
+    _dev_out(counts, torch.int64, layered.num_polys, "counts", layered.device)
+    rc = load().spade_join_count_layered(layered.handle, ctypes.c_void_p(xy.data_ptr()), n,
+                                         ctypes.c_void_p(counts.data_ptr()), _stream(stream))
+    _check(rc, "spade_join_count_layered")
+    return counts
+
+
+def layer_assign(pair_a, pair_b, num_polys: int):
+    """Greedy layer colouring of a conflict graph (spade_layer_assign, host only): numpy int32
+    layer_of[num_polys] and the number of layers."""
+    import numpy as np
+    a = np.ascontiguousarray(pair_a, dtype=np.int32)
+    b = np.ascontiguousarray(pair_b, dtype=np.int32)
+    if a.shape != b.shape:
+        raise ValueError("layer_assign: pair arrays differ in length")
+    out = np.empty(max(num_polys, 0), dtype=np.int32)
+    L = ctypes.c_int32()
+    rc = load().spade_layer_assign(a.ctypes.data_as(ctypes.c_void_p), b.ctypes.data_as(ctypes.c_void_p), len(a),
+                                   num_polys, out.ctypes.data_as(ctypes.c_void_p), ctypes.byref(L))
+    _check(rc, "spade_layer_assign")
+    return out, L.value
 
 
 def join_polygons(polys1, polys2, capacity: int | None = None, max_dim: int = 4096, log2_pixel: int = -1,

@@ -8,7 +8,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libspade.so")
-SOURCES = ["spade_api.cu", "canvas_build.cu", "probe.cu", "knn.cu", "polygon_join.cu"]
+SOURCES = ["spade_api.cu", "canvas_build.cu", "probe.cu", "knn.cu", "polygon_join.cu", "layers.cu"]
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
               "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-Xptxas", "-v"]
 

@@ -654,7 +654,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   unsigned int* myhist = hist + (lane & (prm.hcopies - 1));
   __shared__ unsigned int s_dfill;              // deferred entries reserved by this CTA
   __shared__ int s_qn[kNW];                     // QUEUE: per-warp queue fill
-  QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? prm.hcopies * (P + 1) * 4 : MODE == kCountGlobal ? prm.cache_slots * 8 : 0)) +
+  // (the histogram's size rounded up to 16 B: the queue after it holds 8-B entries)
+  QEntry* wq = (QEntry*)(rest + (MODE == kCountSmem ? (prm.hcopies * (P + 1) * 4 + 15u) & ~15u : MODE == kCountGlobal ? prm.cache_slots * 8 : 0)) +
                warp * kQCap;
   uint32_t* wqi = (MODE == kCountSmem || MODE == kCountGlobal ? (uint32_t*)wq - warp * kQCap * 2 : (uint32_t*)rest) +
                   warp * kQCap;                                   // SELECT/PAIRS queue, TMA COUNT queue
@@ -1949,6 +1950,8 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   // boundary points tested in the loop (warp queues) when those fit too, else deferred
   const size_t tiles = tiles_bytes_for(c->d.Wc, c->d.Hc);
   const size_t one = (size_t)(c->d.num_polys + 1) * 4;
+  // shared memory of hc histogram copies, rounded up to 16 B (what follows is 8- or 16-B aligned)
+  auto hb = [&](uint32_t hc) { return ((size_t)hc * one + 15) & ~(size_t)15; };
   const size_t queue = queue_bytes(kCountSmem);
   const int force_defer = options().defer, force_global = options().count_global;
   // Mostly-mixed canvases whose only shared-memory histogram option is a single copy filling
@@ -1962,16 +1965,16 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
     if (options().pipe_notile && c->mixed_tile_frac >= 0.999 && !c->d.compact && !force_global) {
       const size_t ring2 = pipe_ring_bytes(kPipeNoTileD);
       for (uint32_t hc = 8; hc >= 1; hc >>= 1)
-        if (((hc * one + 15) & ~(size_t)15) + ring2 <= kPipeSmem) {
+        if (((hb(hc) + 15) & ~(size_t)15) + ring2 <= kPipeSmem) {
           p.hcopies = hc;
-          return launch_layout<kCountSmem, 0, 2>(c, (const int2*)xy, n, p, hc * one, st);
+          return launch_layout<kCountSmem, 0, 2>(c, (const int2*)xy, n, p, hb(hc), st);
         }
     }
     const size_t ring = pipe_ring_bytes();
     for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {
-      if (tiles + ((hc * one + 15) & ~(size_t)15) + ring <= kPipeSmem) {
+      if (tiles + ((hb(hc) + 15) & ~(size_t)15) + ring <= kPipeSmem) {
         p.hcopies = hc;
-        return launch_layout<kCountSmem, 0, 1>(c, (const int2*)xy, n, p, hc * one, st);
+        return launch_layout<kCountSmem, 0, 1>(c, (const int2*)xy, n, p, hb(hc), st);
       }
     }
     uint32_t slots = 0;
@@ -1989,28 +1992,28 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   const uint32_t hmax = (uint32_t)options().hist_copies_max;
   const int idxq = options().idx_queue;
   for (uint32_t hc = hmax; hc >= 1 && !force_global; hc >>= 1) {
-    if (!force_defer && idxq != 1 && tiles + hc * one + queue <= kSmemSoft) {
+    if (!force_defer && idxq != 1 && tiles + hb(hc) + queue <= kSmemSoft) {
       p.hcopies = hc;
       // A/B option "tma": the same launch with the point stream staged by TMA (+33 KB of stages)
       if (options().tma) {
         // the TMA variant (index queue + 33 KB of stages) with as many histogram copies as fit
         for (uint32_t ht = hc; ht >= 1; ht >>= 1)
-          if (tiles + ht * one + queue_bytes(kCountSmem, 2) + 128 + (size_t)kNW * 1032 <= kSmemSoft + options().tma_slack_kb * 1024) {
+          if (tiles + hb(ht) + queue_bytes(kCountSmem, 2) + 128 + (size_t)kNW * 1032 <= kSmemSoft + options().tma_slack_kb * 1024) {
             p.hcopies = ht;
-            return launch_layout<kCountSmem, 2>(c, (const int2*)xy, n, p, ht * one, st);
+            return launch_layout<kCountSmem, 2>(c, (const int2*)xy, n, p, hb(ht), st);
           }
       }
-      return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hc * one, st);
+      return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hb(hc), st);
     }
-    if (!force_defer && idxq != 0 && tiles + hc * one + queue_bytes(kCountSmem, 3) <= kSmemSoft) {
+    if (!force_defer && idxq != 0 && tiles + hb(hc) + queue_bytes(kCountSmem, 3) <= kSmemSoft) {
       p.hcopies = hc;
-      return launch_layout<kCountSmem, 3>(c, (const int2*)xy, n, p, hc * one, st);
+      return launch_layout<kCountSmem, 3>(c, (const int2*)xy, n, p, hb(hc), st);
     }
   }
   for (uint32_t hc = 8; hc >= 1 && !force_global; hc >>= 1) {
-    if (tiles + hc * one <= kSmemSoft || (hc == 1 && tiles + one <= 227 * 1024)) {
+    if (tiles + hb(hc) <= kSmemSoft || (hc == 1 && tiles + one <= 227 * 1024)) {
       p.hcopies = hc;
-      return launch_layout<kCountSmem>(c, (const int2*)xy, n, p, hc * one, st);
+      return launch_layout<kCountSmem>(c, (const int2*)xy, n, p, hb(hc), st);
     }
   }
   // global counts with a shared-memory count cache in the space the tiles leave

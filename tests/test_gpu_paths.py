@@ -57,6 +57,8 @@ COUNT_PATHS = [
     {"hist_copies_max": 8, "idx_queue": 0},
     {"hist_copies_max": 1, "idx_queue": 1},
     {"hist_copies_max": 16, "multi_agg": 0},
+    {"hist_copies_max": 1},                         # an odd-sized histogram before the 8-B point queue
+    {"hist_copies_max": 1, "k_agg": 1},
 ]
 
 
