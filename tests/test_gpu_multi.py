@@ -4,7 +4,8 @@
   arrays hash equal, on any device) and sensitive (one moved vertex changes it).
 * The NCCL path: min(8, device_count) ranks each build the canvas, compare checksums, COUNT their
   contiguous shard through the CUDA path and all_reduce; every rank must hold the single-rank
-  counts, PAIRS stay sharded with global ids by default and gather exactly on request.  On a
+  counts, PAIRS stay sharded with global ids by default and gather exactly on request, and kNN
+  across the shards (default CUDA step functions) equals the single-device kNN.  On a
   one-GPU box this runs as a one-rank NCCL group (the collectives execute on the device, with
   nothing to exchange); the multi-rank exchange itself is covered there by the gloo tests.
 """
@@ -84,7 +85,10 @@ def _nccl_worker(rank, world, port, out):
         pt, pl = sd.join_pairs_distributed(cv, xy, a)             # sharded (default)
         sharded_ok = bool(pt.numel() == b - a and int(pt.min()) >= a and int(pt.max()) < b)
         g = sd.join_pairs_distributed(cv, xy, a, gather=True, dst=0)
-        res = {"agree": agree, "counts": counts.cpu().numpy().tolist(), "sharded_ok": sharded_ok}
+        # kNN across the shards with the default (CUDA) step functions
+        ki, kd = sd.knn_distributed(xy, (8_400_000, 8_300_000), 50, a)
+        res = {"agree": agree, "counts": counts.cpu().numpy().tolist(), "sharded_ok": sharded_ok,
+               "knn": (ki.cpu().numpy(), kd.cpu().numpy())}
         if rank == 0:
             res["gathered"] = (g[0].cpu().numpy(), g[1].cpu().numpy())
         out[rank] = res
@@ -107,6 +111,11 @@ def test_nccl_count_pairs_and_checksums(spade):
         assert out[r]["agree"]
         assert out[r]["sharded_ok"]
         np.testing.assert_array_equal(np.array(out[r]["counts"]), ref)
+    xy_all = gen.points_device(w.points, w.point_seed, 0, N)
+    ri, rd = spade.knn(xy_all, (8_400_000, 8_300_000), 50)
+    for r in range(world):
+        np.testing.assert_array_equal(out[r]["knn"][0], ri.cpu().numpy())
+        np.testing.assert_array_equal(out[r]["knn"][1], rd.cpu().numpy())
     gpt, gpl = out[0]["gathered"]
     assert len(gpt) == N and len(np.unique(gpt)) == N
     np.testing.assert_array_equal(np.bincount(gpl, minlength=len(ref)), ref)
