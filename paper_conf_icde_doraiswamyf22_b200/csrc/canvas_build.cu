@@ -17,6 +17,7 @@
 //          cu(X, py) ^ cr(X, py) ^ cr(px, py))
 // where cr / cu are the half-open rightward / upward ray tests (perturbation reading of C1).
 #include <cub/cub.cuh>
+#include <thrust/iterator/transform_iterator.h>
 #include <nvtx3/nvToolsExt.h>
 #include <vector>
 #include <algorithm>
@@ -1127,8 +1128,8 @@ static int build_any(int kind, const int32_t* ring_xy, const int64_t* ring_off, 
   if (NB > 0) {
     LAUNCH(k_kset<0>, NB, NB, pix_of, g, corner, csets, crng, mbeg, mcnt, run_seg, run_mask,
            pbeg, pcnt, rec_polys, ksize, nullptr, nullptr, nullptr, kind);
-    cub::TransformInputIterator<int64_t, BigSize, const int32_t*> it_sz(ksize, BigSize());
-    cub::TransformInputIterator<int32_t, BigFlag, const int32_t*> it_b(ksize, BigFlag());
+    thrust::transform_iterator<BigSize, const int32_t*, int64_t, int64_t> it_sz(ksize, BigSize());
+    thrust::transform_iterator<BigFlag, const int32_t*, int32_t, int32_t> it_b(ksize, BigFlag());
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, it_sz, koff, NB, st); }), "scan K");
     TRYF(cub_call(tmp, [&](void* t, size_t& sz) { return cub::DeviceScan::ExclusiveSum(t, sz, it_b, kidx, NB, st); }), "scan K idx");
     int64_t last_off = 0; int32_t last_sz = 0, last_idx = 0;

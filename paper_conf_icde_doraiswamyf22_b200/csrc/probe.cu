@@ -140,7 +140,6 @@ __device__ __forceinline__ uint32_t rec_of_point(const CanvasDev* __restrict__ c
 struct U4 {
   uint32_t c[4];
   __device__ __forceinline__ uint32_t& operator[](int i) { return c[i]; }
-  __device__ __forceinline__ uint32_t operator[](int i) const { return c[i]; }
 };
 
 // Output side of a launch (what the sinks write).
@@ -695,7 +694,7 @@ __global__ void __launch_bounds__(kT, 1) k_probe(const __grid_constant__ Params 
   const uint32_t minx = (uint32_t)cv.minx, miny = (uint32_t)cv.miny;
   const uint32_t sb = (uint32_t)(cv.s + cv.b), s = (uint32_t)cv.s, Wc = (uint32_t)cv.Wc, W = (uint32_t)cv.W;
   const uint32_t Hc = (uint32_t)cv.Hc, Wc1 = Wc + 1u;
-  const uint32_t b = (uint32_t)cv.b, bm = (1u << cv.b) - 1u, mixmin = cv.mix_min;
+  const uint32_t bm = (1u << cv.b) - 1u, mixmin = cv.mix_min;
   const int32_t* __restrict__ finep = COMPACT == 1 ? cv.cfine : cv.fine;
   const uint16_t* __restrict__ f16p = cv.fine16;
   auto load_batch = [&](Vec4& v, uint32_t base) {
@@ -1131,7 +1130,8 @@ __global__ void __launch_bounds__(kT, 1) k_probe_pipe(const __grid_constant__ Pa
   int32_t* ring = (int32_t*)(rest + ((sink_bytes + 15) & ~(size_t)15));   // [D][NPT][T] pixel values
   __shared__ unsigned int s_dfill;
 
-  for (uint32_t i = tid; i < tbytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
+  if constexpr (!NOTILE)
+    for (uint32_t i = tid; i < tbytes / 16; i += T) ((int4*)tiles)[i] = __ldg((const int4*)cv.coarse + i);
   if (MODE == kCountSmem)
     for (uint32_t i = tid; i < prm.hcopies * (P + 1); i += T) hist[i] = 0u;
   if (MODE == kCountGlobal)
