@@ -30,8 +30,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     # the builder's ~1 MB module, not the probe's ~16 MB (C5 cold build 2.0 s -> see DESIGN.md).
     # probe.cu keeps separate compilation (-dc + its own device link: its register allocation
     # was tuned that way).
-    objs = []
-    for s in srcs:
+    def compile_one(s):
         o = os.path.join(CSRC, os.path.basename(s).replace(".cu", ".o"))
         rdc = os.path.basename(s) == "probe.cu"
         cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-dc" if rdc else "-c", "-o", o, s]
@@ -40,14 +39,22 @@ def build(force: bool = False, verbose: bool = False) -> str:
             raise RuntimeError(f"nvcc failed for {s}:\n{r.stdout}\n{r.stderr}")
         if verbose:
             print(r.stderr)
-        objs.append(o)
+        out = [o]
         if rdc:
             dl = o.replace(".o", "_dlink.o")
             cmd = ["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-Xcompiler", "-fPIC", "-dlink", "-o", dl, o]
             r = subprocess.run(cmd, capture_output=True, text=True)
             if r.returncode != 0:
                 raise RuntimeError(f"device link failed for {s}:\n{r.stdout}\n{r.stderr}")
-            objs.append(dl)
+            out.append(dl)
+        return out
+
+    # the translation units compile in parallel (probe.cu, the longest, first)
+    from concurrent.futures import ThreadPoolExecutor
+    order = sorted(srcs, key=lambda s: os.path.basename(s) != "probe.cu")
+    with ThreadPoolExecutor(max_workers=min(len(order), os.cpu_count() or 1)) as ex:
+        done = dict(zip(order, ex.map(compile_one, order)))
+    objs = [o for s in srcs for o in done[s]]
     cmd = ["g++", "-shared", "-fPIC", "-o", LIB, *objs, "-L/usr/local/cuda/lib64", "-lcudadevrt", "-lcudart_static", "-lrt", "-lpthread", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
