@@ -1707,8 +1707,18 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
   if constexpr (PIPE == 2) kern = k_probe_pipe<MODE, COMPACT, KIND, 2>;
   else if constexpr (PIPE != 0) kern = k_probe_pipe<MODE, COMPACT, KIND, 1>;
   else kern = k_probe<MODE, COMPACT, QUEUE, KIND>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
+  // (the attribute is set when it grows, once per device and instantiation: a driver call per
+  // probe call showed as host latency on short calls)
+  static std::atomic<int> smem_set[16];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  cudaError_t e = cudaSuccess;
+  if (smem_set[dev & 15].load(std::memory_order_relaxed) < (int)smem) {
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return check_cuda(e, "probe smem attribute");
+    int cur = smem_set[dev & 15].load();
+    while (cur < (int)smem && !smem_set[dev & 15].compare_exchange_weak(cur, (int)smem)) {}
+  }
   const int sms = device_sm_count();
   keep_pool_memory();
   g_stages.begin(st);
@@ -1888,7 +1898,11 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
       k_fixup<<<1, kFixT, 0, st>>>(p.o.holes, grid * kNW, p.o.total, p.o.cap, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
       count_launch();
       const int msm = (int)(sizeof(long long) * (2 * kMaxHoles + 1));
-      cudaFuncSetAttribute(k_move<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, msm);
+      static std::atomic<uint32_t> move_set{0};          // (bit per device: set once)
+      if (!(move_set.load(std::memory_order_relaxed) & (1u << (dev & 15)))) {
+        cudaFuncSetAttribute(k_move<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, msm);
+        move_set.fetch_or(1u << (dev & 15));
+      }
       k_move<MODE><<<sms, 1024, msm, st>>>(p.o, fix_ds, fix_dp, fix_ss, fix_sp, fix_meta);
       count_launch();
       e = cudaGetLastError();

@@ -100,11 +100,19 @@ int run_with_capacity(int64_t capacity, int64_t* n_out, cudaStream_t st, const c
   if (e != cudaSuccess) return check_cuda(e, fn);
   e = cudaMemsetAsync(d_total, 0, sizeof(unsigned long long), st);
   int rc = e == cudaSuccess ? launch(d_total) : check_cuda(e, fn);
+  // the count comes back through a pinned word (one per thread, allocated once): a DMA instead of a
+  // staged copy into pageable memory
+  static thread_local unsigned long long* pinned = nullptr;
+  if (!pinned && cudaMallocHost((void**)&pinned, sizeof(unsigned long long)) != cudaSuccess) {
+    pinned = nullptr;
+    cudaGetLastError();
+  }
   unsigned long long h = 0;
   if (rc == SPADE_OK) {
-    e = cudaMemcpyAsync(&h, d_total, sizeof(h), cudaMemcpyDeviceToHost, st);
+    e = cudaMemcpyAsync(pinned ? pinned : &h, d_total, sizeof(h), cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     if (e != cudaSuccess) rc = check_cuda(e, fn);
+    else if (pinned) h = *pinned;
   }
   cudaFreeAsync(d_total, st);
   if (rc != SPADE_OK) return rc;
