@@ -323,9 +323,11 @@ SPADE_API int spade_knn(const int32_t* xy, int64_t n, int64_t point_id_base, int
  *                  (measured slower on C5: 13.6 vs 11.2 ms; A/B only)
  *   "hist_copies_max"  16 (default), 32, 8, 4, 2, 1: most copies of the COUNT shared-memory
  *                  histogram (copy = lane mod copies; 32 = one bank per lane, no conflicts)
- *   "idx_queue"    0 (default) / 1 / -1 (when it makes room for more histogram copies): COUNT
- *                  in-loop queues hold 4-B point indices instead of 8-B points (A/B: C3 with
- *                  32 copies and index queues 1.95 ms vs 1.73 ms with 16 copies and point queues)
+ *   "idx_queue"    -1 (default) / 0 / 1: COUNT in-loop queues of 4-B point indices instead of 8-B
+ *                  points: -1 = for K-aggregated (overlap-heavy) canvases when that keeps the CTA
+ *                  at or below the 164 KB shared-memory step (a larger L1 for their record walks:
+ *                  ov 29.2 -> 27.1 ms), point queues otherwise (C3 1.69 vs 1.88 ms with index
+ *                  queues); 0 = always point queues; 1 = index queues whenever they fit
  *   "stage_events" 0 (default) / 1: record CUDA events between the stages of every COUNT / SELECT /
  *                  PAIRS call on its stream (synchronises once per sub-launch to read them; see
  *                  spade_last_call_stages)

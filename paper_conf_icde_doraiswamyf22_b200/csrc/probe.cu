@@ -47,6 +47,7 @@ constexpr int kNPT = 4;            // points per thread per batch (one 256-bit v
 // Shared memory above ~196 KB per CTA shrinks the L1 carve-out below ~60 KB and costs ~35%
 // (measured on B200); the histogram copies are chosen to stay under it.
 constexpr size_t kSmemSoft = 196 * 1024;
+constexpr size_t kSmemL1Step = 164 * 1024;   // the next carve-out step down (L1 60 -> ~92 KB)
 
 struct alignas(32) Vec4 { int4 a, b; };   // 4 points
 
@@ -1694,6 +1695,13 @@ struct ScratchGuard {
   ~ScratchGuard() { if (p) cudaFreeAsync(p, st); }
 };
 
+// COUNT with K aggregation (boundary points counted per record for the corner set K): heavily
+// overlapping polygon sets
+bool kagg_for(const spade_canvas* c) {
+  const int o = options().k_agg;
+  return c->num_runs > 0 && (o == 1 || (o < 0 && 2 * c->num_set_entries > c->num_records));
+}
+
 template <int MODE, int COMPACT, int QUEUE, int KIND, int PIPE = 0>
 int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base, size_t extra_smem, cudaStream_t st) {
   const size_t base_smem = PIPE == 2 ? ((extra_smem + 15) & ~(size_t)15) + pipe_ring_bytes(kPipeNoTileD)
@@ -1737,9 +1745,7 @@ int launch(const spade_canvas* c, const int2* xy, int64_t n, const Params& base,
   }
   // COUNT over heavily overlapping polygons (owner sets much larger than one polygon on average):
   // boundary points counted per record for the term set K + per-point parity deltas
-  const int kagg_opt = options().k_agg;
-  const bool kagg = kCnt && c->num_runs > 0 &&
-                    (kagg_opt == 1 || (kagg_opt < 0 && 2 * c->num_set_entries > c->num_records));
+  const bool kagg = kCnt && kagg_for(c);
   unsigned int* kcnt = nullptr;
   if (options().debug_defer)
     fprintf(stderr, "[spade] records %lld (boundary %lld), set entries %lld, k_agg %d\n", (long long)c->num_records,
@@ -2005,6 +2011,17 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
   // 4-B point indices (the drain re-reads its points) makes room for them beside big tile grids.
   const uint32_t hmax = (uint32_t)options().hist_copies_max;
   const int idxq = options().idx_queue;
+  // Overlap-heavy (K-aggregated) canvases: the exact tests walk records for a third of the points,
+  // and the L1 that serves those walks grows in steps with the shared memory left free (the
+  // carve-out); auto (-1) takes 4-B index queues and as many histogram copies as keep the CTA at
+  // or below the 164 KB step (measured: ov 29.2 -> 27.1 ms; C3 and C4, which re-read few queued
+  // points but gather more, are faster with point queues and stay on them).
+  if (idxq < 0 && !force_defer && !force_global && kagg_for(c))
+    for (uint32_t hc = hmax; hc >= 1; hc >>= 1)
+      if (tiles + hb(hc) + queue_bytes(kCountSmem, 3) <= kSmemL1Step) {
+        p.hcopies = hc;
+        return launch_layout<kCountSmem, 3>(c, (const int2*)xy, n, p, hb(hc), st);
+      }
   for (uint32_t hc = hmax; hc >= 1 && !force_global; hc >>= 1) {
     if (!force_defer && idxq != 1 && tiles + hb(hc) + queue <= kSmemSoft) {
       p.hcopies = hc;
@@ -2019,7 +2036,7 @@ int launch_count(const spade_canvas* c, const int32_t* xy, int64_t n, int64_t* c
       }
       return launch_layout<kCountSmem, 1>(c, (const int2*)xy, n, p, hb(hc), st);
     }
-    if (!force_defer && idxq != 0 && tiles + hb(hc) + queue_bytes(kCountSmem, 3) <= kSmemSoft) {
+    if (!force_defer && idxq == 1 && tiles + hb(hc) + queue_bytes(kCountSmem, 3) <= kSmemSoft) {
       p.hcopies = hc;
       return launch_layout<kCountSmem, 3>(c, (const int2*)xy, n, p, hb(hc), st);
     }

@@ -138,7 +138,7 @@ Options& options() {
                    (int64_t)1 << 25, (1ll << 31) - 64, 4096, env_int("SPADE_FINE16", 1),
                    env_int("SPADE_STAGE_EVENTS", 0), env_int("SPADE_TMA", 0), env_int("SPADE_SMEM_PAD_KB", 0),
                    env_int("SPADE_TMA_SLACK_KB", 0), env_int("SPADE_PIPE_NOTILE", 0),
-                   env_int("SPADE_HIST_COPIES_MAX", 16), env_int("SPADE_IDX_QUEUE", 0)};
+                   env_int("SPADE_HIST_COPIES_MAX", 16), env_int("SPADE_IDX_QUEUE", -1)};
   return o;
 }
 }  // namespace spade

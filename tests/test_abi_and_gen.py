@@ -76,7 +76,7 @@ def test_set_option_validates_names_and_values_without_a_gpu():
     lib = sp.load()
     for name, value in [("defer", 1), ("defer", 0), ("coop", 8), ("coop", -1), ("cache_slots", 4096),
                         ("cache_slots", 16384), ("count_global", 0), ("global_queue", 0), ("debug_defer", 0), ("pipe", 1), ("pipe", -1),
-                        ("hist_copies_max", 1), ("hist_copies_max", 16), ("idx_queue", 1), ("idx_queue", 0)]:
+                        ("hist_copies_max", 1), ("hist_copies_max", 16), ("idx_queue", 1), ("idx_queue", 0), ("idx_queue", -1)]:
         assert lib.spade_set_option(name.encode(), value) == 0, name
     for name, value in [("coop", 3), ("cache_slots", 1000), ("defer", 2), ("pipe", 2), ("nope", 0),
                         ("hist_copies_max", 64), ("hist_copies_max", 12), ("idx_queue", 2)]:

@@ -18,7 +18,7 @@ pytestmark = pytest.mark.gpu
 
 DEFAULTS = {"defer": 0, "count_global": 0, "global_queue": 0, "cache_slots": 4096, "coop": 0, "pipe": -1,
             "defer_xy": 0, "multi_agg": 1, "k_agg": -1, "tma": 0, "fine16": 1, "pipe_notile": 0,
-            "hist_copies_max": 16, "idx_queue": 0}
+            "hist_copies_max": 16, "idx_queue": -1}
 
 COUNT_PATHS = [
     {},
