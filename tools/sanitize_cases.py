@@ -106,6 +106,13 @@ def main():
         oa, ob = oracle.polygon_join(A, B)
         assert np.array_equal(a.cpu().numpy(), oa) and np.array_equal(b.cpu().numpy(), ob)
         n_checks += 1
+    # the layer index (one canvas and one pass per layer) over an overlapping valid set
+    from tests.helpers import lattice
+    xl = lattice(-2, -2, 62, 62) * 16
+    lc = sp.LayeredCanvas(A, max_dim=256)
+    got = sp.join_count_layered(lc, torch.as_tensor(xl.astype(np.int32)).cuda()).cpu().numpy()
+    assert np.array_equal(got, oracle.join_count(xl.astype(np.int32), A))
+    n_checks += 1
     torch.cuda.synchronize()
     print(f"sanitize cases: {n_checks} checks ok, {sp.launch_count()} kernel launches", flush=True)
 
